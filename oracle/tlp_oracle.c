@@ -1,0 +1,266 @@
+/*
+ * tlp_oracle.c -- plain, slow, single-threaded fp64 CPU oracle for the
+ * TLPGNN graph-convolution (neighbor aggregation) hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load this library.
+ * It shares no code, header, table or helper with the CUDA path
+ * (paper_conf_hpdc_fujh22_b200/csrc), and it never includes include/tlp.h.
+ *
+ * Citations: "P:<line>" = /root/reference/PAPER.md line (HPDC'22 TLPGNN),
+ * "c2 #k" = SURVEY.md section 8(c) reading k, restated in DESIGN.md.
+ *
+ * What it computes (Eq. 1: a_u = (+)_{v in N(u)} psi(h_u, e_vu, h_v)),
+ * for a destination row v whose in-edges are e in [rowptr[v], rowptr[v+1]) with
+ * source u = colidx[e] (the pull / in-edge CSR of Fig. 7):
+ *
+ *   GCN  ("weighted based on degree", "weighted sum";
+ *         norm modes are c2 #1, #3, #4):
+ *        Y[v,f] = c_in[v] * sum_e w_e * c_out[u] * X[u,f]
+ *   GIN  (Xu et al. [51]; c2 #2, #5, #9):
+ *        Y[v,f] = (1+eps) * X[row_offset+v, f] + sum_e w_e * X[u,f]
+ *   GAT  (attention coefficient per edge, softmax over all the
+ *         attentions of v, aggregate weighted by the softmax; Velickovic [43];
+ *         c2 #5-#8): plain TWO-PASS softmax, deliberately not the online form.
+ *
+ * Alongside every output it returns the bound term A[v,f] = sum |terms| used by
+ * the parity criterion |Y_gpu - Y| <= 1e-5 * A + 1e-6 (BASELINE.json north star).
+ *
+ * Arithmetic: every fp32 input is promoted to double; sums run in CSR order
+ * in double; exp() is libm's.  No blocking, fusion or reordering.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define ORACLE_NORM_NONE 0
+#define ORACLE_NORM_RIGHT 1
+#define ORACLE_NORM_BOTH 2
+
+/* ---- structure ---------------------------------------------------------- */
+
+/* In-degree of each destination row: number of entries in its CSR range
+ * (c2 #3: unweighted edge counts; multi-edges and self-loops count). */
+void oracle_in_degree(int64_t n_dst, const int64_t *rowptr, int32_t *in_deg)
+{
+    for (int64_t v = 0; v < n_dst; ++v)
+        in_deg[v] = (int32_t)(rowptr[v + 1] - rowptr[v]);
+}
+
+/* Out-degree of each source vertex: number of edges whose source is u
+ * (c2 #3).  A plain count over colidx. */
+void oracle_out_degree(int64_t n_src, int64_t nnz, const int32_t *colidx,
+                       int32_t *out_deg)
+{
+    for (int64_t u = 0; u < n_src; ++u)
+        out_deg[u] = 0;
+    for (int64_t e = 0; e < nnz; ++e)
+        out_deg[colidx[e]] += 1;
+}
+
+/* CSR validity (SURVEY 8(b) create contract): rowptr[0]=0, monotone,
+ * rowptr[n]=nnz, 0 <= colidx < n_src.  Returns 0 if valid, else 1. */
+int oracle_csr_invalid(int64_t n_dst, int64_t n_src, int64_t nnz,
+                       const int64_t *rowptr, const int32_t *colidx)
+{
+    if (rowptr[0] != 0)
+        return 1;
+    for (int64_t v = 0; v < n_dst; ++v)
+        if (rowptr[v + 1] < rowptr[v])
+            return 1;
+    if (rowptr[n_dst] != nnz)
+        return 1;
+    for (int64_t e = 0; e < nnz; ++e)
+        if (colidx[e] < 0 || (int64_t)colidx[e] >= n_src)
+            return 1;
+    return 0;
+}
+
+/* Destination-row partition balanced by edge count (north star: "destination-
+ * row ranges balanced by edge count"; c1 "Partition", c2 #16):
+ *   b_0 = 0, b_P = N,
+ *   b_k = min{ r in [0,N] : rowptr[r] >= floor(k*E/P) }   for 0 < k < P.
+ * Written as a linear scan (obviously correct, O(P*N)). */
+void oracle_partition(int64_t n, const int64_t *rowptr, int parts,
+                      int64_t *bounds)
+{
+    int64_t nnz = rowptr[n];
+    bounds[0] = 0;
+    for (int k = 1; k < parts; ++k) {
+        int64_t target = ((int64_t)k * nnz) / parts; /* floor for nnz >= 0 */
+        int64_t r = 0;
+        while (r < n && rowptr[r] < target)
+            ++r;
+        bounds[k] = r;
+    }
+    bounds[parts] = n;
+}
+
+/* ---- aggregations -------------------------------------------------------- */
+
+/* The destination rows to evaluate: rows[i] if rows != NULL, else i. */
+static int64_t pick_row(const int64_t *rows, int64_t i)
+{
+    return rows ? rows[i] : i;
+}
+
+/* GCN (c1 row "GCN").  norm: 0 NONE (c_in=c_out=1), 1 RIGHT (c_in = 1/max(in_deg,1),
+ * c_out = 1), 2 BOTH (c_in = 1/sqrt(max(in_deg,1)), c_out = 1/sqrt(max(out_deg,1))),
+ * Kipf [26].  out_deg counts edges over the whole CSR given (c2 #3).
+ * ew may be NULL (w_e = 1); weights multiply, degrees stay unweighted (c2 #4).
+ * Outputs Y[i*F + f] and (if A != NULL) A[i*F + f] for i < n_rows.
+ * Returns 0, or -1 on bad arguments / allocation failure. */
+int oracle_gcn(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+               const int32_t *colidx, const float *ew, const float *X,
+               int64_t F, int64_t ldx, int norm, int64_t n_rows,
+               const int64_t *rows, double *Y, double *A)
+{
+    if (norm < 0 || norm > 2 || F < 0 || ldx < F)
+        return -1;
+    int64_t nnz = rowptr[n_dst];
+    int32_t *out_deg = NULL;
+    if (norm == ORACLE_NORM_BOTH) {
+        out_deg = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n_src > 0 ? n_src : 1));
+        if (!out_deg)
+            return -1;
+        oracle_out_degree(n_src, nnz, colidx, out_deg);
+    }
+    for (int64_t i = 0; i < n_rows; ++i) {
+        int64_t v = pick_row(rows, i);
+        int64_t deg = rowptr[v + 1] - rowptr[v];
+        double dclamp = (double)(deg > 1 ? deg : 1);
+        double c_in = 1.0;
+        if (norm == ORACLE_NORM_RIGHT)
+            c_in = 1.0 / dclamp;
+        else if (norm == ORACLE_NORM_BOTH)
+            c_in = 1.0 / sqrt(dclamp);
+        for (int64_t f = 0; f < F; ++f) {
+            double s = 0.0, a = 0.0;
+            for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e) {
+                int64_t u = colidx[e];
+                double w = ew ? (double)ew[e] : 1.0;
+                double c_out = 1.0;
+                if (norm == ORACLE_NORM_BOTH) {
+                    int32_t od = out_deg[u];
+                    c_out = 1.0 / sqrt((double)(od > 1 ? od : 1));
+                }
+                double term = w * c_out * (double)X[u * ldx + f];
+                s += term;
+                a += fabs(term);
+            }
+            Y[i * F + f] = c_in * s;
+            if (A)
+                A[i * F + f] = c_in * a;
+        }
+    }
+    free(out_deg);
+    return 0;
+}
+
+/* GIN (c1 row "GIN"): Y[v,f] = (1+eps) X[row_offset+v, f] + sum_e w_e X[u,f].
+ * The self row of destination v is X[row_offset + v] (row_offset = 0 for a
+ * whole graph, b_k for a row slice).  Requires row_offset + n_dst <= n_src. */
+int oracle_gin(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+               const int32_t *colidx, const float *ew, const float *X,
+               int64_t F, int64_t ldx, double eps, int64_t row_offset,
+               int64_t n_rows, const int64_t *rows, double *Y, double *A)
+{
+    if (F < 0 || ldx < F || row_offset < 0 || row_offset + n_dst > n_src)
+        return -1;
+    double self_w = 1.0 + eps;
+    for (int64_t i = 0; i < n_rows; ++i) {
+        int64_t v = pick_row(rows, i);
+        for (int64_t f = 0; f < F; ++f) {
+            double self = self_w * (double)X[(row_offset + v) * ldx + f];
+            double s = self, a = fabs(self);
+            for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e) {
+                int64_t u = colidx[e];
+                double w = ew ? (double)ew[e] : 1.0;
+                double term = w * (double)X[u * ldx + f];
+                s += term;
+                a += fabs(term);
+            }
+            Y[i * F + f] = s;
+            if (A)
+                A[i * F + f] = a;
+        }
+    }
+    return 0;
+}
+
+/* LeakyReLU, c2 #6: x >= 0 ? x : slope*x. */
+static double leaky_relu(double x, double slope)
+{
+    return x >= 0.0 ? x : slope * x;
+}
+
+/* GAT, single head (c1 row "GAT").  For destination v with
+ * in-degree d > 0:
+ *   t_e = el[u] + er[row_offset+v];  s_e = LeakyReLU(t_e, slope)
+ *   m = max_e s_e;  z = sum_e exp(s_e - m);  alpha_e = exp(s_e - m) / z
+ *   Y[v,f] = sum_e alpha_e X[u,f];  A[v,f] = sum_e alpha_e |X[u,f]|
+ * d = 0 gives Y = A = 0 (c2 #8).  Edge weights are not an input (c2 #5).
+ * If alpha_sum != NULL, alpha_sum[i] = sum_e alpha_e (pin P5), 0 for d = 0. */
+int oracle_gat(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+               const int32_t *colidx, const float *X, int64_t F, int64_t ldx,
+               const float *el, const float *er, double slope,
+               int64_t row_offset, int64_t n_rows, const int64_t *rows,
+               double *Y, double *A, double *alpha_sum)
+{
+    (void)n_src;
+    if (F < 0 || ldx < F || row_offset < 0)
+        return -1;
+    for (int64_t i = 0; i < n_rows; ++i) {
+        int64_t v = pick_row(rows, i);
+        int64_t e0 = rowptr[v], e1 = rowptr[v + 1];
+        int64_t d = e1 - e0;
+        if (d == 0) {
+            for (int64_t f = 0; f < F; ++f) {
+                Y[i * F + f] = 0.0;
+                if (A)
+                    A[i * F + f] = 0.0;
+            }
+            if (alpha_sum)
+                alpha_sum[i] = 0.0;
+            continue;
+        }
+        double *alpha = (double *)malloc(sizeof(double) * (size_t)d);
+        if (!alpha)
+            return -1;
+        /* pass 1: scores and their maximum */
+        double er_v = (double)er[row_offset + v];
+        double m = -INFINITY;
+        for (int64_t e = e0; e < e1; ++e) {
+            double s = leaky_relu((double)el[colidx[e]] + er_v, slope);
+            alpha[e - e0] = s;
+            if (s > m)
+                m = s;
+        }
+        /* pass 2: normaliser, then the softmax weights */
+        double z = 0.0;
+        for (int64_t k = 0; k < d; ++k)
+            z += exp(alpha[k] - m);
+        double asum = 0.0;
+        for (int64_t k = 0; k < d; ++k) {
+            alpha[k] = exp(alpha[k] - m) / z;
+            asum += alpha[k];
+        }
+        if (alpha_sum)
+            alpha_sum[i] = asum;
+        /* aggregation weighted by the softmax */
+        for (int64_t f = 0; f < F; ++f) {
+            double s = 0.0, a = 0.0;
+            for (int64_t e = e0; e < e1; ++e) {
+                double x = (double)X[(int64_t)colidx[e] * ldx + f];
+                s += alpha[e - e0] * x;
+                a += alpha[e - e0] * fabs(x);
+            }
+            Y[i * F + f] = s;
+            if (A)
+                A[i * F + f] = a;
+        }
+        free(alpha);
+    }
+    return 0;
+}
