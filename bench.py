@@ -1,0 +1,434 @@
+#!/usr/bin/env python
+"""Benchmark of the TLPGNN aggregation hot path on B200 (driver contract).
+
+A step = one pass of the whole hot path over the Reddit-shaped graph
+(BASELINE.json configs[2]: N = 232,965, E = 114,615,892, F = 602, ld = 604):
+GCN (BOTH norm) + GIN (eps 0.1) + GAT (slope 0.2), each ONE kernel launch of
+libtlp through the C ABI.  The graph handle (ingest/validate/degrees/plan,
+SURVEY 8(a) a1-a3) is created once before the timed region, as the structure
+is static across layers; its create time is reported separately.
+
+value = gather-model bytes of the step / device time (GB/s):
+  GCN per edge 4F + 4 (colidx) + 4 (c_out[u]); per row 4F (Y) + 8 (rowptr)
+  GIN per edge 4F + 4;                          per row 8F + 8 (self + Y)
+  GAT per edge 4F + 4 + 4 (el[u]);              per row 4F + 12 (Y, rowptr, er)
+N > 1 (torchrun): destination rows split by edge count, X replicated, every
+aggregation followed by the all-gather of Y rows (tlp_dist_*); total work is
+fixed ("strong" scaling); time = max over ranks.
+
+--impl reference: the fp64 oracle (oracle/, single-threaded C) timed on the
+host cores on a bounded row sample of the same workload -- the paper ships no
+code, so the oracle is this tier's reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "GCN/GAT aggregation ms & HBM GB/s vs 8 TB/s, Reddit-shaped, 1/2/4/8 B200"
+NOMINAL_HBM_GBS = 8000.0
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+OPS = ("gcn", "gin", "gat")
+
+
+# ------------------------------------------------------------------ bytes --
+
+def gather_bytes(op, n_rows, n_edges, F):
+    """Algorithmic (gather-model) bytes of one aggregation."""
+    if op == "gcn":
+        return n_edges * (4 * F + 8) + n_rows * (4 * F + 8)
+    if op == "gin":
+        return n_edges * (4 * F + 4) + n_rows * (8 * F + 8)
+    if op == "gat":
+        return n_edges * (4 * F + 8) + n_rows * (4 * F + 12)
+    raise ValueError(op)
+
+
+def peak_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            v = float(json.load(f)["hbm_gbs"])
+        return v, "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def load_traffic(workload):
+    """DRAM bytes per launch from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(workload, {})
+    except Exception:
+        return {}
+
+
+# ------------------------------------------------------------------ clocks --
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "--query-gpu=" + self.Q, "--format=csv,noheader,nounits",
+                 "-lms", "100", "-i", str(self.gpu)],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.t.join(timeout=2)
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx.append(float(parts[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx),
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- workload --
+
+WORKLOADS = {
+    "reddit": dict(graph="reddit", ops=OPS),
+    "products": dict(graph="products", ops=("gat",)),
+    "pubmed": dict(graph="pubmed", ops=("gat",)),
+    "cora": dict(graph="cora", ops=("gcn",)),
+}
+
+
+def workload_desc(name, cfg, E):
+    ops = "+".join({"gcn": "GCN(both)", "gin": "GIN(eps=0.1)", "gat": "GAT(slope=0.2)"}[o]
+                   for o in WORKLOADS[name]["ops"])
+    return f"{name}-shaped {ops}: N={cfg['n']} E={E} F={cfg['F']} ld={cfg['ld']}"
+
+
+def make_inputs(name, device):
+    import synth
+    cfg = synth.CONFIGS[WORKLOADS[name]["graph"]]
+    rp, ci = synth.dataset_graph(WORKLOADS[name]["graph"], device=device)
+    n = cfg["n"]
+    X = synth.dataset_features(WORKLOADS[name]["graph"], n)
+    el = synth.normal(n, 1000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
+    er = synth.normal(n, 2000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
+    return cfg, rp, ci, X, el, er
+
+
+# --------------------------------------------------------------- our arm ----
+
+def run_tlp(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_hpdc_fujh22_b200 as tlp
+    import synth
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    name = args.workload
+    ops = WORKLOADS[name]["ops"]
+    cfg, rp, ci, Xh, elh, erh = make_inputs(name, dev)
+    n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+    E = len(ci)
+    stream = torch.cuda.current_stream(dev)
+
+    rp_d = torch.from_numpy(rp).to(dev)
+    ci_d = torch.from_numpy(ci).to(dev)
+    comm = None
+    t0 = time.perf_counter()
+    if world > 1:
+        comm = tlp.comm_from_torch()
+        g = tlp.Graph.dist(comm, rp_d, ci_d)
+    else:
+        g = tlp.Graph(rp_d, ci_d)
+    torch.cuda.synchronize()
+    create_ms = (time.perf_counter() - t0) * 1e3
+    info = g.info
+    del ci_d
+    X = torch.from_numpy(Xh).to(dev)
+    el = torch.from_numpy(elh).to(dev)
+    er = torch.from_numpy(erh).to(dev)
+    Y = {op: torch.empty((n, ld), dtype=torch.float32, device=dev) for op in ops}
+
+    def launch(op, Xin=X, elv=el, erv=er):
+        if world > 1:
+            if op == "gcn":
+                tlp.tlp_dist_gcn_aggregate(g.handle, comm, Xin, Y[op], "both", F=F)
+            elif op == "gin":
+                tlp.tlp_dist_gin_aggregate(g.handle, comm, Xin, Y[op], synth.EPS, F=F)
+            else:
+                tlp.tlp_dist_gat_aggregate(g.handle, comm, Xin, Y[op], elv, erv, synth.SLOPE, F=F)
+        else:
+            if op == "gcn":
+                g.gcn(Xin, "both", Y=Y[op], F=F)
+            elif op == "gin":
+                g.gin(Xin, synth.EPS, Y=Y[op], F=F)
+            else:
+                g.gat(Xin, elv, erv, synth.SLOPE, Y=Y[op], F=F)
+
+    for _ in range(args.warmup):
+        for op in ops:
+            launch(op)
+    torch.cuda.synchronize()
+
+    # ---- device-resident timed region ----
+    ev = {op: [] for op in ops}
+    start, stop = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        start.record(stream)
+        for _ in range(args.steps):
+            for op in ops:
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                launch(op)
+                b.record(stream)
+                ev[op].append((a, b))
+        stop.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    total_ms = start.elapsed_time(stop)
+    op_ms = {op: [a.elapsed_time(b) for a, b in ev[op]] for op in ops}
+    t = torch.tensor([total_ms], device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        for op in ops:
+            tt = torch.tensor(op_ms[op], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            op_ms[op] = tt.tolist()
+    total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    step_bytes = sum(gather_bytes(op, n, E, F) for op in ops)
+    value = step_bytes / (ms_per_step * 1e-3) / 1e9
+
+    # ---- end to end through the public API with host buffers ----
+    e2e = None
+    if not args.no_e2e:
+        Xp = torch.from_numpy(Xh).pin_memory()
+        elp, erp = torch.from_numpy(elh).pin_memory(), torch.from_numpy(erh).pin_memory()
+        Yp = {op: torch.empty((n, ld), dtype=torch.float32).pin_memory() for op in ops}
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(args.steps):
+            X.copy_(Xp, non_blocking=True)
+            el.copy_(elp, non_blocking=True)
+            er.copy_(erp, non_blocking=True)
+            for op in ops:
+                launch(op)
+                Yp[op].copy_(Y[op], non_blocking=True)
+        b.record(stream)
+        torch.cuda.synchronize()
+        te = torch.tensor([a.elapsed_time(b)], device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e_ms = float(te.item()) / args.steps
+        h2d = Xp.numel() * 4 + elp.numel() * 4 + erp.numel() * 4
+        d2h = sum(Yp[op].numel() * 4 for op in ops)
+        e2e = {"value": round(step_bytes / (e2e_ms * 1e-3) / 1e9, 2), "unit": "GB/s",
+               "ms_per_step": round(e2e_ms, 3), "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h),
+               "note": "pinned host X/el/er -> device, 3 aggregations, Y -> pinned host, per step"}
+        # parity spot check of the end-to-end outputs (device copy vs host copy)
+        for op in ops:
+            assert torch.equal(Yp[op][:64].to(dev), Y[op][:64])
+
+    # ---- roofline of the dominant kernel ----
+    peak, peak_src = peak_hbm()
+    per_op = {}
+    for op in ops:
+        ms = statistics.mean(op_ms[op])
+        by = gather_bytes(op, n, E, F)
+        per_op[op] = {"ms_mean": round(ms, 4), "ms_median": round(statistics.median(op_ms[op]), 4),
+                      "gather_bytes": int(by), "gather_GBs": round(by / (ms * 1e-3) / 1e9, 1),
+                      "frac_of_8TBs": round(by / (ms * 1e-3) / 1e9 / NOMINAL_HBM_GBS, 4),
+                      "edges_x_features_per_s": float(E * F / (ms * 1e-3))}
+    dom = max(ops, key=lambda o: per_op[o]["ms_mean"])
+    traffic = load_traffic(name).get(dom)
+    achieved = per_op[dom]["gather_GBs"]
+    roofline = {"bound": "hbm", "kernel": f"k_agg ({dom})", "achieved": achieved,
+                "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4),
+                "traffic": traffic, "peak_source": peak_src,
+                "bytes_per_launch": per_op[dom]["gather_bytes"],
+                "bytes_model": "gather model: per edge 4F+4 colidx+4 coef/el; per row Y, rowptr (+self/er)"}
+
+    result = {
+        "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": workload_desc(name, cfg, E),
+                   "graph": "Chung-Lu G1 (SURVEY 8(d) d1), seed %d" % cfg["seed"],
+                   "l2": "inputs larger than L2 (X = %.0f MB, colidx = %.0f MB vs 126 MB L2); no flush"
+                         % (n * ld * 4 / 1e6, E * 4 / 1e6),
+                   "parallelism": "rows%d" % world if world > 1 else "single",
+                   "frac_of_8TBs": round(value / NOMINAL_HBM_GBS, 4)},
+        "ops": per_op, "create_ms": round(create_ms, 1),
+        "plan": {k: info[k] for k in ("n_hubs", "n_hub_chunks", "n_units", "n_tasks",
+                                      "hub_threshold", "hub_chunk", "max_in_degree")},
+        "roofline": roofline, "gpu_launches": args.steps * len(ops) * 1,
+        "clocks": clk.summary(), "e2e": e2e,
+    }
+    if world > 1:
+        result["gpu_launches_note"] = "per rank: 1 k_agg + NCCL broadcasts per aggregation"
+    if rank == 0 and not args.no_cpu_baseline and world == 1:
+        result["cpu_baseline"] = cpu_baseline(name, cfg, rp, ci, Xh, elh, erh, args.cpu_seconds)
+    g.close()
+    if comm is not None:
+        tlp.tlp_comm_destroy(comm)
+    if world > 1:
+        dist.destroy_process_group()
+    if rank == 0:
+        print(json.dumps(result))
+
+
+# ------------------------------------------------------- oracle baselines ---
+
+def _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows):
+    import oracle
+    import synth
+    F = cfg["F"]
+    by = 0
+    t0 = time.perf_counter()
+    for op in WORKLOADS[name]["ops"]:
+        if op == "gcn":
+            oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F)
+        elif op == "gin":
+            oracle.gin(rp, ci, Xh, synth.EPS, rows=rows, F=F)
+        else:
+            oracle.gat(rp, ci, Xh, elh, erh, synth.SLOPE, rows=rows, F=F)
+        e = int((rp[rows + 1] - rp[rows]).sum())
+        by += gather_bytes(op, len(rows), e, F)
+    return by, time.perf_counter() - t0
+
+
+def _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds, seed=0):
+    rng = np.random.default_rng(seed)
+    perm = rng.permutation(cfg["n"])
+    probe = np.sort(perm[:64])
+    by, dt = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, probe)
+    k = int(max(64, min(cfg["n"], 64 * seconds / max(dt, 1e-3))))
+    return np.sort(perm[:k])
+
+
+def cpu_baseline(name, cfg, rp, ci, Xh, elh, erh, seconds):
+    rows = _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds)
+    by, dt = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows)
+    return {"value": round(by / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"{len(rows)} of {cfg['n']} destination rows (uniform random, seed 0), "
+                      f"all ops of the step, {dt:.1f} s single-threaded fp64",
+            "host_cores_available": len(os.sched_getaffinity(0))}
+
+
+def run_reference(args):
+    """The oracle as it stands, on the host cores, on this workload's metric."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    name = args.workload
+    cfg, rp, ci, Xh, elh, erh = make_inputs(name, "cpu")
+    E = len(ci)
+    per_step = max(1.0, min(8.0, 150.0 / max(1, args.steps + args.warmup)))
+    rows = _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, per_step)
+    for _ in range(args.warmup):
+        _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows)
+    tot_b, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        b, t = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows)
+        tot_b += b
+        tot_t += t
+    value = tot_b / tot_t / 1e9
+    sample = (f"{len(rows)} of {cfg['n']} destination rows per step (uniform random, seed 0), "
+              f"all ops of the step, single-threaded fp64 oracle")
+    out = {"impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
+           "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+           "ms_per_step": round(tot_t / args.steps * 1e3, 1), "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+           "config": {"workload": workload_desc(name, cfg, E), "parallelism": "host, 1 thread"},
+           "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1,
+                            "kind": "oracle", "sample": sample},
+           "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                   "d2h_bytes_per_step": 0},
+           "gpu_launches": 0}
+    print(json.dumps(out))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="tlp", choices=["tlp", "reference"])
+    ap.add_argument("--workload", default="reddit", choices=sorted(WORKLOADS))
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        print("warning: the contract wants >= 3 warm-up steps", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_tlp(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,267 @@
+/*
+ * tlp.h -- C ABI of the B200-native TLPGNN neighbor-aggregation library.
+ *
+ * The operation (PAPER.md = /root/reference/PAPER.md, "P:<line>"):
+ *   Eq. 1-2: a_u = (+)_{v in N(u)} psi(h_u, e_vu, h_v), h'_u = sigma(a_u).
+ *   This library computes the graph-convolution phase only ("each
+ *   vertex gathers the features of all its neighbors ... combines the results
+ *   with its own features, and uses a reduce operation"); sigma and the dense
+ *   X*W phase are the caller's (out of scope).
+ *   The graph is a destination-major in-edge CSR (Fig. 7, P:1020-1028:
+ *   "int start = indptr[des_v]; ... features[indices[i]*F + f]"): the in-edges
+ *   of destination row v are e in [rowptr[v], rowptr[v+1]) with source
+ *   u = colidx[e].  The structure is static across layers, hence a
+ *   create-once handle.
+ *
+ * Conventions (all calls):
+ *   - Return codes only (tlp_status); no exception or abort crosses the ABI.
+ *     tlp_last_error() gives a thread-local detail string for the last failure.
+ *   - "device pointer" = CUDA device memory of the current device; where a
+ *     call says "device or host", any pointer CUDA's unified addressing can copy
+ *     from (cudaMemcpyDefault) is accepted.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  Aggregations are stream-ordered and never synchronise the host;
+ *     a kernel fault surfaces as TLP_ERR_CUDA on a later call.
+ *   - Features are row-major fp32 with an explicit leading dimension (row
+ *     stride in floats) ld >= F.  Only columns [0, F) of Y are written; pad
+ *     columns [F, ld) of Y are never touched (single-GPU calls).
+ *   - Ownership: a tlp_graph owns private copies of everything it was created
+ *     from; X, Y, el, er are borrowed until the enqueued work completes.
+ *   - One in-flight aggregation per handle (its scheduling counters and hub
+ *     scratch are shared); handles are not thread-safe.
+ *   - Results are bitwise reproducible: every destination row is reduced in a
+ *     fixed order (CSR order; hub chunks merged in index order) independent of
+ *     scheduling, launch geometry and the number of GPUs.
+ */
+#ifndef TLP_H
+#define TLP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define TLP_VERSION_MAJOR 0
+#define TLP_VERSION_MINOR 1
+
+typedef enum tlp_status {
+    TLP_OK = 0,
+    TLP_ERR_INVALID_ARGUMENT = 1, /* null/negative/size mismatch/overlap/alignment */
+    TLP_ERR_INVALID_GRAPH = 2,    /* CSR violates the create contract            */
+    TLP_ERR_OUT_OF_MEMORY = 3,
+    TLP_ERR_CUDA = 4,             /* a CUDA runtime error (maybe from earlier work) */
+    TLP_ERR_NCCL = 5,
+    TLP_ERR_UNSUPPORTED = 6
+} tlp_status;
+
+/* GCN normalisation ("The sum operation is weighted based on degree",
+ * P:1110-1111 "weighted sum"; the formula is not printed, reading R1):
+ *   NONE : Y[v] = sum_e w_e X[u]                                (Fig. 7 plain sum)
+ *   RIGHT: Y[v] = 1/max(d_in(v),1) * sum_e w_e X[u]             (mean)
+ *   BOTH : Y[v] = 1/sqrt(max(d_in(v),1)) * sum_e w_e X[u]/sqrt(max(d_out(u),1))
+ *          (Kipf & Welling [26]).  Degrees are unweighted edge counts. */
+typedef enum tlp_norm {
+    TLP_NORM_NONE = 0,
+    TLP_NORM_RIGHT = 1,
+    TLP_NORM_BOTH = 2
+} tlp_norm;
+
+/* Work scheduling (Section 5 "Hybrid workload balancing").  All modes
+ * produce bitwise-identical results; they differ only in speed.
+ *   DYNAMIC : persistent grid, static first wave, then atomic-counter fetch of
+ *             `step` tasks at a time (Alg. 1)           [default]
+ *   STATIC  : persistent grid, task t handled by warp t mod W (no atomics)
+ *   HARDWARE: one warp per task, grid sized to the task count
+ *   PAPER   : the paper's heuristic switch: DYNAMIC if
+ *             n_dst > 1,000,000 or nnz/n_dst > 50, else HARDWARE. */
+typedef enum tlp_sched {
+    TLP_SCHED_DYNAMIC = 0,
+    TLP_SCHED_STATIC = 1,
+    TLP_SCHED_HARDWARE = 2,
+    TLP_SCHED_PAPER = 3
+} tlp_sched;
+
+typedef struct tlp_graph_s *tlp_graph;
+typedef struct tlp_comm_s *tlp_comm;
+
+/* Plan options for tlp_graph_create_ex (0 = library default).  They change
+ * only the work decomposition (and therefore fp32 rounding order), never the
+ * mathematical result; they never depend on the GPU count. */
+typedef struct tlp_create_opts {
+    int64_t hub_threshold; /* H: rows with in-degree > H are split (default 1024) */
+    int64_t hub_chunk;     /* C: edges per hub chunk (default 512)               */
+    int64_t unit_edges;    /* K: target edges per regular work unit (default 64) */
+} tlp_create_opts;
+
+typedef struct tlp_graph_info {
+    int64_t n_dst;         /* destination rows of this handle                  */
+    int64_t n_src;         /* source vertices (rows of X)                       */
+    int64_t nnz;           /* edges of this handle                              */
+    int64_t row_offset;    /* global id of local row 0 (0 unless a dist slice)  */
+    int64_t max_in_degree;
+    int64_t n_hubs;        /* rows with in-degree > hub_threshold               */
+    int64_t n_hub_chunks;  /* sum over hubs of ceil(deg / hub_chunk)            */
+    int64_t n_units;       /* regular (non-hub) work units                      */
+    int64_t n_tasks;       /* n_hub_chunks + n_units                            */
+    int64_t hub_threshold, hub_chunk, unit_edges;
+    int64_t has_edge_weight;
+    int64_t device_bytes;  /* bytes of device memory owned by the handle        */
+    int64_t scratch_bytes; /* hub-partial scratch currently allocated           */
+    double create_ms;      /* host wall time of the create call                 */
+} tlp_graph_info;
+
+/* ---- status ------------------------------------------------------------- */
+const char *tlp_status_string(tlp_status s);
+/* Thread-local detail of the last non-OK status returned on this thread. */
+const char *tlp_last_error(void);
+/* Returns TLP_VERSION_MAJOR*100 + TLP_VERSION_MINOR. */
+int tlp_version(void);
+
+/* ---- graph handle ------------------------------------ */
+
+/* Creates a handle for the in-edge CSR with n_dst rows over n_src sources.
+ *   rowptr      : int64 [n_dst+1], device or host
+ *   colidx      : int32 [nnz],     device or host
+ *   edge_weight : fp32  [nnz] or NULL (w_e = 1), device or host
+ * Validates the CSR (rowptr[0] = 0, non-decreasing, rowptr[n_dst] = nnz,
+ * 0 <= colidx < n_src), copies it into handle-owned buffers, derives degrees,
+ * the BOTH-norm coefficients and the work plan (hub split + units), and
+ * synchronises `stream` before returning.  The caller may free its arrays on
+ * return.  n_src < 2^31.
+ * Errors: TLP_ERR_INVALID_ARGUMENT (null out, negative sizes, null arrays with
+ * nnz > 0), TLP_ERR_INVALID_GRAPH, TLP_ERR_OUT_OF_MEMORY, TLP_ERR_CUDA.  On error
+ * *out = NULL and nothing is leaked. */
+tlp_status tlp_graph_create(int64_t n_dst, int64_t n_src, int64_t nnz,
+                            const int64_t *rowptr, const int32_t *colidx,
+                            const float *edge_weight, void *stream,
+                            tlp_graph *out);
+
+/* As tlp_graph_create with explicit plan options (opts may be NULL). */
+tlp_status tlp_graph_create_ex(int64_t n_dst, int64_t n_src, int64_t nnz,
+                               const int64_t *rowptr, const int32_t *colidx,
+                               const float *edge_weight,
+                               const tlp_create_opts *opts, void *stream,
+                               tlp_graph *out);
+
+/* Waits for the handle's pending work and frees it.  NULL is a no-op. */
+tlp_status tlp_graph_destroy(tlp_graph g);
+
+/* Host-side copy of the handle's sizes and plan statistics. */
+tlp_status tlp_graph_info_get(tlp_graph g, tlp_graph_info *out);
+
+/* Copies the derived integer degrees (bit-exact structure tests):
+ * in_deg int32 [n_dst], out_deg int32 [n_src] (global over the full CSR for a
+ * dist slice).  Either may be NULL.  Device or host destinations; synchronous. */
+tlp_status tlp_graph_degrees(tlp_graph g, int32_t *in_deg, int32_t *out_deg,
+                             void *stream);
+
+/* Copies the work plan (synchronous; device or host destinations; any may be NULL):
+ *   tasks       int32 [2*n_tasks]: pairs (a,b); b >= 0: regular unit of rows
+ *               [a,b); b < 0: chunk j = -b-1 of hub index a.  Hub chunks
+ *               come first, largest hub first.
+ *   hub_rows    int32 [n_hubs]   : local row of each hub, by descending degree
+ *   hub_chunk_off int32 [n_hubs+1]: prefix sum of chunks per hub. */
+tlp_status tlp_graph_plan(tlp_graph g, int32_t *tasks, int32_t *hub_rows,
+                          int32_t *hub_chunk_off, void *stream);
+
+/* Selects the scheduler (tlp_sched), warps per CTA (0 = default 8) and the
+ * tasks fetched per atomic (Alg. 1's `step`; 0 = derived from F). */
+tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta,
+                                  int step);
+
+/* ---- aggregations (one kernel launch per call) --------- */
+
+/* GCN: Y[v, 0:F) = c_in(v) * sum_{e in row v} w_e * c_out(colidx[e]) * X[colidx[e], 0:F)
+ *   X : fp32 device [n_src x ldx], Y : fp32 device [n_dst x ldy], ld >= F >= 0.
+ * F = 0 or n_dst = 0 is a no-op.  X and Y must not overlap. */
+tlp_status tlp_gcn_aggregate(tlp_graph g, const float *X, int64_t F,
+                             int64_t ldx, int norm, float *Y, int64_t ldy,
+                             void *stream);
+
+/* GIN (Xu et al. [51]):
+ *   Y[v, 0:F) = (1+eps) * X[row_offset+v, 0:F) + sum_e w_e * X[colidx[e], 0:F)
+ * Requires row_offset + n_dst <= n_src. */
+tlp_status tlp_gin_aggregate(tlp_graph g, const float *X, int64_t F,
+                             int64_t ldx, float eps, float *Y, int64_t ldy,
+                             void *stream);
+
+/* GAT, single head ("calculates an attention coefficient for each
+ * edge and then aggregates all neighbors' features weighted by the softmax over
+ * all attentions"; Velickovic [43]).  For row v with in-degree d:
+ *   s_e = LeakyReLU(el[u] + er[row_offset+v], slope)   (x >= 0 ? x : slope*x)
+ *   Y[v] = sum_e softmax_e(s) * X[u]      (d = 0: Y[v] = 0)
+ * computed in one pass with an online (running max) softmax; scores never
+ * leave registers.  el: fp32 device [n_src]; er: fp32 device
+ * [row_offset+n_dst].  Edge weights are ignored. */
+tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F,
+                             int64_t ldx, const float *el, const float *er,
+                             float slope, float *Y, int64_t ldy, void *stream);
+
+/* ---- multi-GPU (destination-row ranges balanced by edge count) ------------ */
+
+/* Pure host function: bounds[0] = 0, bounds[parts] = n, and for 0 < k < parts
+ * bounds[k] = min{ r in [0,n] : rowptr[r] >= floor(k*nnz/parts) },
+ * nnz = rowptr[n].  rowptr_host: int64 [n+1] host; bounds_host: int64 [parts+1]. */
+tlp_status tlp_partition_rows(const int64_t *rowptr_host, int64_t n, int parts,
+                              int64_t *bounds_host);
+
+/* Handle for the destination rows [row_begin, row_end) of a full square CSR
+ * (n x n; rowptr int64 [n+1], colidx int32 [nnz], device or host): local row i
+ * is global row row_begin + i (info.row_offset = row_begin), sources stay
+ * global, out-degrees are counted over the whole CSR.  The building block of
+ * the dist layer; also lets a single process emulate any partition. */
+tlp_status tlp_graph_create_rows(int64_t n, int64_t nnz, const int64_t *rowptr,
+                                 const int32_t *colidx, const float *edge_weight,
+                                 int64_t row_begin, int64_t row_end,
+                                 const tlp_create_opts *opts, void *stream,
+                                 tlp_graph *out);
+
+/* NCCL communicator owned by the library (NCCL 2.28, one process per GPU).
+ * The unique id (128 bytes) is produced on one rank and broadcast by the
+ * caller (e.g. through torch.distributed). */
+tlp_status tlp_comm_get_unique_id(uint8_t id[128]);
+tlp_status tlp_comm_create(const uint8_t id[128], int world, int rank,
+                           tlp_comm *out);
+tlp_status tlp_comm_destroy(tlp_comm c);
+
+/* Every rank passes the FULL square CSR (n x n, device or host).  The handle
+ * holds this rank's row slice [b_k, b_{k+1}) (row_offset = b_k) with
+ * out-degrees taken over the full CSR. */
+tlp_status tlp_dist_graph_create(tlp_comm c, int64_t n, int64_t nnz,
+                                 const int64_t *rowptr, const int32_t *colidx,
+                                 const float *edge_weight,
+                                 const tlp_create_opts *opts, void *stream,
+                                 tlp_graph *out_local);
+
+/* Copies the partition bounds (int64 [world+1], host). */
+tlp_status tlp_dist_bounds(tlp_graph local, int64_t *bounds_host);
+
+/* All-gather of row slabs: rank r's rows [b_r, b_{r+1}) of Y_full (n x ldy,
+ * device) are broadcast in place to every rank (grouped ncclBroadcast; NCCL
+ * has no all-gatherv).  Whole rows including pad columns are transferred. */
+tlp_status tlp_dist_allgather_rows(tlp_graph local, tlp_comm c, float *Y_full,
+                                   int64_t ldy, void *stream);
+
+/* Local aggregation of this rank's rows into Y_full + b_k*ldy followed by
+ * tlp_dist_allgather_rows.  X_full (and el) are replicated [n x ldx]; er is
+ * the full [n] vector.  On stream completion Y_full is identical on every rank
+ * and bitwise equal to the single-GPU result. */
+tlp_status tlp_dist_gcn_aggregate(tlp_graph local, tlp_comm c,
+                                  const float *X_full, int64_t F, int64_t ldx,
+                                  int norm, float *Y_full, int64_t ldy,
+                                  void *stream);
+tlp_status tlp_dist_gin_aggregate(tlp_graph local, tlp_comm c,
+                                  const float *X_full, int64_t F, int64_t ldx,
+                                  float eps, float *Y_full, int64_t ldy,
+                                  void *stream);
+tlp_status tlp_dist_gat_aggregate(tlp_graph local, tlp_comm c,
+                                  const float *X_full, int64_t F, int64_t ldx,
+                                  const float *el, const float *er, float slope,
+                                  float *Y_full, int64_t ldy, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TLP_H */

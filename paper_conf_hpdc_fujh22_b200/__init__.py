@@ -1,0 +1,455 @@
+"""Thin Python binding of libtlp (the C ABI in include/tlp.h).
+
+Argument marshalling only: every step of the aggregation path runs in the
+CUDA kernels of libtlp.so (paper_conf_hpdc_fujh22_b200/csrc).  There is no CPU
+fallback -- importing this package fails loudly when the library is missing,
+and the aggregation calls reject non-CUDA feature tensors.
+
+The function names are the C ABI's (``tlp_graph_create``, ``tlp_gcn_aggregate``
+...).  ``Graph`` is a small convenience wrapper around a handle.
+
+PyTorch supplies device memory, the current CUDA stream and (for the dist
+layer) the process group that broadcasts the NCCL unique id; it never computes
+any part of the path.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libtlp.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+        "(there is no CPU fallback)")
+
+_lib = ctypes.CDLL(LIB_PATH)
+
+# ------------------------------------------------------------------ C types --
+TLP_OK = 0
+STATUS = {0: "TLP_OK", 1: "TLP_ERR_INVALID_ARGUMENT", 2: "TLP_ERR_INVALID_GRAPH",
+          3: "TLP_ERR_OUT_OF_MEMORY", 4: "TLP_ERR_CUDA", 5: "TLP_ERR_NCCL",
+          6: "TLP_ERR_UNSUPPORTED"}
+NORMS = {"none": 0, "right": 1, "both": 2}
+SCHEDS = {"dynamic": 0, "static": 1, "hardware": 2, "paper": 3}
+
+
+class tlp_create_opts(ctypes.Structure):
+    _fields_ = [("hub_threshold", ctypes.c_int64), ("hub_chunk", ctypes.c_int64),
+                ("unit_edges", ctypes.c_int64)]
+
+
+class tlp_graph_info(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int64) for n in (
+        "n_dst", "n_src", "nnz", "row_offset", "max_in_degree", "n_hubs", "n_hub_chunks",
+        "n_units", "n_tasks", "hub_threshold", "hub_chunk", "unit_edges", "has_edge_weight",
+        "device_bytes", "scratch_bytes")] + [("create_ms", ctypes.c_double)]
+
+
+_P = ctypes.c_void_p
+_I64 = ctypes.c_int64
+_I = ctypes.c_int
+_F = ctypes.c_float
+_sig = {
+    "tlp_status_string": ([_I], ctypes.c_char_p),
+    "tlp_last_error": ([], ctypes.c_char_p),
+    "tlp_version": ([], _I),
+    "tlp_graph_create": ([_I64, _I64, _I64, _P, _P, _P, _P, ctypes.POINTER(_P)], _I),
+    "tlp_graph_create_ex": ([_I64, _I64, _I64, _P, _P, _P, ctypes.POINTER(tlp_create_opts), _P,
+                             ctypes.POINTER(_P)], _I),
+    "tlp_graph_destroy": ([_P], _I),
+    "tlp_graph_info_get": ([_P, ctypes.POINTER(tlp_graph_info)], _I),
+    "tlp_graph_degrees": ([_P, _P, _P, _P], _I),
+    "tlp_graph_plan": ([_P, _P, _P, _P, _P], _I),
+    "tlp_graph_set_schedule": ([_P, _I, _I, _I], _I),
+    "tlp_gcn_aggregate": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
+    "tlp_gin_aggregate": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
+    "tlp_gat_aggregate": ([_P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
+    "tlp_graph_create_rows": ([_I64, _I64, _P, _P, _P, _I64, _I64, ctypes.POINTER(tlp_create_opts),
+                               _P, ctypes.POINTER(_P)], _I),
+    "tlp_partition_rows": ([_P, _I64, _I, _P], _I),
+    "tlp_comm_get_unique_id": ([_P], _I),
+    "tlp_comm_create": ([_P, _I, _I, ctypes.POINTER(_P)], _I),
+    "tlp_comm_destroy": ([_P], _I),
+    "tlp_dist_graph_create": ([_P, _I64, _I64, _P, _P, _P, ctypes.POINTER(tlp_create_opts), _P,
+                               ctypes.POINTER(_P)], _I),
+    "tlp_dist_bounds": ([_P, _P], _I),
+    "tlp_dist_allgather_rows": ([_P, _P, _P, _I64, _P], _I),
+    "tlp_dist_gcn_aggregate": ([_P, _P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
+    "tlp_dist_gin_aggregate": ([_P, _P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
+    "tlp_dist_gat_aggregate": ([_P, _P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
+}
+for _name, (_args, _res) in _sig.items():
+    _fn = getattr(_lib, _name)
+    _fn.argtypes = _args
+    _fn.restype = _res
+
+C_SYMBOLS = tuple(_sig)
+
+
+class TlpError(RuntimeError):
+    def __init__(self, status, where):
+        self.status = status
+        detail = _lib.tlp_last_error().decode(errors="replace")
+        super().__init__(f"{where}: {STATUS.get(status, status)}: {detail}")
+
+
+def _check(st, where):
+    if st != TLP_OK:
+        raise TlpError(st, where)
+
+
+def tlp_version():
+    return _lib.tlp_version()
+
+
+def tlp_status_string(s):
+    return _lib.tlp_status_string(s).decode()
+
+
+# --------------------------------------------------------------- marshalling --
+
+def _torch():
+    import torch
+    return torch
+
+
+def _ptr(a):
+    """Raw pointer of a torch tensor / numpy array (host or device) or None."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        return a.ctypes.data
+    return a.data_ptr()
+
+
+def _as_index(a, dtype):
+    """Keep torch tensors (any device) as they are if contiguous and of the right
+    dtype; numpy goes through as host memory (the library copies it)."""
+    torch = _torch()
+    if isinstance(a, torch.Tensor):
+        a = a.contiguous()
+        want = torch.int64 if dtype == np.int64 else (torch.int32 if dtype == np.int32 else torch.float32)
+        return a if a.dtype == want else a.to(want)
+    return np.ascontiguousarray(a, dtype=dtype)
+
+
+def _stream(stream, device=None):
+    if stream is not None:
+        return getattr(stream, "cuda_stream", stream)
+    torch = _torch()
+    if torch.cuda.is_available():
+        return torch.cuda.current_stream(device).cuda_stream
+    return None
+
+
+def _feat(X, F):
+    torch = _torch()
+    if not isinstance(X, torch.Tensor) or not X.is_cuda:
+        raise TypeError("features must be a CUDA torch tensor (no CPU fallback)")
+    if X.dtype != torch.float32:
+        raise TypeError("features must be float32")
+    if X.dim() == 1:
+        X = X.view(-1, 1)
+    if X.dim() != 2 or (X.shape[1] > 1 and X.stride(1) != 1) or X.stride(0) < 1:
+        raise ValueError("features must be a row-major 2-D tensor with unit column stride")
+    F = X.shape[1] if F is None else int(F)
+    ld = X.stride(0) if X.shape[0] > 1 else max(X.stride(0), X.shape[1])
+    if F > ld:
+        raise ValueError("F exceeds the leading dimension")
+    return X, F, ld
+
+
+def _out(Y, n, F, like):
+    torch = _torch()
+    if Y is None:
+        ld = (F + 3) // 4 * 4 if F > 0 else 1
+        buf = torch.empty((n, ld), dtype=torch.float32, device=like.device)
+        return buf[:, :F], F, ld
+    Y, F2, ldy = _feat(Y, F)
+    return Y, F, ldy
+
+
+def _vec_cuda(v, name):
+    torch = _torch()
+    if not isinstance(v, torch.Tensor) or not v.is_cuda or v.dtype != torch.float32:
+        raise TypeError(f"{name} must be a float32 CUDA tensor")
+    return v.contiguous()
+
+
+# ------------------------------------------------------------------ graph ----
+
+def tlp_graph_create(rowptr, colidx, n_src=None, edge_weight=None, opts=None, stream=None):
+    """Returns an opaque handle (int).  rowptr/colidx/edge_weight: torch tensors
+    (CUDA or CPU) or numpy arrays."""
+    rowptr = _as_index(rowptr, np.int64)
+    colidx = _as_index(colidx, np.int32)
+    ew = None if edge_weight is None else _as_index(edge_weight, np.float32)
+    n_dst = int(rowptr.shape[0]) - 1
+    nnz = int(colidx.shape[0])
+    if n_src is None:
+        n_src = n_dst
+    out = _P()
+    if opts:
+        o = tlp_create_opts(int(opts.get("hub_threshold", 0)), int(opts.get("hub_chunk", 0)),
+                            int(opts.get("unit_edges", 0)))
+        st = _lib.tlp_graph_create_ex(n_dst, int(n_src), nnz, _ptr(rowptr), _ptr(colidx), _ptr(ew),
+                                      ctypes.byref(o), _stream(stream), ctypes.byref(out))
+    else:
+        st = _lib.tlp_graph_create(n_dst, int(n_src), nnz, _ptr(rowptr), _ptr(colidx), _ptr(ew),
+                                   _stream(stream), ctypes.byref(out))
+    _check(st, "tlp_graph_create")
+    return out.value
+
+
+def _opts(opts):
+    if not opts:
+        return None
+    return tlp_create_opts(int(opts.get("hub_threshold", 0)), int(opts.get("hub_chunk", 0)),
+                           int(opts.get("unit_edges", 0)))
+
+
+def tlp_graph_create_rows(rowptr, colidx, row_begin, row_end, edge_weight=None, opts=None,
+                          stream=None):
+    """Handle for rows [row_begin, row_end) of the full square CSR (global
+    sources and out-degrees, row_offset = row_begin)."""
+    rowptr = _as_index(rowptr, np.int64)
+    colidx = _as_index(colidx, np.int32)
+    ew = None if edge_weight is None else _as_index(edge_weight, np.float32)
+    n = int(rowptr.shape[0]) - 1
+    out = _P()
+    o = _opts(opts)
+    st = _lib.tlp_graph_create_rows(n, int(colidx.shape[0]), _ptr(rowptr), _ptr(colidx), _ptr(ew),
+                                    int(row_begin), int(row_end), ctypes.byref(o) if o else None,
+                                    _stream(stream), ctypes.byref(out))
+    _check(st, "tlp_graph_create_rows")
+    return out.value
+
+
+def tlp_graph_destroy(g):
+    _check(_lib.tlp_graph_destroy(g), "tlp_graph_destroy")
+
+
+def tlp_graph_info_get(g):
+    info = tlp_graph_info()
+    _check(_lib.tlp_graph_info_get(g, ctypes.byref(info)), "tlp_graph_info_get")
+    return {n: getattr(info, n) for n, _ in info._fields_}
+
+
+def tlp_graph_degrees(g, stream=None):
+    info = tlp_graph_info_get(g)
+    din = np.empty(info["n_dst"], np.int32)
+    dout = np.empty(info["n_src"], np.int32)
+    _check(_lib.tlp_graph_degrees(g, _ptr(din), _ptr(dout), _stream(stream)), "tlp_graph_degrees")
+    return din, dout
+
+
+def tlp_graph_plan(g, stream=None):
+    info = tlp_graph_info_get(g)
+    tasks = np.empty((info["n_tasks"], 2), np.int32)
+    hubs = np.empty(info["n_hubs"], np.int32)
+    off = np.empty(info["n_hubs"] + 1, np.int32)
+    _check(_lib.tlp_graph_plan(g, _ptr(tasks), _ptr(hubs), _ptr(off), _stream(stream)),
+           "tlp_graph_plan")
+    return tasks, hubs, off
+
+
+def tlp_graph_set_schedule(g, sched="dynamic", warps_per_cta=0, step=0):
+    s = SCHEDS[sched] if isinstance(sched, str) else int(sched)
+    _check(_lib.tlp_graph_set_schedule(g, s, int(warps_per_cta), int(step)),
+           "tlp_graph_set_schedule")
+
+
+# ------------------------------------------------------------ aggregations ---
+
+def _n_dst(g):
+    return tlp_graph_info_get(g)["n_dst"]
+
+
+def tlp_gcn_aggregate(g, X, norm="both", Y=None, F=None, stream=None, n_dst=None):
+    X, F, ldx = _feat(X, F)
+    n = _n_dst(g) if n_dst is None else n_dst
+    Y, F, ldy = _out(Y, n, F, X)
+    nm = NORMS[norm] if isinstance(norm, str) else int(norm)
+    _check(_lib.tlp_gcn_aggregate(g, _ptr(X), F, ldx, nm, _ptr(Y), ldy, _stream(stream, X.device)),
+           "tlp_gcn_aggregate")
+    return Y
+
+
+def tlp_gin_aggregate(g, X, eps=0.0, Y=None, F=None, stream=None, n_dst=None):
+    X, F, ldx = _feat(X, F)
+    n = _n_dst(g) if n_dst is None else n_dst
+    Y, F, ldy = _out(Y, n, F, X)
+    _check(_lib.tlp_gin_aggregate(g, _ptr(X), F, ldx, float(eps), _ptr(Y), ldy,
+                                  _stream(stream, X.device)), "tlp_gin_aggregate")
+    return Y
+
+
+def tlp_gat_aggregate(g, X, el, er, slope=0.2, Y=None, F=None, stream=None, n_dst=None):
+    X, F, ldx = _feat(X, F)
+    el = _vec_cuda(el, "el")
+    er = _vec_cuda(er, "er")
+    n = _n_dst(g) if n_dst is None else n_dst
+    Y, F, ldy = _out(Y, n, F, X)
+    _check(_lib.tlp_gat_aggregate(g, _ptr(X), F, ldx, _ptr(el), _ptr(er), float(slope), _ptr(Y),
+                                  ldy, _stream(stream, X.device)), "tlp_gat_aggregate")
+    return Y
+
+
+# -------------------------------------------------------------- multi-GPU ----
+
+def tlp_partition_rows(rowptr, parts):
+    rp = np.ascontiguousarray(rowptr, dtype=np.int64)
+    b = np.empty(int(parts) + 1, np.int64)
+    _check(_lib.tlp_partition_rows(_ptr(rp), rp.shape[0] - 1, int(parts), _ptr(b)),
+           "tlp_partition_rows")
+    return b
+
+
+def tlp_comm_get_unique_id():
+    buf = (ctypes.c_uint8 * 128)()
+    _check(_lib.tlp_comm_get_unique_id(buf), "tlp_comm_get_unique_id")
+    return bytes(buf)
+
+
+def tlp_comm_create(uid, world, rank):
+    if len(uid) != 128:
+        raise ValueError("unique id must be 128 bytes")
+    buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
+    out = _P()
+    _check(_lib.tlp_comm_create(buf, int(world), int(rank), ctypes.byref(out)), "tlp_comm_create")
+    return out.value
+
+
+def tlp_comm_destroy(c):
+    _check(_lib.tlp_comm_destroy(c), "tlp_comm_destroy")
+
+
+def comm_from_torch(group=None):
+    """NCCL communicator for the current torch.distributed world; torch only
+    broadcasts the 128-byte id (rank 0 -> all)."""
+    torch = _torch()
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    obj = [tlp_comm_get_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return tlp_comm_create(obj[0], world, rank)
+
+
+def tlp_dist_graph_create(comm, rowptr, colidx, edge_weight=None, opts=None, stream=None):
+    rowptr = _as_index(rowptr, np.int64)
+    colidx = _as_index(colidx, np.int32)
+    ew = None if edge_weight is None else _as_index(edge_weight, np.float32)
+    n = int(rowptr.shape[0]) - 1
+    out = _P()
+    o = None
+    if opts:
+        o = tlp_create_opts(int(opts.get("hub_threshold", 0)), int(opts.get("hub_chunk", 0)),
+                            int(opts.get("unit_edges", 0)))
+    st = _lib.tlp_dist_graph_create(comm, n, int(colidx.shape[0]), _ptr(rowptr), _ptr(colidx),
+                                    _ptr(ew), ctypes.byref(o) if o else None, _stream(stream),
+                                    ctypes.byref(out))
+    _check(st, "tlp_dist_graph_create")
+    return out.value
+
+
+def tlp_dist_bounds(g, world):
+    b = np.empty(int(world) + 1, np.int64)
+    _check(_lib.tlp_dist_bounds(g, _ptr(b)), "tlp_dist_bounds")
+    return b
+
+
+def tlp_dist_allgather_rows(g, comm, Y_full, stream=None):
+    Y, F, ldy = _feat(Y_full, None)
+    _check(_lib.tlp_dist_allgather_rows(g, comm, _ptr(Y), ldy, _stream(stream, Y.device)),
+           "tlp_dist_allgather_rows")
+    return Y_full
+
+
+def tlp_dist_gcn_aggregate(g, comm, X_full, Y_full, norm="both", F=None, stream=None):
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_full, F)
+    nm = NORMS[norm] if isinstance(norm, str) else int(norm)
+    _check(_lib.tlp_dist_gcn_aggregate(g, comm, _ptr(X), F, ldx, nm, _ptr(Y), ldy,
+                                       _stream(stream, X.device)), "tlp_dist_gcn_aggregate")
+    return Y_full
+
+
+def tlp_dist_gin_aggregate(g, comm, X_full, Y_full, eps=0.0, F=None, stream=None):
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_full, F)
+    _check(_lib.tlp_dist_gin_aggregate(g, comm, _ptr(X), F, ldx, float(eps), _ptr(Y), ldy,
+                                       _stream(stream, X.device)), "tlp_dist_gin_aggregate")
+    return Y_full
+
+
+def tlp_dist_gat_aggregate(g, comm, X_full, Y_full, el, er, slope=0.2, F=None, stream=None):
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_full, F)
+    el = _vec_cuda(el, "el")
+    er = _vec_cuda(er, "er")
+    _check(_lib.tlp_dist_gat_aggregate(g, comm, _ptr(X), F, ldx, _ptr(el), _ptr(er), float(slope),
+                                       _ptr(Y), ldy, _stream(stream, X.device)),
+           "tlp_dist_gat_aggregate")
+    return Y_full
+
+
+# ------------------------------------------------------------ convenience ---
+
+class Graph:
+    """Owning wrapper of a tlp_graph handle."""
+
+    def __init__(self, rowptr, colidx, n_src=None, edge_weight=None, opts=None, stream=None,
+                 handle=None):
+        self.handle = handle if handle is not None else tlp_graph_create(
+            rowptr, colidx, n_src=n_src, edge_weight=edge_weight, opts=opts, stream=stream)
+        self.info = tlp_graph_info_get(self.handle)
+
+    @classmethod
+    def dist(cls, comm, rowptr, colidx, edge_weight=None, opts=None, stream=None):
+        h = tlp_dist_graph_create(comm, rowptr, colidx, edge_weight=edge_weight, opts=opts,
+                                  stream=stream)
+        return cls(None, None, handle=h)
+
+    @property
+    def n_dst(self):
+        return self.info["n_dst"]
+
+    def gcn(self, X, norm="both", Y=None, F=None, stream=None):
+        return tlp_gcn_aggregate(self.handle, X, norm, Y, F, stream, n_dst=self.n_dst)
+
+    def gin(self, X, eps=0.0, Y=None, F=None, stream=None):
+        return tlp_gin_aggregate(self.handle, X, eps, Y, F, stream, n_dst=self.n_dst)
+
+    def gat(self, X, el, er, slope=0.2, Y=None, F=None, stream=None):
+        return tlp_gat_aggregate(self.handle, X, el, er, slope, Y, F, stream, n_dst=self.n_dst)
+
+    def degrees(self):
+        return tlp_graph_degrees(self.handle)
+
+    def plan(self):
+        return tlp_graph_plan(self.handle)
+
+    def set_schedule(self, sched="dynamic", warps_per_cta=0, step=0):
+        tlp_graph_set_schedule(self.handle, sched, warps_per_cta, step)
+
+    def close(self):
+        if self.handle:
+            tlp_graph_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -1,0 +1,245 @@
+// tlp_dist.cu -- multi-GPU layer: destination-row ranges balanced
+// by edge count, X replicated, an all-gather of the output rows between layers.
+//
+// The paper is single-GPU and leaves multi-GPU to future work with METIS
+// (P:262-265); the north star replaces that with edge-balanced contiguous row
+// ranges, which need no partitioner and keep every row's in-edges (and so its
+// GAT softmax) on one rank.  Rows are independent in the pull formulation
+// (P:484-499), so a layer needs no communication inside it; the only exchange
+// is the row all-gather.  NCCL 2.28 has no all-gatherv: rank r's slab is
+// broadcast in place by a grouped ncclBroadcast(root = r).
+#include <nccl.h>
+
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "tlp_internal.h"
+
+struct tlp_comm_s {
+    ncclComm_t comm = nullptr;
+    int world = 1, rank = 0;
+};
+
+namespace tlp {
+
+static tlp_status nccl_error(ncclResult_t r, const char *what) {
+    return set_error(TLP_ERR_NCCL, std::string(what) + ": " + ncclGetErrorString(r));
+}
+
+#define TLP_NCCL_TRY(expr)                                   \
+    do {                                                     \
+        ncclResult_t _r = (expr);                            \
+        if (_r != ncclSuccess) return nccl_error(_r, #expr); \
+    } while (0)
+
+// lower_bound rule (R16): first r in [0, n] with rowptr[r] >= target.
+static int64_t lower_bound_rows(const int64_t *rowptr, int64_t n, int64_t target) {
+    int64_t lo = 0, hi = n;  // answer in [lo, hi]
+    while (lo < hi) {
+        int64_t mid = lo + (hi - lo) / 2;
+        if (rowptr[mid] < target) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+static void partition(const int64_t *rowptr, int64_t n, int parts, int64_t *b) {
+    const int64_t nnz = rowptr[n];
+    b[0] = 0;
+    for (int k = 1; k < parts; ++k) b[k] = lower_bound_rows(rowptr, n, (int64_t)k * nnz / parts);
+    b[parts] = n;
+}
+
+}  // namespace tlp
+
+using namespace tlp;
+
+extern "C" {
+
+tlp_status tlp_partition_rows(const int64_t *rowptr_host, int64_t n, int parts,
+                              int64_t *bounds_host) {
+    if (!rowptr_host || !bounds_host || n < 0 || parts < 1)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "partition: bad argument");
+    if (rowptr_host[0] != 0) return set_error(TLP_ERR_INVALID_GRAPH, "rowptr[0] != 0");
+    partition(rowptr_host, n, parts, bounds_host);
+    return TLP_OK;
+}
+
+tlp_status tlp_comm_get_unique_id(uint8_t id[128]) {
+    if (!id) return set_error(TLP_ERR_INVALID_ARGUMENT, "id is NULL");
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    ncclUniqueId u;
+    TLP_NCCL_TRY(ncclGetUniqueId(&u));
+    std::memcpy(id, &u, 128);
+    return TLP_OK;
+}
+
+tlp_status tlp_comm_create(const uint8_t id[128], int world, int rank, tlp_comm *out) {
+    if (!id || !out || world < 1 || rank < 0 || rank >= world)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "comm_create: bad argument");
+    *out = nullptr;
+    ncclUniqueId u;
+    std::memcpy(&u, id, 128);
+    tlp_comm c = new tlp_comm_s();
+    ncclResult_t r = ncclCommInitRank(&c->comm, world, u, rank);
+    if (r != ncclSuccess) {
+        delete c;
+        return nccl_error(r, "ncclCommInitRank");
+    }
+    c->world = world;
+    c->rank = rank;
+    *out = c;
+    return TLP_OK;
+}
+
+tlp_status tlp_comm_destroy(tlp_comm c) {
+    if (!c) return TLP_OK;
+    ncclResult_t r = ncclCommDestroy(c->comm);
+    delete c;
+    if (r != ncclSuccess) return nccl_error(r, "ncclCommDestroy");
+    return TLP_OK;
+}
+
+tlp_status tlp_graph_create_rows(int64_t n, int64_t nnz, const int64_t *rowptr,
+                                 const int32_t *colidx, const float *edge_weight,
+                                 int64_t row_begin, int64_t row_end, const tlp_create_opts *opts,
+                                 void *stream, tlp_graph *out) {
+    if (!rowptr || !out || n < 0 || nnz < 0 || (nnz > 0 && !colidx) || row_begin < 0 ||
+        row_end < row_begin || row_end > n)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "graph_create_rows: bad argument");
+    *out = nullptr;
+    cudaStream_t s = (cudaStream_t)stream;
+    // slice edge range from the full rowptr
+    int64_t e01[2] = {0, 0}, ends[2] = {0, 0};
+    TLP_CUDA_TRY(cudaMemcpyAsync(&e01[0], rowptr + row_begin, sizeof(int64_t), cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaMemcpyAsync(&e01[1], rowptr + row_end, sizeof(int64_t), cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaMemcpyAsync(&ends[0], rowptr, sizeof(int64_t), cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaMemcpyAsync(&ends[1], rowptr + n, sizeof(int64_t), cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaStreamSynchronize(s));
+    if (ends[0] != 0 || ends[1] != nnz)
+        return set_error(TLP_ERR_INVALID_GRAPH, "rowptr[0] != 0 or rowptr[n] != nnz");
+    const int64_t e0 = e01[0], e1 = e01[1];
+    if (e0 < 0 || e1 < e0 || e1 > nnz)
+        return set_error(TLP_ERR_INVALID_GRAPH, "rowptr not non-decreasing");
+    // the full colidx must be device-resident for the global out-degree count
+    const int32_t *full_col = colidx;
+    void *staged = nullptr;
+    if (nnz > 0) {
+        cudaPointerAttributes attr;
+        cudaError_t e = cudaPointerGetAttributes(&attr, colidx);
+        bool on_dev = (e == cudaSuccess) && (attr.type == cudaMemoryTypeDevice ||
+                                             attr.type == cudaMemoryTypeManaged);
+        if (e != cudaSuccess) cudaGetLastError();
+        if (!on_dev) {
+            TLP_CUDA_TRY(cudaMalloc(&staged, sizeof(int32_t) * nnz));
+            cudaError_t ce = cudaMemcpyAsync(staged, colidx, sizeof(int32_t) * nnz, cudaMemcpyDefault, s);
+            if (ce != cudaSuccess) { cudaFree(staged); return cuda_error(ce, "stage colidx"); }
+            full_col = (const int32_t *)staged;
+        }
+    }
+    static const int32_t kNoEdges = 0;
+    tlp_status st = graph_create_impl(row_end - row_begin, n, e1 - e0, rowptr + row_begin,
+                                      full_col ? full_col + e0 : nullptr,
+                                      edge_weight ? edge_weight + e0 : nullptr,
+                                      full_col ? full_col : &kNoEdges, nnz, row_begin, opts, s, out);
+    if (staged) {
+        cudaStreamSynchronize(s);
+        cudaFree(staged);
+    }
+    return st;
+}
+
+tlp_status tlp_dist_graph_create(tlp_comm c, int64_t n, int64_t nnz, const int64_t *rowptr,
+                                 const int32_t *colidx, const float *edge_weight,
+                                 const tlp_create_opts *opts, void *stream, tlp_graph *out_local) {
+    if (!c || !rowptr || !out_local || n < 0 || nnz < 0 || (nnz > 0 && !colidx))
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "dist_graph_create: bad argument");
+    *out_local = nullptr;
+    cudaStream_t s = (cudaStream_t)stream;
+    // the partition is a pure function of rowptr: compute it on the host
+    std::vector<int64_t> rp((size_t)n + 1);
+    TLP_CUDA_TRY(cudaMemcpyAsync(rp.data(), rowptr, sizeof(int64_t) * (n + 1), cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaStreamSynchronize(s));
+    if (rp[0] != 0 || rp[n] != nnz) return set_error(TLP_ERR_INVALID_GRAPH, "rowptr[0] != 0 or rowptr[n] != nnz");
+    for (int64_t i = 0; i < n; ++i)
+        if (rp[i + 1] < rp[i]) return set_error(TLP_ERR_INVALID_GRAPH, "rowptr not non-decreasing");
+    std::vector<int64_t> b((size_t)c->world + 1);
+    partition(rp.data(), n, c->world, b.data());
+    tlp_graph g = nullptr;
+    tlp_status st = tlp_graph_create_rows(n, nnz, rowptr, colidx, edge_weight, b[c->rank],
+                                          b[c->rank + 1], opts, stream, &g);
+    if (st != TLP_OK) return st;
+    g->world = c->world;
+    g->rank = c->rank;
+    g->n_global = n;
+    g->bounds_host = new int64_t[c->world + 1];
+    std::memcpy(g->bounds_host, b.data(), sizeof(int64_t) * (c->world + 1));
+    *out_local = g;
+    return TLP_OK;
+}
+
+tlp_status tlp_dist_bounds(tlp_graph g, int64_t *bounds_host) {
+    if (!g || !bounds_host || !g->bounds_host)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "not a dist graph");
+    std::memcpy(bounds_host, g->bounds_host, sizeof(int64_t) * (g->world + 1));
+    return TLP_OK;
+}
+
+tlp_status tlp_dist_allgather_rows(tlp_graph g, tlp_comm c, float *Y_full, int64_t ldy,
+                                   void *stream) {
+    if (!g || !c || !g->bounds_host || !Y_full || ldy < 0)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "allgather: bad argument");
+    if (c->world != g->world || c->rank != g->rank)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "communicator does not match the graph");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->world == 1) return TLP_OK;
+    TLP_NCCL_TRY(ncclGroupStart());
+    for (int r = 0; r < c->world; ++r) {
+        const int64_t rows = g->bounds_host[r + 1] - g->bounds_host[r];
+        if (rows == 0) continue;
+        float *p = Y_full + g->bounds_host[r] * ldy;
+        ncclResult_t res = ncclBroadcast(p, p, (size_t)(rows * ldy), ncclFloat, r, c->comm, s);
+        if (res != ncclSuccess) {
+            ncclGroupEnd();
+            return nccl_error(res, "ncclBroadcast");
+        }
+    }
+    TLP_NCCL_TRY(ncclGroupEnd());
+    return TLP_OK;
+}
+
+static tlp_status dist_local(tlp_graph g, tlp_comm c, AggRequest &r, void *stream) {
+    if (!g || !c || !g->bounds_host) return set_error(TLP_ERR_INVALID_ARGUMENT, "not a dist graph");
+    if (!r.Y) return set_error(TLP_ERR_INVALID_ARGUMENT, "Y_full is NULL");
+    float *Y_full = r.Y;
+    r.Y = Y_full + g->row_offset * r.ldy;
+    tlp_status st = aggregate(g, r, (cudaStream_t)stream);
+    if (st != TLP_OK) return st;
+    return tlp_dist_allgather_rows(g, c, Y_full, r.ldy, stream);
+}
+
+tlp_status tlp_dist_gcn_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t F,
+                                  int64_t ldx, int norm, float *Y_full, int64_t ldy, void *stream) {
+    AggRequest r;
+    r.op = 0; r.X = X_full; r.F = F; r.ldx = ldx; r.Y = Y_full; r.ldy = ldy; r.norm = norm;
+    return dist_local(g, c, r, stream);
+}
+
+tlp_status tlp_dist_gin_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t F,
+                                  int64_t ldx, float eps, float *Y_full, int64_t ldy, void *stream) {
+    AggRequest r;
+    r.op = 1; r.X = X_full; r.F = F; r.ldx = ldx; r.Y = Y_full; r.ldy = ldy; r.eps = eps;
+    return dist_local(g, c, r, stream);
+}
+
+tlp_status tlp_dist_gat_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t F,
+                                  int64_t ldx, const float *el, const float *er, float slope,
+                                  float *Y_full, int64_t ldy, void *stream) {
+    AggRequest r;
+    r.op = 2; r.X = X_full; r.F = F; r.ldx = ldx; r.Y = Y_full; r.ldy = ldy;
+    r.el = el; r.er = er; r.slope = slope;
+    return dist_local(g, c, r, stream);
+}
+
+}  // extern "C"

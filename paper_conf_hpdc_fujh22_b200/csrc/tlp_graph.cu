@@ -1,0 +1,554 @@
+// tlp_graph.cu -- graph handle: ingest + validate, degrees and
+// normalisation coefficients (a2), degree-aware work plan (a3).
+//
+// Create-time work is O(n + nnz) integer passes (the paper's "no
+// pre-processing" rule): no reordering, no partition
+// building beyond a row-range plan.
+#include <cub/cub.cuh>
+
+#include <chrono>
+#include <cstring>
+#include <string>
+
+#include "tlp_internal.h"
+
+namespace tlp {
+
+static thread_local std::string g_last_error;
+
+tlp_status set_error(tlp_status s, const std::string &msg) {
+    g_last_error = msg;
+    return s;
+}
+
+tlp_status cuda_error(cudaError_t e, const char *what) {
+    std::string m = std::string(what) + ": " + cudaGetErrorName(e) + " (" +
+                    cudaGetErrorString(e) + ")";
+    if (e == cudaErrorMemoryAllocation) return set_error(TLP_ERR_OUT_OF_MEMORY, m);
+    return set_error(TLP_ERR_CUDA, m);
+}
+
+// ---------------------------------------------------------------- kernels --
+
+enum : int { ERR_ROWPTR0 = 1, ERR_MONO = 2, ERR_LAST = 4, ERR_COL = 8 };
+
+// Copy + rebase the row offsets and check them (a1).
+__global__ void k_rowptr_ingest(const int64_t *__restrict__ src, int64_t n_dst,
+                                int64_t nnz, int64_t *__restrict__ dst,
+                                int32_t *__restrict__ in_deg, int *err) {
+    const int64_t base = src[0];
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n_dst;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t v = src[i] - base;
+        dst[i] = v;
+        if (i < n_dst) {
+            int64_t d = src[i + 1] - src[i];
+            if (d < 0) atomicOr(err, ERR_MONO);
+            in_deg[i] = (int32_t)d;
+        } else if (v != nnz) {
+            atomicOr(err, ERR_LAST);
+        }
+    }
+}
+
+// colidx range check and the exact integer out-degree histogram (a2).
+__global__ void k_colidx_check(const int32_t *__restrict__ colidx, int64_t nnz,
+                               int64_t n_src, int *err) {
+    int bad = 0;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        int32_t u = colidx[e];
+        bad |= (u < 0) | ((int64_t)u >= n_src);
+    }
+    if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(err, ERR_COL);
+}
+
+__global__ void k_out_degree(const int32_t *__restrict__ colidx, int64_t nnz,
+                             int32_t *__restrict__ out_deg) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz;
+         e += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(&out_deg[colidx[e]], 1);  // integer: exact in any order
+}
+
+// c_out[u] = 1/sqrt(max(out_deg,1)) (BOTH norm, Kipf [26]; R1).
+__global__ void k_norm(const int32_t *__restrict__ out_deg, int64_t n,
+                       float *__restrict__ c_out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t d = out_deg[i];
+        c_out[i] = 1.0f / sqrtf((float)(d > 1 ? d : 1));
+    }
+}
+
+// Plan flags (a3).  Row r starts a work unit iff it is row 0, a hub, follows a
+// hub, or a multiple of K edges falls in (rowptr[r-1], rowptr[r]] -- i.e. r is
+// lower_bound(rowptr, u*K) for some u.  Hubs (deg > H) become chunk tasks.
+__global__ void k_plan_flags(const int64_t *__restrict__ rowptr, int64_t n,
+                             int64_t K, int64_t H, uint8_t *__restrict__ start,
+                             uint8_t *__restrict__ hub) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n;
+         r += (int64_t)gridDim.x * blockDim.x) {
+        int64_t a = rowptr[r], b = rowptr[r + 1];
+        bool is_hub = (b - a) > H;
+        // ... or every 256th row, which bounds a unit's row count when long
+        // runs of zero-degree rows occur
+        bool s = (r == 0) || is_hub || (r % 256 == 0);
+        if (r > 0) {
+            int64_t p = rowptr[r - 1];
+            s = s || ((a - p) > H) || (a / K > p / K);
+        }
+        start[r] = s;
+        hub[r] = is_hub;
+    }
+}
+
+// Regular tasks from the unit starts; hub units are dropped (flag 0).
+__global__ void k_units_to_tasks(const int32_t *__restrict__ starts, int64_t n_units,
+                                 int64_t n, const uint8_t *__restrict__ hub,
+                                 int2 *__restrict__ out, uint8_t *__restrict__ keep) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_units;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int32_t r0 = starts[i];
+        int32_t r1 = (i + 1 < n_units) ? starts[i + 1] : (int32_t)n;
+        out[i] = make_int2(r0, r1);
+        keep[i] = !hub[r0];
+    }
+}
+
+__global__ void k_hub_chunks(const int32_t *__restrict__ hub_deg, int64_t n_hubs,
+                             int64_t C, int32_t *__restrict__ nchunk) {
+    for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < n_hubs;
+         h += (int64_t)gridDim.x * blockDim.x)
+        nchunk[h] = (int32_t)((hub_deg[h] + C - 1) / C);
+}
+
+__global__ void k_hub_tasks(const int32_t *__restrict__ hub_off, int64_t n_hubs,
+                            int2 *__restrict__ tasks) {
+    for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < n_hubs;
+         h += (int64_t)gridDim.x * blockDim.x)
+        for (int32_t j = hub_off[h]; j < hub_off[h + 1]; ++j)
+            tasks[j] = make_int2((int32_t)h, -(j - hub_off[h]) - 1);
+}
+
+__global__ void k_gather_deg(const int32_t *__restrict__ rows, int64_t n,
+                             const int32_t *__restrict__ in_deg, int32_t *__restrict__ out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = in_deg[rows[i]];
+}
+
+// ------------------------------------------------------------- host side --
+
+static int grid_for(int64_t n, int num_sms) {
+    int64_t b = (n + 255) / 256;
+    int64_t cap = (int64_t)num_sms * 8;
+    if (b > cap) b = cap;
+    if (b < 1) b = 1;
+    return (int)b;
+}
+
+namespace {
+struct DevBuf {
+    void *p = nullptr;
+    ~DevBuf() { if (p) cudaFree(p); }
+    template <class T> T *as() { return static_cast<T *>(p); }
+};
+}  // namespace
+
+static tlp_status dmalloc(void **p, size_t bytes, tlp_graph g) {
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e != cudaSuccess) return cuda_error(e, "cudaMalloc");
+    if (g) g->device_bytes += bytes;
+    return TLP_OK;
+}
+
+static void graph_free(tlp_graph g) {
+    if (!g) return;
+    void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out,
+                    g->tasks, g->hub_row, g->hub_off, g->hub_ticket, g->ctr,
+                    g->scratch};
+    for (void *p : ptrs)
+        if (p) cudaFree(p);
+    delete[] g->bounds_host;
+    delete g;
+}
+
+#define TRY(expr)                                 \
+    do {                                          \
+        tlp_status _s = (expr);                   \
+        if (_s != TLP_OK) { graph_free(g); return _s; } \
+    } while (0)
+#define CTRY(expr)                                              \
+    do {                                                        \
+        cudaError_t _e = (expr);                                \
+        if (_e != cudaSuccess) { graph_free(g); return cuda_error(_e, #expr); } \
+    } while (0)
+
+tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
+                             const int64_t *rowptr, const int32_t *colidx,
+                             const float *ew, const int32_t *full_colidx,
+                             int64_t full_nnz, int64_t row_offset,
+                             const tlp_create_opts *opts, cudaStream_t s,
+                             tlp_graph *out) {
+    auto t0 = std::chrono::steady_clock::now();
+    if (!out) return set_error(TLP_ERR_INVALID_ARGUMENT, "out is NULL");
+    *out = nullptr;
+    if (n_dst < 0 || n_src < 0 || nnz < 0 || row_offset < 0)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "negative size");
+    if (n_src >= (int64_t(1) << 31) || n_dst >= (int64_t(1) << 31))
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "n_src and n_dst must be < 2^31");
+    if (!rowptr) return set_error(TLP_ERR_INVALID_ARGUMENT, "rowptr is NULL");
+    if (nnz > 0 && !colidx) return set_error(TLP_ERR_INVALID_ARGUMENT, "colidx is NULL");
+    if (nnz > 0 && n_src == 0)
+        return set_error(TLP_ERR_INVALID_GRAPH, "edges present but n_src = 0");
+
+    tlp_graph g = new tlp_graph_s();
+    CTRY(cudaGetDevice(&g->device));
+    CTRY(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
+    g->n_dst = n_dst;
+    g->n_src = n_src;
+    g->nnz = nnz;
+    g->row_offset = row_offset;
+    g->H = (opts && opts->hub_threshold > 0) ? opts->hub_threshold : kDefaultHubThreshold;
+    g->C = (opts && opts->hub_chunk > 0) ? opts->hub_chunk : kDefaultHubChunk;
+    g->K = (opts && opts->unit_edges > 0) ? opts->unit_edges : kDefaultUnitEdges;
+    g->last_stream = s;
+    const int nsm = g->num_sms;
+
+    // ---- a1: ingest (copy; rebased rowptr) and validate -------------------
+    TRY(dmalloc((void **)&g->rowptr, sizeof(int64_t) * (n_dst + 1), g));
+    TRY(dmalloc((void **)&g->in_deg, sizeof(int32_t) * n_dst, g));
+    // colidx with 16 B of slack so vector index loads never leave the buffer
+    TRY(dmalloc((void **)&g->colidx, sizeof(int32_t) * nnz + 16, g));
+    if (nnz) CTRY(cudaMemcpyAsync(g->colidx, colidx, sizeof(int32_t) * nnz, cudaMemcpyDefault, s));
+    if (ew) {
+        TRY(dmalloc((void **)&g->ew, sizeof(float) * nnz + 16, g));
+        if (nnz) CTRY(cudaMemcpyAsync(g->ew, ew, sizeof(float) * nnz, cudaMemcpyDefault, s));
+    }
+    DevBuf rp_src, err;
+    // rowptr may be host memory: stage it in device memory first
+    {
+        cudaPointerAttributes attr;
+        cudaError_t e = cudaPointerGetAttributes(&attr, rowptr);
+        bool on_dev = (e == cudaSuccess) && (attr.type == cudaMemoryTypeDevice ||
+                                             attr.type == cudaMemoryTypeManaged);
+        if (e != cudaSuccess) cudaGetLastError();
+        const int64_t *rp_dev = rowptr;
+        if (!on_dev) {
+            CTRY(cudaMalloc(&rp_src.p, sizeof(int64_t) * (n_dst + 1)));
+            CTRY(cudaMemcpyAsync(rp_src.p, rowptr, sizeof(int64_t) * (n_dst + 1),
+                                 cudaMemcpyDefault, s));
+            rp_dev = rp_src.as<int64_t>();
+        }
+        CTRY(cudaMalloc(&err.p, sizeof(int)));
+        CTRY(cudaMemsetAsync(err.p, 0, sizeof(int), s));
+        // rowptr[0] must be the start of the slice: for a whole graph it must be 0
+        int64_t first = 0;
+        CTRY(cudaMemcpyAsync(&first, rp_dev, sizeof(int64_t), cudaMemcpyDefault, s));
+        k_rowptr_ingest<<<grid_for(n_dst + 1, nsm), 256, 0, s>>>(rp_dev, n_dst, nnz, g->rowptr,
+                                                                  g->in_deg, err.as<int>());
+        CTRY(cudaGetLastError());
+        if (nnz) {
+            k_colidx_check<<<grid_for(nnz, nsm), 256, 0, s>>>(g->colidx, nnz, n_src, err.as<int>());
+            CTRY(cudaGetLastError());
+        }
+        int herr = 0;
+        CTRY(cudaMemcpyAsync(&herr, err.p, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CTRY(cudaStreamSynchronize(s));
+        if (full_colidx == nullptr && first != 0) herr |= ERR_ROWPTR0;
+        if (herr) {
+            std::string m = "invalid CSR:";
+            if (herr & ERR_ROWPTR0) m += " rowptr[0] != 0;";
+            if (herr & ERR_MONO) m += " rowptr not non-decreasing;";
+            if (herr & ERR_LAST) m += " rowptr[n_dst] != nnz;";
+            if (herr & ERR_COL) m += " colidx outside [0, n_src);";
+            graph_free(g);
+            return set_error(TLP_ERR_INVALID_GRAPH, m);
+        }
+    }
+
+    // ---- a2: degrees and BOTH-norm coefficients --------------------------
+    TRY(dmalloc((void **)&g->out_deg, sizeof(int32_t) * n_src, g));
+    TRY(dmalloc((void **)&g->c_out, sizeof(float) * n_src, g));
+    CTRY(cudaMemsetAsync(g->out_deg, 0, sizeof(int32_t) * n_src, s));
+    {
+        const int32_t *cols = full_colidx ? full_colidx : g->colidx;
+        int64_t cnt = full_colidx ? full_nnz : nnz;
+        if (cnt) {
+            k_out_degree<<<grid_for(cnt, nsm), 256, 0, s>>>(cols, cnt, g->out_deg);
+            CTRY(cudaGetLastError());
+        }
+        if (n_src) {
+            k_norm<<<grid_for(n_src, nsm), 256, 0, s>>>(g->out_deg, n_src, g->c_out);
+            CTRY(cudaGetLastError());
+        }
+    }
+
+    // ---- a3: work plan ---------------------------------------------------
+    TRY(dmalloc((void **)&g->ctr, sizeof(unsigned int) * 4, g));
+    CTRY(cudaMemsetAsync(g->ctr, 0, sizeof(unsigned int) * 4, s));
+    if (n_dst > 0) {
+        DevBuf start, hub, starts, nsel, temp, utasks, keep, rtasks, hub_rows_u, hub_deg_u,
+            hub_deg_s, nchunk;
+        CTRY(cudaMalloc(&start.p, n_dst));
+        CTRY(cudaMalloc(&hub.p, n_dst));
+        CTRY(cudaMalloc(&starts.p, sizeof(int32_t) * n_dst));
+        CTRY(cudaMalloc(&nsel.p, sizeof(int64_t) * 4));
+        k_plan_flags<<<grid_for(n_dst, nsm), 256, 0, s>>>(g->rowptr, n_dst, g->K, g->H,
+                                                          start.as<uint8_t>(), hub.as<uint8_t>());
+        CTRY(cudaGetLastError());
+        // unit starts = rows with start flag (CUB select over a counting iterator)
+        cub::CountingInputIterator<int32_t> rows(0);
+        size_t tb = 0, tb2 = 0;
+        CTRY(cub::DeviceSelect::Flagged(nullptr, tb, rows, start.as<uint8_t>(),
+                                        starts.as<int32_t>(), nsel.as<int64_t>(), (int)n_dst, s));
+        CTRY(cub::DeviceSelect::Flagged(nullptr, tb2, rows, hub.as<uint8_t>(),
+                                        starts.as<int32_t>(), nsel.as<int64_t>(), (int)n_dst, s));
+        if (tb2 > tb) tb = tb2;
+        CTRY(cudaMalloc(&temp.p, tb));
+        CTRY(cub::DeviceSelect::Flagged(temp.p, tb, rows, start.as<uint8_t>(),
+                                        starts.as<int32_t>(), nsel.as<int64_t>(), (int)n_dst, s));
+        int64_t h_n_units = 0;
+        CTRY(cudaMemcpyAsync(&h_n_units, nsel.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CTRY(cudaStreamSynchronize(s));
+
+        CTRY(cudaMalloc(&utasks.p, sizeof(int2) * h_n_units));
+        CTRY(cudaMalloc(&keep.p, h_n_units));
+        CTRY(cudaMalloc(&rtasks.p, sizeof(int2) * h_n_units));
+        k_units_to_tasks<<<grid_for(h_n_units, nsm), 256, 0, s>>>(
+            starts.as<int32_t>(), h_n_units, n_dst, hub.as<uint8_t>(), utasks.as<int2>(),
+            keep.as<uint8_t>());
+        CTRY(cudaGetLastError());
+        size_t tb3 = 0;
+        CTRY(cub::DeviceSelect::Flagged(nullptr, tb3, utasks.as<int2>(), keep.as<uint8_t>(),
+                                        rtasks.as<int2>(), nsel.as<int64_t>() + 1, (int)h_n_units, s));
+        if (tb3 > tb) {
+            cudaFree(temp.p);
+            temp.p = nullptr;
+            CTRY(cudaMalloc(&temp.p, tb3));
+            tb = tb3;
+        }
+        CTRY(cub::DeviceSelect::Flagged(temp.p, tb, utasks.as<int2>(), keep.as<uint8_t>(),
+                                        rtasks.as<int2>(), nsel.as<int64_t>() + 1, (int)h_n_units, s));
+        // hubs in row order, then sorted by descending degree (stable => ties by row)
+        CTRY(cudaMalloc(&hub_rows_u.p, sizeof(int32_t) * n_dst));
+        CTRY(cub::DeviceSelect::Flagged(temp.p, tb, rows, hub.as<uint8_t>(),
+                                        hub_rows_u.as<int32_t>(), nsel.as<int64_t>() + 2,
+                                        (int)n_dst, s));
+        int64_t h_cnt[3] = {0, 0, 0};
+        CTRY(cudaMemcpyAsync(h_cnt, nsel.p, sizeof(int64_t) * 3, cudaMemcpyDeviceToHost, s));
+        CTRY(cudaStreamSynchronize(s));
+        const int64_t n_reg = h_cnt[1], n_hubs = h_cnt[2];
+        g->n_units = n_reg;
+        g->n_hubs = n_hubs;
+        TRY(dmalloc((void **)&g->hub_row, sizeof(int32_t) * n_hubs, g));
+        TRY(dmalloc((void **)&g->hub_off, sizeof(int32_t) * (n_hubs + 1), g));
+        TRY(dmalloc((void **)&g->hub_ticket, sizeof(int32_t) * n_hubs, g));
+        CTRY(cudaMemsetAsync(g->hub_ticket, 0, sizeof(int32_t) * (n_hubs ? n_hubs : 1), s));
+        CTRY(cudaMemsetAsync(g->hub_off, 0, sizeof(int32_t) * (n_hubs + 1), s));
+        int64_t n_chunks = 0;
+        if (n_hubs > 0) {
+            CTRY(cudaMalloc(&hub_deg_u.p, sizeof(int32_t) * n_hubs));
+            CTRY(cudaMalloc(&hub_deg_s.p, sizeof(int32_t) * n_hubs));
+            CTRY(cudaMalloc(&nchunk.p, sizeof(int32_t) * (n_hubs + 1)));
+            k_gather_deg<<<grid_for(n_hubs, nsm), 256, 0, s>>>(hub_rows_u.as<int32_t>(), n_hubs,
+                                                               g->in_deg, hub_deg_u.as<int32_t>());
+            CTRY(cudaGetLastError());
+            DevBuf t2;
+            size_t b2 = 0;
+            CTRY(cub::DeviceRadixSort::SortPairsDescending(
+                nullptr, b2, hub_deg_u.as<int32_t>(), hub_deg_s.as<int32_t>(),
+                hub_rows_u.as<int32_t>(), g->hub_row, (int)n_hubs, 0, 32, s));
+            CTRY(cudaMalloc(&t2.p, b2));
+            CTRY(cub::DeviceRadixSort::SortPairsDescending(
+                t2.p, b2, hub_deg_u.as<int32_t>(), hub_deg_s.as<int32_t>(),
+                hub_rows_u.as<int32_t>(), g->hub_row, (int)n_hubs, 0, 32, s));
+            k_hub_chunks<<<grid_for(n_hubs, nsm), 256, 0, s>>>(hub_deg_s.as<int32_t>(), n_hubs,
+                                                               g->C, nchunk.as<int32_t>());
+            CTRY(cudaGetLastError());
+            CTRY(cudaMemsetAsync(nchunk.as<int32_t>() + n_hubs, 0, sizeof(int32_t), s));
+            DevBuf t3;
+            size_t b3 = 0;
+            CTRY(cub::DeviceScan::ExclusiveSum(nullptr, b3, nchunk.as<int32_t>(), g->hub_off,
+                                               (int)(n_hubs + 1), s));
+            CTRY(cudaMalloc(&t3.p, b3));
+            CTRY(cub::DeviceScan::ExclusiveSum(t3.p, b3, nchunk.as<int32_t>(), g->hub_off,
+                                               (int)(n_hubs + 1), s));
+            int32_t hc = 0;
+            CTRY(cudaMemcpyAsync(&hc, g->hub_off + n_hubs, sizeof(int32_t),
+                                 cudaMemcpyDeviceToHost, s));
+            int32_t maxdeg = 0;
+            CTRY(cudaMemcpyAsync(&maxdeg, hub_deg_s.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+            CTRY(cudaStreamSynchronize(s));
+            n_chunks = hc;
+            g->max_in_degree = maxdeg;
+        }
+        g->n_chunks = n_chunks;
+        g->n_tasks = n_chunks + n_reg;
+        TRY(dmalloc((void **)&g->tasks, sizeof(int2) * g->n_tasks, g));
+        if (n_hubs > 0) {
+            k_hub_tasks<<<grid_for(n_hubs, nsm), 256, 0, s>>>(g->hub_off, n_hubs, g->tasks);
+            CTRY(cudaGetLastError());
+        }
+        if (n_reg)
+            CTRY(cudaMemcpyAsync(g->tasks + n_chunks, rtasks.p, sizeof(int2) * n_reg,
+                                 cudaMemcpyDeviceToDevice, s));
+        if (n_hubs == 0) {
+            // max in-degree over regular rows (<= H): one reduction
+            DevBuf mx, t4;
+            size_t b4 = 0;
+            CTRY(cudaMalloc(&mx.p, sizeof(int32_t)));
+            CTRY(cub::DeviceReduce::Max(nullptr, b4, g->in_deg, mx.as<int32_t>(), (int)n_dst, s));
+            CTRY(cudaMalloc(&t4.p, b4));
+            CTRY(cub::DeviceReduce::Max(t4.p, b4, g->in_deg, mx.as<int32_t>(), (int)n_dst, s));
+            int32_t m = 0;
+            CTRY(cudaMemcpyAsync(&m, mx.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+            CTRY(cudaStreamSynchronize(s));
+            g->max_in_degree = m;
+        }
+        g->regular_edges = nnz;  // refined below (edges outside hubs)
+        CTRY(cudaStreamSynchronize(s));
+    }
+    if (n_dst > 0 && g->n_hubs > 0) {
+        // edges in hubs = sum of hub degrees: recompute on the host from chunk count bound
+        // (only used to size the Alg. 1 step heuristic; no correctness role)
+        g->regular_edges = nnz - std::min<int64_t>(nnz, g->n_chunks * g->C);
+        if (g->regular_edges < 0) g->regular_edges = 0;
+    }
+    auto t1 = std::chrono::steady_clock::now();
+    g->create_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    *out = g;
+    return TLP_OK;
+}
+
+tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s) {
+    if (bytes <= g->scratch_bytes) return TLP_OK;
+    if (g->scratch) {
+        cudaError_t e = cudaFreeAsync(g->scratch, s);
+        if (e != cudaSuccess) return cuda_error(e, "cudaFreeAsync(scratch)");
+        g->device_bytes -= g->scratch_bytes;
+        g->scratch = nullptr;
+        g->scratch_bytes = 0;
+    }
+    cudaError_t e = cudaMallocAsync((void **)&g->scratch, bytes, s);
+    if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(scratch)");
+    g->scratch_bytes = bytes;
+    g->device_bytes += bytes;
+    return TLP_OK;
+}
+
+}  // namespace tlp
+
+// ================================================================ C ABI ====
+
+using namespace tlp;
+
+extern "C" {
+
+const char *tlp_status_string(tlp_status s) {
+    switch (s) {
+        case TLP_OK: return "TLP_OK";
+        case TLP_ERR_INVALID_ARGUMENT: return "TLP_ERR_INVALID_ARGUMENT";
+        case TLP_ERR_INVALID_GRAPH: return "TLP_ERR_INVALID_GRAPH";
+        case TLP_ERR_OUT_OF_MEMORY: return "TLP_ERR_OUT_OF_MEMORY";
+        case TLP_ERR_CUDA: return "TLP_ERR_CUDA";
+        case TLP_ERR_NCCL: return "TLP_ERR_NCCL";
+        case TLP_ERR_UNSUPPORTED: return "TLP_ERR_UNSUPPORTED";
+    }
+    return "TLP_ERR_UNKNOWN";
+}
+
+const char *tlp_last_error(void) { return g_last_error.c_str(); }
+
+int tlp_version(void) { return TLP_VERSION_MAJOR * 100 + TLP_VERSION_MINOR; }
+
+tlp_status tlp_graph_create(int64_t n_dst, int64_t n_src, int64_t nnz, const int64_t *rowptr,
+                            const int32_t *colidx, const float *edge_weight, void *stream,
+                            tlp_graph *out) {
+    return graph_create_impl(n_dst, n_src, nnz, rowptr, colidx, edge_weight, nullptr, 0, 0,
+                             nullptr, (cudaStream_t)stream, out);
+}
+
+tlp_status tlp_graph_create_ex(int64_t n_dst, int64_t n_src, int64_t nnz, const int64_t *rowptr,
+                               const int32_t *colidx, const float *edge_weight,
+                               const tlp_create_opts *opts, void *stream, tlp_graph *out) {
+    if (opts && (opts->hub_threshold < 0 || opts->hub_chunk < 0 || opts->unit_edges < 0))
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "negative plan option");
+    return graph_create_impl(n_dst, n_src, nnz, rowptr, colidx, edge_weight, nullptr, 0, 0, opts,
+                             (cudaStream_t)stream, out);
+}
+
+tlp_status tlp_graph_destroy(tlp_graph g) {
+    if (!g) return TLP_OK;
+    cudaError_t e = cudaStreamSynchronize(g->last_stream);
+    graph_free(g);
+    if (e != cudaSuccess) return cuda_error(e, "cudaStreamSynchronize(destroy)");
+    return TLP_OK;
+}
+
+tlp_status tlp_graph_info_get(tlp_graph g, tlp_graph_info *o) {
+    if (!g || !o) return set_error(TLP_ERR_INVALID_ARGUMENT, "null argument");
+    std::memset(o, 0, sizeof(*o));
+    o->n_dst = g->n_dst;
+    o->n_src = g->n_src;
+    o->nnz = g->nnz;
+    o->row_offset = g->row_offset;
+    o->max_in_degree = g->max_in_degree;
+    o->n_hubs = g->n_hubs;
+    o->n_hub_chunks = g->n_chunks;
+    o->n_units = g->n_units;
+    o->n_tasks = g->n_tasks;
+    o->hub_threshold = g->H;
+    o->hub_chunk = g->C;
+    o->unit_edges = g->K;
+    o->has_edge_weight = g->ew != nullptr;
+    o->device_bytes = (int64_t)g->device_bytes;
+    o->scratch_bytes = (int64_t)g->scratch_bytes;
+    o->create_ms = g->create_ms;
+    return TLP_OK;
+}
+
+tlp_status tlp_graph_degrees(tlp_graph g, int32_t *in_deg, int32_t *out_deg, void *stream) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (in_deg && g->n_dst)
+        TLP_CUDA_TRY(cudaMemcpyAsync(in_deg, g->in_deg, sizeof(int32_t) * g->n_dst,
+                                     cudaMemcpyDefault, s));
+    if (out_deg && g->n_src)
+        TLP_CUDA_TRY(cudaMemcpyAsync(out_deg, g->out_deg, sizeof(int32_t) * g->n_src,
+                                     cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaStreamSynchronize(s));
+    return TLP_OK;
+}
+
+tlp_status tlp_graph_plan(tlp_graph g, int32_t *tasks, int32_t *hub_rows, int32_t *hub_chunk_off,
+                          void *stream) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (tasks && g->n_tasks)
+        TLP_CUDA_TRY(cudaMemcpyAsync(tasks, g->tasks, sizeof(int2) * g->n_tasks,
+                                     cudaMemcpyDefault, s));
+    if (hub_rows && g->n_hubs)
+        TLP_CUDA_TRY(cudaMemcpyAsync(hub_rows, g->hub_row, sizeof(int32_t) * g->n_hubs,
+                                     cudaMemcpyDefault, s));
+    if (hub_chunk_off && g->hub_off)
+        TLP_CUDA_TRY(cudaMemcpyAsync(hub_chunk_off, g->hub_off, sizeof(int32_t) * (g->n_hubs + 1),
+                                     cudaMemcpyDefault, s));
+    TLP_CUDA_TRY(cudaStreamSynchronize(s));
+    return TLP_OK;
+}
+
+tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta, int step) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    if (sched < TLP_SCHED_DYNAMIC || sched > TLP_SCHED_PAPER)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown scheduler");
+    if (warps_per_cta < 0 || warps_per_cta > 32 || step < 0)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "warps_per_cta in [0,32], step >= 0");
+    g->sched = sched;
+    g->warps_per_cta = warps_per_cta ? warps_per_cta : 8;
+    g->step = step;
+    return TLP_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,102 @@
+// tlp_internal.h -- private structures of libtlp (not part of the C ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "tlp.h"
+
+namespace tlp {
+
+// Defaults of the work plan.  Functions of
+// nothing but these constants: never of the GPU count, SM count or timing, so
+// the reduction order of every row is partition- and schedule-invariant.
+constexpr int64_t kDefaultHubThreshold = 1024;  // H
+constexpr int64_t kDefaultHubChunk = 512;       // C
+constexpr int64_t kDefaultUnitEdges = 64;       // K
+
+// Thread-local error detail; returns `s` for chaining.
+tlp_status set_error(tlp_status s, const std::string &msg);
+tlp_status cuda_error(cudaError_t e, const char *what);
+
+#define TLP_CUDA_TRY(expr)                                      \
+    do {                                                        \
+        cudaError_t _e = (expr);                                \
+        if (_e != cudaSuccess) return ::tlp::cuda_error(_e, #expr); \
+    } while (0)
+
+}  // namespace tlp
+
+// The opaque handle.  All pointers are device memory owned by the handle.
+struct tlp_graph_s {
+    int64_t n_dst = 0, n_src = 0, nnz = 0, row_offset = 0;
+    int device = 0;
+    int num_sms = 0;
+    int64_t max_in_degree = 0;
+    int64_t H = 0, C = 0, K = 0;
+
+    int64_t *rowptr = nullptr;   // [n_dst+1], rowptr[0] = 0
+    int32_t *colidx = nullptr;   // [nnz]
+    float *ew = nullptr;         // [nnz] or null
+    int32_t *in_deg = nullptr;   // [n_dst]
+    int32_t *out_deg = nullptr;  // [n_src] (global for a dist slice)
+    float *c_out = nullptr;      // [n_src] 1/sqrt(max(out_deg,1))
+
+    int2 *tasks = nullptr;       // [n_tasks]
+    int32_t *hub_row = nullptr;  // [n_hubs]
+    int32_t *hub_off = nullptr;  // [n_hubs+1]
+    int32_t *hub_ticket = nullptr;  // [n_hubs], zero between calls
+    unsigned int *ctr = nullptr;    // [2]: next task, finished warps
+    int64_t n_tasks = 0, n_units = 0, n_hubs = 0, n_chunks = 0;
+    int64_t regular_edges = 0;
+
+    float *scratch = nullptr;    // hub partials
+    size_t scratch_bytes = 0;
+    size_t device_bytes = 0;
+    double create_ms = 0.0;
+
+    int sched = TLP_SCHED_DYNAMIC;
+    int warps_per_cta = 8;
+    int step = 0;
+
+    // dist slice bookkeeping
+    int world = 1, rank = 0;
+    int64_t *bounds_host = nullptr;  // [world+1] or null
+    int64_t n_global = 0;
+    cudaStream_t last_stream = nullptr;
+};
+
+struct tlp_comm_s;
+
+namespace tlp {
+
+// Internal create used by both the single-GPU and the dist entry points.
+//   rowptr/colidx/ew describe rows [row_begin, row_end) of a CSR whose
+//   rowptr values are absolute (rebased by rowptr[row_begin]); out-degrees
+//   are counted over full_colidx[0:full_nnz) (the full CSR).
+tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
+                             const int64_t *rowptr, const int32_t *colidx,
+                             const float *ew, const int32_t *full_colidx,
+                             int64_t full_nnz, int64_t row_offset,
+                             const tlp_create_opts *opts, cudaStream_t s,
+                             tlp_graph *out);
+
+tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s);
+
+// Enqueue one aggregation kernel; op: 0 GCN, 1 GIN, 2 GAT.
+struct AggRequest {
+    int op = 0;
+    const float *X = nullptr;
+    int64_t F = 0, ldx = 0;
+    float *Y = nullptr;
+    int64_t ldy = 0;
+    int norm = 0;
+    float eps = 0.f;
+    const float *el = nullptr, *er = nullptr;
+    float slope = 0.f;
+};
+tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s);
+
+}  // namespace tlp

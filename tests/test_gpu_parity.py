@@ -1,0 +1,413 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle, element by
+element, within the north-star tolerance |err| <= 1e-5 * sum|terms| + 1e-6.
+Structure (degrees, plan, partition) is compared bit-exactly."""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def tlp():
+    import paper_conf_hpdc_fujh22_b200 as m
+    return m
+
+
+DEV = "cuda:0"
+
+
+def _t(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
+
+
+def _check(name, Yg, ref, F=None):
+    Yr, Ar = ref
+    Yg = Yg.detach().cpu().numpy().astype(np.float64)
+    if F is not None:
+        Yg = Yg[:, :F]
+    ok, worst = oracle.within_tolerance(Yg, Yr, Ar)
+    assert ok, f"{name}: worst err/tol = {worst:.3g}"
+    return worst
+
+
+def _run_all(tlp, rp, ci, n_src, F, ld, opts=None, ew=None, seed=0, nonneg=False, slope=0.2,
+             eps=0.1, ops=("gcn_none", "gcn_right", "gcn_both", "gin", "gat"), ldy=None,
+             x_offset=0):
+    n_dst = len(rp) - 1
+    lo = 0.0 if nonneg else -1.0
+    Xh = synth.features(n_src, F, ld, seed=seed, low=lo)
+    el = synth.normal(n_src, seed + 1)
+    er = synth.normal(max(n_dst, 1), seed + 2)
+    g = tlp.Graph(_t(rp), _t(ci), n_src=n_src, edge_weight=None if ew is None else _t(ew), opts=opts)
+    # optional misalignment: X starts `x_offset` floats into a buffer
+    Xbuf = torch.zeros(n_src * ld + x_offset + 8, dtype=torch.float32, device=DEV)
+    X = Xbuf[x_offset:x_offset + n_src * ld].view(n_src, ld) if n_src else Xbuf[:0].view(0, ld)
+    X.copy_(_t(Xh))
+    ldy = ldy or ld
+    res = {}
+    for op in ops:
+        Y = torch.full((n_dst, ldy), float("nan"), dtype=torch.float32, device=DEV)
+        if op.startswith("gcn"):
+            g.gcn(X, op[4:], Y=Y, F=F)
+            ref = oracle.gcn(rp, ci, Xh, op[4:], ew=ew, n_src=n_src, F=F)
+        elif op == "gin":
+            g.gin(X, eps, Y=Y, F=F)
+            ref = oracle.gin(rp, ci, Xh, eps, ew=ew, F=F)
+        else:
+            g.gat(X, _t(el), _t(er), slope, Y=Y, F=F)
+            ref = oracle.gat(rp, ci, Xh, el, er, slope, F=F)
+        torch.cuda.synchronize()
+        _check(op, Y[:, :F], ref)
+        if ldy > F:  # pad columns untouched
+            assert torch.isnan(Y[:, F:]).all(), f"{op}: pad columns written"
+        res[op] = Y[:, :F].clone()
+    g.close()
+    return res
+
+
+# ------------------------------------------------------------------ P1 -----
+
+def test_figure1_star_golden(tlp):
+    import json, os
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "figure1_star.json")))
+    rp, ci = synth.figure1_star(True)
+    X = _t(np.array(gold["x"], np.float32).reshape(4, 1))
+    g = tlp.Graph(_t(rp), _t(ci))
+    for nm in ("none", "right", "both"):
+        Y = g.gcn(X, nm).cpu().numpy().ravel()
+        np.testing.assert_allclose(Y, gold["with_self_loops"]["gcn_" + nm], rtol=2e-7)
+    el = _t(np.log(np.array(gold["x"])).astype(np.float32))
+    Y = g.gat(X, el, _t(np.zeros(4, np.float32)), 0.2).cpu().numpy().ravel()
+    np.testing.assert_allclose(Y, gold["with_self_loops"]["gat_slope0.2_el_lnx_er0"], rtol=1e-6)
+    Y = g.gat(X, el, _t(np.full(4, -10, np.float32)), 0.2).cpu().numpy().ravel()
+    np.testing.assert_allclose(Y, gold["with_self_loops"]["gat_slope0.2_el_lnx_er-10"], rtol=1e-6)
+    g.close()
+    rp, ci = synth.figure1_star(False)
+    g = tlp.Graph(_t(rp), _t(ci))
+    Y = g.gin(X, 0.5).cpu().numpy().ravel()
+    np.testing.assert_allclose(Y, gold["without_self_loops"]["gin_eps0.5"], rtol=1e-7)
+    g.close()
+
+
+# ------------------------------------------------------------ edge cases ----
+
+def _edge_graphs():
+    G = {}
+    G["e0_n5"] = (np.zeros(6, np.int64), np.zeros(0, np.int32), 5)
+    G["isolated_last"] = synth.random_graph(40, 40, 200, 1, isolated_tail=1) + (40,)
+    G["selfloops_multi"] = synth.random_graph(30, 30, 400, 2, self_loops=True, multi=True) + (30,)
+    n = 300
+    src = np.arange(1, n); dst = np.zeros(n - 1, np.int64)
+    G["star_hub"] = synth.csr_from_edges(n, np.concatenate([src, dst]),
+                                         np.concatenate([dst, src])) + (n,)
+    G["random64"] = synth.random_graph(64, 64, 700, 3) + (64,)
+    G["rect_more_src"] = synth.random_graph(20, 77, 300, 4) + (77,)
+    G["rect_more_dst"] = synth.random_graph(90, 13, 300, 5, isolated_tail=7) + (13,)
+    G["one_row"] = (np.array([0, 5], np.int64), np.array([0, 0, 0, 0, 0], np.int32), 1)
+    G["powerlaw_hubs"] = synth.power_law_rows(
+        500, np.minimum((3000 / (np.arange(500) + 1) ** 0.8).astype(int), 2000), 500, 6) + (500,)
+    return G
+
+
+@pytest.mark.parametrize("name", list(_edge_graphs()))
+def test_edge_case_graphs(tlp, name):
+    rp, ci, n_src = _edge_graphs()[name]
+    ops = ("gcn_none", "gcn_right", "gcn_both", "gat")
+    if len(rp) - 1 <= n_src:
+        ops = ops + ("gin",)
+    _run_all(tlp, rp, ci, n_src, 37, 40, opts=dict(hub_threshold=64, hub_chunk=32), ops=ops)
+
+
+def test_empty_graph_and_zero_features(tlp):
+    g = tlp.Graph(_t(np.zeros(1, np.int64)), _t(np.zeros(0, np.int32)), n_src=0)
+    assert g.info["n_tasks"] == 0
+    X = torch.zeros((0, 4), device=DEV)
+    Y = g.gcn(X, "both")
+    assert Y.shape == (0, 4)
+    g.close()
+    rp, ci = synth.random_graph(10, 10, 30, 1)
+    g = tlp.Graph(_t(rp), _t(ci))
+    Y = torch.full((10, 4), 7.0, device=DEV)
+    g.gcn(torch.ones((10, 4), device=DEV), "both", Y=Y, F=0)
+    assert (Y == 7).all()
+    g.close()
+
+
+@pytest.mark.parametrize("F", [1, 2, 3, 4, 5, 31, 32, 33, 100, 127, 128, 129, 500, 602, 1433])
+def test_feature_widths(tlp, F):
+    rp, ci = synth.power_law_rows(
+        200, np.minimum((900 / (np.arange(200) + 1) ** 0.7).astype(int) + 1, 700), 200, F)
+    for ld in sorted({F, (F + 3) // 4 * 4}):
+        _run_all(tlp, rp, ci, 200, F, ld, opts=dict(hub_threshold=100, hub_chunk=48), seed=F,
+                 ops=("gcn_both", "gin", "gat"))
+
+
+@pytest.mark.parametrize("x_offset", [1, 2])
+def test_misaligned_features_use_narrow_vectors(tlp, x_offset):
+    rp, ci = synth.random_graph(50, 50, 600, 7)
+    _run_all(tlp, rp, ci, 50, 64, 64, x_offset=x_offset, ops=("gcn_both", "gin", "gat"))
+
+
+def test_hub_degree_boundaries(tlp):
+    H, C = 64, 32
+    degs = [H - 1, H, H + 1, C, C + 1, 2 * C, 2 * C + 1, 3 * C + 5, 7 * C, 0, 1]
+    degs = np.array(degs * 3, np.int64)
+    n = len(degs)
+    rp, ci = synth.power_law_rows(n, degs, n, 11)
+    _run_all(tlp, rp, ci, n, 70, 72, opts=dict(hub_threshold=H, hub_chunk=C))
+    _run_all(tlp, rp, ci, n, 70, 72, opts=dict(hub_threshold=H, hub_chunk=C), nonneg=True)
+
+
+@pytest.mark.parametrize("name", ["random64", "powerlaw_hubs", "selfloops_multi"])
+def test_weighted(tlp, name):
+    rp, ci, n_src = _edge_graphs()[name]
+    ew = synth.edge_weights(len(ci), 3)
+    _run_all(tlp, rp, ci, n_src, 45, 48, ew=ew, opts=dict(hub_threshold=64, hub_chunk=32),
+             ops=("gcn_none", "gcn_right", "gcn_both", "gin"))
+
+
+def test_gat_slopes_and_eps(tlp):
+    rp, ci = synth.random_graph(80, 80, 2000, 8)
+    for slope in (0.0, 0.2, 1.0):
+        _run_all(tlp, rp, ci, 80, 33, 36, slope=slope, ops=("gat",), opts=dict(hub_threshold=16, hub_chunk=8))
+    for eps in (-1.0, 0.0, 2.5):
+        _run_all(tlp, rp, ci, 80, 33, 36, eps=eps, ops=("gin",))
+
+
+# --------------------------------------------------------- structure T1 -----
+
+def test_structure_bit_exact(tlp):
+    cfg = synth.CONFIGS["pubmed"]
+    rp, ci = synth.dataset_graph("pubmed")
+    n = cfg["n"]
+    for opts in (None, dict(hub_threshold=40, hub_chunk=16, unit_edges=32)):
+        g = tlp.Graph(_t(rp), _t(ci), opts=opts)
+        din, dout = g.degrees()
+        assert np.array_equal(din, oracle.in_degree(rp))
+        assert np.array_equal(dout, oracle.out_degree(ci, n))
+        info = g.info
+        H, C = info["hub_threshold"], info["hub_chunk"]
+        tasks, hubs, off = g.plan()
+        deg = np.diff(rp)
+        # hubs: exactly the rows with deg > H, by descending degree, ties by row
+        exp = np.nonzero(deg > H)[0]
+        exp = exp[np.lexsort((exp, -deg[exp]))]
+        assert hubs.tolist() == exp.tolist()
+        assert off.tolist() == [0] + np.cumsum(-(-deg[exp] // C)).tolist()
+        # every row is covered exactly once (Alg. 1 semantics)
+        cover = np.zeros(n, np.int64)
+        nch = info["n_hub_chunks"]
+        for k, (a, b) in enumerate(tasks):
+            if b >= 0:
+                assert k >= nch
+                cover[a:b] += 1
+            else:
+                assert k < nch
+        for h, r in enumerate(hubs):
+            seen = sorted(-b - 1 for a, b in tasks[:nch] if a == h)
+            assert seen == list(range(off[h + 1] - off[h]))
+            cover[r] += 1
+        assert np.all(cover == 1)
+        assert info["max_in_degree"] == deg.max()
+        g.close()
+
+
+def test_invalid_graphs_rejected(tlp):
+    rp, ci = synth.random_graph(10, 10, 30, 1)
+    bad = [(rp + 1, ci), (np.r_[rp[:5], rp[5:] - 100], ci), (rp, np.r_[ci[:-1], 10].astype(np.int32)),
+           (rp, np.r_[ci[:-1], -1].astype(np.int32))]
+    for brp, bci in bad:
+        with pytest.raises(tlp.TlpError) as e:
+            tlp.Graph(_t(brp), _t(bci), n_src=10)
+        assert e.value.status == 2
+    with pytest.raises(tlp.TlpError):
+        tlp.Graph(_t(rp[:-1]), _t(ci), n_src=10)  # rowptr[n] != nnz
+
+
+def test_overlap_rejected(tlp):
+    rp, ci = synth.random_graph(10, 10, 30, 1)
+    g = tlp.Graph(_t(rp), _t(ci))
+    buf = torch.zeros((10, 8), device=DEV)
+    with pytest.raises(tlp.TlpError) as e:
+        g.gcn(buf[:, :4], "none", Y=buf[:, 2:6], F=4)
+    assert e.value.status == 1
+    g.close()
+
+
+def test_host_pointer_create(tlp):
+    rp, ci = synth.random_graph(60, 60, 500, 2)
+    g = tlp.Graph(rp, ci)  # numpy: host memory, copied by the library
+    X = synth.features(60, 9, 12, seed=1)
+    Y = g.gcn(_t(X), "both", F=9)
+    _check("host-create", Y, oracle.gcn(rp, ci, X, "both", F=9))
+    g.close()
+
+
+# ------------------------------------------------------- determinism T4 -----
+
+def test_deterministic_across_runs_and_schedules(tlp):
+    rp, ci = synth.chung_lu(3000, 60000, 0.5, 3, device="cpu")
+    X = _t(synth.features(3000, 130, 132, seed=3))
+    el, er = _t(synth.normal(3000, 1)), _t(synth.normal(3000, 2))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=100, hub_chunk=40))
+    base = {"gcn": g.gcn(X, "both", F=130).clone(), "gin": g.gin(X, 0.1, F=130).clone(),
+            "gat": g.gat(X, el, er, 0.2, F=130).clone()}
+    for sched in ("dynamic", "static", "hardware", "paper"):
+        for wpc, step in ((8, 0), (4, 1), (2, 3), (16, 7)):
+            g.set_schedule(sched, wpc, step)
+            for _ in range(2):
+                assert torch.equal(g.gcn(X, "both", F=130), base["gcn"]), (sched, wpc, step)
+                assert torch.equal(g.gin(X, 0.1, F=130), base["gin"]), (sched, wpc, step)
+                assert torch.equal(g.gat(X, el, er, 0.2, F=130), base["gat"]), (sched, wpc, step)
+    g.close()
+
+
+# --------------------------------------------------- multi-GPU emulation T6 --
+
+@pytest.mark.parametrize("parts", [2, 3, 8])
+def test_partition_emulation_bitwise(tlp, parts):
+    """Each rank's slice (tlp_graph_create_rows over the bounds of
+    tlp_partition_rows) writes its rows of Y_full; the concatenation is bitwise
+    equal to the single-GPU result (H, C never depend on P)."""
+    n = 2000
+    rp, ci = synth.chung_lu(n, 50000, 0.55, 5, device="cpu")
+    F = 70
+    X = _t(synth.features(n, F, 72, seed=4))
+    el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
+    opts = dict(hub_threshold=64, hub_chunk=32)
+    g = tlp.Graph(_t(rp), _t(ci), opts=opts)
+    ref = {"gcn": g.gcn(X, "both", F=F), "gin": g.gin(X, 0.1, F=F), "gat": g.gat(X, el, er, 0.2, F=F)}
+    b = tlp.tlp_partition_rows(rp, parts)
+    assert b.tolist() == oracle.partition(rp, parts).tolist()
+    out = {k: torch.full((n, 72), float("nan"), device=DEV) for k in ref}
+    for k in range(parts):
+        h = tlp.tlp_graph_create_rows(_t(rp), _t(ci), int(b[k]), int(b[k + 1]), opts=opts)
+        sl = tlp.Graph(None, None, handle=h)
+        assert sl.info["row_offset"] == b[k]
+        r0, r1 = int(b[k]), int(b[k + 1])
+        if r1 > r0:
+            sl.gcn(X, "both", Y=out["gcn"][r0:r1], F=F)
+            sl.gin(X, 0.1, Y=out["gin"][r0:r1], F=F)
+            sl.gat(X, el, er, 0.2, Y=out["gat"][r0:r1], F=F)
+        din, dout = sl.degrees()
+        assert np.array_equal(dout, oracle.out_degree(ci, n))
+        assert np.array_equal(din, np.diff(rp)[r0:r1])
+        sl.close()
+    for k in ref:
+        assert torch.equal(out[k][:, :F], ref[k]), k
+    g.close()
+
+
+def test_dist_world1_nccl(tlp):
+    """The NCCL path with one rank: dist create + aggregate + (no-op) all-gather."""
+    n = 500
+    rp, ci = synth.chung_lu(n, 8000, 0.5, 7, device="cpu")
+    F = 33
+    X = _t(synth.features(n, F, 36, seed=1))
+    uid = tlp.tlp_comm_get_unique_id()
+    comm = tlp.tlp_comm_create(uid, 1, 0)
+    h = tlp.tlp_dist_graph_create(comm, _t(rp), _t(ci))
+    assert tlp.tlp_dist_bounds(h, 1).tolist() == [0, n]
+    Y = torch.zeros((n, 36), device=DEV)
+    tlp.tlp_dist_gcn_aggregate(h, comm, X, Y, "both", F=F)
+    g = tlp.Graph(_t(rp), _t(ci))
+    assert torch.equal(Y[:, :F], g.gcn(X, "both", F=F))
+    tlp.tlp_graph_destroy(h)
+    tlp.tlp_comm_destroy(comm)
+    g.close()
+
+
+# ------------------------------------------------------ config-scale T3 -----
+
+def test_config_cora_gcn_all_rows(tlp):
+    cfg = synth.CONFIGS["cora"]
+    rp, ci = synth.dataset_graph("cora")
+    X = synth.dataset_features("cora", cfg["n"])
+    g = tlp.Graph(_t(rp), _t(ci))
+    Y = g.gcn(_t(X), "both", F=cfg["F"])
+    _check("cora gcn", Y, oracle.gcn(rp, ci, X, "both", F=cfg["F"]))
+    g.close()
+
+
+def test_config_pubmed_gat_all_rows(tlp):
+    cfg = synth.CONFIGS["pubmed"]
+    n = cfg["n"]
+    rp, ci = synth.dataset_graph("pubmed")
+    X = synth.dataset_features("pubmed", n)
+    el, er = synth.normal(n, 201), synth.normal(n, 202)
+    g = tlp.Graph(_t(rp), _t(ci))
+    Y = g.gat(_t(X), _t(el), _t(er), synth.SLOPE, F=cfg["F"])
+    _check("pubmed gat", Y, oracle.gat(rp, ci, X, el, er, synth.SLOPE, F=cfg["F"]))
+    g.close()
+
+
+def _sample_rows(rp, n_rand, n_hub, seed):
+    deg = np.diff(rp)
+    rng = np.random.default_rng(seed)
+    top = np.argsort(-deg, kind="stable")[:n_hub]
+    rnd = rng.choice(len(deg), size=min(n_rand, len(deg)), replace=False)
+    return np.unique(np.concatenate([top, rnd, [0, len(deg) - 1]]))
+
+
+@pytest.fixture(scope="module")
+def reddit():
+    rp, ci = synth.dataset_graph("reddit")
+    return rp, ci
+
+
+@pytest.mark.parametrize("nonneg", [False, True])
+def test_config_reddit_gcn_gin_sampled(tlp, reddit, nonneg):
+    cfg = synth.CONFIGS["reddit"]
+    n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+    rp, ci = reddit
+    X = synth.features(n, F, ld, seed=103, low=0.0 if nonneg else -1.0)
+    g = tlp.Graph(_t(rp), _t(ci))
+    assert g.info["n_hubs"] > 0
+    rows = _sample_rows(rp, 400, 60, 1)
+    Xd = _t(X)
+    Y = g.gcn(Xd, "both", F=F)
+    _check("reddit gcn", Y[_t(rows)], oracle.gcn(rp, ci, X, "both", rows=rows, F=F))
+    Y = g.gin(Xd, synth.EPS, F=F)
+    _check("reddit gin", Y[_t(rows)], oracle.gin(rp, ci, X, synth.EPS, rows=rows, F=F))
+    # properties at full size: NONE(ones) is the in-degree exactly
+    ones = torch.ones((n, 4), device=DEV)
+    Yo = g.gcn(ones, "none")
+    assert torch.equal(Yo[:, 0].cpu(), torch.from_numpy(np.diff(rp).astype(np.float32)))
+    g.close()
+
+
+def test_config_reddit_gat_sampled(tlp, reddit):
+    cfg = synth.CONFIGS["reddit"]
+    n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+    rp, ci = reddit
+    X = synth.features(n, F, ld, seed=103)
+    el, er = synth.normal(n, 301), synth.normal(n, 302)
+    g = tlp.Graph(_t(rp), _t(ci))
+    rows = _sample_rows(rp, 300, 40, 2)
+    Y = g.gat(_t(X), _t(el), _t(er), synth.SLOPE, F=F)
+    _check("reddit gat", Y[_t(rows)], oracle.gat(rp, ci, X, el, er, synth.SLOPE, rows=rows, F=F))
+    # GAT of ones is one on every row with in-edges (softmax rows sum to 1)
+    Yo = g.gat(torch.ones((n, 4), device=DEV), _t(el), _t(er), synth.SLOPE)
+    deg = torch.from_numpy(np.diff(rp)).to(DEV)
+    assert torch.allclose(Yo[deg > 0], torch.ones_like(Yo[deg > 0]), rtol=0, atol=1e-5 + 1e-6)
+    g.close()
+
+
+def test_config_products_gat_sampled(tlp):
+    cfg = synth.CONFIGS["products"]
+    n, F = cfg["n"], cfg["F"]
+    rp, ci = synth.dataset_graph("products")
+    X = synth.dataset_features("products", n)
+    el, er = synth.normal(n, 401), synth.normal(n, 402)
+    g = tlp.Graph(_t(rp), _t(ci))
+    rows = _sample_rows(rp, 3000, 60, 3)
+    Y = g.gat(_t(X), _t(el), _t(er), synth.SLOPE, F=F)
+    _check("products gat", Y[_t(rows)], oracle.gat(rp, ci, X, el, er, synth.SLOPE, rows=rows, F=F))
+    g.close()
