@@ -20,7 +20,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtlp.so")
+# TLP_LIB_PATH selects an in-tree tuning variant of the library (bench/profiling)
+LIB_PATH = os.environ.get("TLP_LIB_PATH") or os.path.join(_HERE, "libtlp.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

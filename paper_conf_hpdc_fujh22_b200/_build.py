@@ -56,19 +56,23 @@ def up_to_date():
     return all(os.path.getmtime(d) <= t for d in _deps())
 
 
-def build(force=False, verbose=False, ptxas_verbose=False):
-    if not force and up_to_date():
+def build(force=False, verbose=False, ptxas_verbose=False, defines=(), out=None):
+    """defines: extra -D macros (tuning variants); out: alternative .so path."""
+    lib = out or LIB
+    if not force and not defines and out is None and up_to_date():
         return LIB
-    os.makedirs(BUILD, exist_ok=True)
+    bdir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
+    os.makedirs(bdir, exist_ok=True)
     nccl_inc, nccl_lib = nccl_dirs()
     flags = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O3",
                     "--expt-relaxed-constexpr", "-I" + INCLUDE, "-I" + CSRC, "-I" + nccl_inc]
     if ptxas_verbose:
         flags += ["-Xptxas", "-v"]
+    flags += ["-D" + d for d in defines]
     objs = []
 
     def compile_one(src):
-        obj = os.path.join(BUILD, os.path.basename(src) + ".o")
+        obj = os.path.join(bdir, os.path.basename(src) + ".o")
         cmd = [nvcc()] + flags + ["-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
@@ -81,7 +85,7 @@ def build(force=False, verbose=False, ptxas_verbose=False):
 
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 2)) as ex:
         objs = list(ex.map(compile_one, _sources()))
-    tmp = LIB + ".tmp%d" % os.getpid()
+    tmp = lib + ".tmp%d" % os.getpid()
     nccl_so = sorted(glob.glob(os.path.join(nccl_lib, "libnccl.so*")))[0]
     cmd = [nvcc()] + ARCH + ["-shared", "-o", tmp] + objs + [
         "-L" + nccl_lib, "-l:" + os.path.basename(nccl_so), "-Xlinker", "-rpath," + nccl_lib,
@@ -91,11 +95,12 @@ def build(force=False, verbose=False, ptxas_verbose=False):
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="-v" in sys.argv,
-          ptxas_verbose="--ptxas" in sys.argv)
-    print(LIB)
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv,
+                ptxas_verbose="--ptxas" in sys.argv, defines=defs, out=outs[0] if outs else None))

@@ -29,6 +29,8 @@
 #include <math.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
 
 #include "tlp_internal.h"
 
@@ -39,6 +41,21 @@ enum Coef : int { COEF_NONE = 0, COEF_COUT = 1, COEF_W = 2, COEF_W_COUT = 3 };
 enum Sched : int { S_DYNAMIC = 0, S_STATIC = 1, S_HARDWARE = 2 };
 
 constexpr unsigned FULL = 0xffffffffu;
+
+// Compile-time tuning knobs: source rows per
+// gather group (two groups in flight per warp) and the launch bounds.
+#ifndef TLP_U
+#define TLP_U 2        // register path: rows per gather group (2 groups in flight)
+#endif
+#ifndef TLP_MAXT
+#define TLP_MAXT 256   // threads per CTA at most (8 warps)
+#endif
+#ifndef TLP_MINB
+#define TLP_MINB 4     // register path: 4 CTAs/SM -> 64 registers, 32 warps/SM
+#endif
+#ifndef TLP_MINB_ASYNC
+#define TLP_MINB_ASYNC 3  // async path: 3 CTAs/SM (ring = 3 x 64 KB of shared memory)
+#endif
 
 struct AggArgs {
     const int64_t *__restrict__ rowptr;
@@ -57,8 +74,8 @@ struct AggArgs {
     float *md;       // GAT hub (m, den) pairs [n_chunks x 2]
     unsigned long long *ctr;
     unsigned int *done;
-    int64_t ldx, ldy, ldp, row_offset, n_tasks, C;
-    int F, n_strips, norm, step, sched;
+    int64_t ldx, ldy, ldp, row_offset, n_tasks, n_items, n_hubs, n_chunks, C;
+    int F, n_strips, norm, step, sched, panel;
     float eps1, slope;
 };
 
@@ -134,67 +151,264 @@ __device__ __forceinline__ float warp_sum(float v) {
     return v;
 }
 
+// Issue the gathers of edges [j, j+U) of the current 32-edge chunk (lane k of
+// the chunk holds source u and coefficient c of edge k).
+template <int VEC, int U, bool HASC>
+__device__ __forceinline__ void issue_group(const float *__restrict__ Xc, unsigned ldx, int j, int n,
+                                            bool active, int u_l, float c_l, Vec<VEC> (&xv)[U],
+                                            float (&ck)[U]) {
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+        const int jj = j + k;
+        const int u = __shfl_sync(FULL, u_l, jj & 31);
+        if constexpr (HASC) ck[k] = __shfl_sync(FULL, c_l, jj & 31);
+        if (jj < n && active) {
+            xv[k] = ld_vec<VEC>(Xc + (size_t)((unsigned)u) * ldx);  // IMAD.WIDE.U32
+        } else {
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) xv[k].v[c] = 0.f;
+        }
+    }
+}
+
+// Accumulate a gathered group in CSR order.
+template <int VEC, int U, bool HASC>
+__device__ __forceinline__ void consume_group(int j, int n, const Vec<VEC> (&xv)[U],
+                                              const float (&ck)[U], Vec<VEC> &acc) {
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+        if (j + k < n) {
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) {
+                if constexpr (HASC) acc.v[c] = fmaf(ck[k], xv[k].v[c], acc.v[c]);
+                else acc.v[c] += xv[k].v[c];
+            }
+        }
+    }
+}
+
 // Reduce the edges [e0, e1) of one destination row for the feature vector at
 // `col` (a6 / a7).  GCN/GIN: acc = sum_e c_e X[u_e] in CSR order.  GAT: online
 // softmax state (m, den, acc = sum_e exp(s_e - m) X[u_e]).
+//
+// Latency hiding (the kernel is bound by bytes in flight, not by arithmetic):
+//  * edge indices are loaded 32 at a time by the lanes two chunks ahead, and
+//    the index-dependent values (c_out[u] or el[u]) one chunk ahead, so the
+//    gathers of a chunk never wait on an index load;
+//  * the gathers of a chunk are issued in double-buffered groups of U source
+//    rows: the next group is in flight while the current one is accumulated.
 template <int VEC, int OP, int COEF, int U>
 __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64_t e1,
                                              int col, bool active, float er_v, int lane,
                                              Vec<VEC> &acc, float &m, float &den) {
+    constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT);
+    constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);  // index-dependent value
     const float *__restrict__ Xc = a.X + col;
-    for (int64_t base = e0; base < e1; base += 32) {
-        const int n = (int)min((int64_t)32, e1 - base);
-        int u_l = 0;
-        float c_l = 1.f;
-        if (lane < n) {
-            u_l = __ldg(a.colidx + base + lane);
-            if constexpr (COEF & COEF_COUT) c_l = __ldg(a.c_out + u_l);
-            if constexpr (COEF & COEF_W) c_l *= __ldg(a.ew + base + lane);
+    const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
+    const unsigned ldx = (unsigned)a.ldx;
+    // 32-bit edge offsets relative to e0 (a row or hub chunk has < 2^31 edges)
+    const int32_t *__restrict__ ci = a.colidx + e0;
+    const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
+    const int len = (int)(e1 - e0);
+    if (len <= 0) return;
+    int off = 0;
+    int n0 = min(32, len);
+    int n1 = min(32, len - 32);
+    int u0 = 0, u1 = 0;
+    float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
+    if (lane < n0) {
+        u0 = __ldg(ci + lane);
+        if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
+    }
+    if (lane < n1) {
+        u1 = __ldg(ci + 32 + lane);
+        if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
+    }
+    if constexpr (DEP)
+        if (lane < n0) d0 = __ldg(dep + u0);
+    while (true) {
+        // two chunks ahead: indices; one chunk ahead: index-dependent values
+        const int n2 = min(32, len - off - 64);
+        int u2 = 0;
+        float w2 = 1.f;
+        if (lane < n2) {
+            u2 = __ldg(ci + off + 64 + lane);
+            if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
         }
+        if constexpr (DEP)
+            if (lane < n1) d1 = __ldg(dep + u1);
+        // coefficients of the current chunk
+        float c_l = 1.f;
         if constexpr (OP == OP_GAT) {
             float s = -INFINITY;
-            if (lane < n) {
-                float t = __ldg(a.el + u_l) + er_v;
+            if (lane < n0) {
+                const float t = d0 + er_v;
                 s = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
             }
             const float m_new = fmaxf(m, warp_max(s));
             const float scale = __expf(m - m_new);  // m = -inf -> 0
-            c_l = (lane < n) ? __expf(s - m_new) : 0.f;
+            c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
             den = fmaf(den, scale, warp_sum(c_l));
 #pragma unroll
             for (int c = 0; c < VEC; ++c) acc.v[c] *= scale;
             m = m_new;
+        } else {
+            if constexpr (COEF & COEF_COUT) c_l = d0;
+            if constexpr (COEF & COEF_W) c_l *= w0;
         }
-        for (int j = 0; j < n; j += U) {
-            Vec<VEC> xv[U];
-            float ck[U];
-#pragma unroll
-            for (int k = 0; k < U; ++k) {
-                const int jj = j + k;
-                const int u = __shfl_sync(FULL, u_l, jj & 31);
-                if constexpr (COEF != COEF_NONE || OP == OP_GAT)
-                    ck[k] = __shfl_sync(FULL, c_l, jj & 31);
-                if (jj < n && active) {
-                    xv[k] = ld_vec<VEC>(Xc + (int64_t)u * a.ldx);
-                } else {
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) xv[k].v[c] = 0.f;
-                }
-            }
-#pragma unroll
-            for (int k = 0; k < U; ++k) {
-                if (j + k < n) {
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) {
-                        if constexpr (COEF != COEF_NONE || OP == OP_GAT)
-                            acc.v[c] = fmaf(ck[k], xv[k].v[c], acc.v[c]);
-                        else
-                            acc.v[c] += xv[k].v[c];
-                    }
-                }
+        // gathers: double-buffered groups of U rows
+        {
+            Vec<VEC> xa[U], xb[U];
+            float ca[U], cb[U];
+            issue_group<VEC, U, HASC>(Xc, ldx, 0, n0, active, u0, c_l, xa, ca);
+            for (int j = 0; j < n0; j += 2 * U) {
+                issue_group<VEC, U, HASC>(Xc, ldx, j + U, n0, active, u0, c_l, xb, cb);
+                consume_group<VEC, U, HASC>(j, n0, xa, ca, acc);
+                issue_group<VEC, U, HASC>(Xc, ldx, j + 2 * U, n0, active, u0, c_l, xa, ca);
+                consume_group<VEC, U, HASC>(j + U, n0, xb, cb, acc);
             }
         }
+        if (n1 <= 0) break;
+        off += 32;
+        n0 = n1; n1 = n2;
+        u0 = u1; u1 = u2;
+        w0 = w1; w1 = w2;
+        d0 = d1;
     }
+}
+
+// ---- asynchronous-copy variant (TLP_ASYNC) --------------------------------
+// The gathered rows land in a per-warp shared-memory ring through cp.async
+// (LDGSTS, L2 -> SMEM, bypassing L1 and the register file), D edges deep.  Bytes
+// in flight then cost no registers, so occupancy and depth are decoupled.
+#ifndef TLP_DEPTH
+#define TLP_DEPTH 16   // edges in flight per warp on the async path
+#endif
+
+template <int VEC>
+__device__ __forceinline__ void cp_async_vec(float *dst_smem, const float *src, bool pred) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
+    const int bytes = pred ? 4 * VEC : 0;  // src-size 0 => zero fill, no global read
+    if constexpr (VEC == 4)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
+    else if constexpr (VEC == 2)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
+    else
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+template <int VEC>
+__device__ __forceinline__ float *warp_ring() {
+    extern __shared__ __align__(16) float tlp_smem[];
+    const int w = threadIdx.x >> 5;
+    return tlp_smem + (size_t)w * TLP_DEPTH * 32 * VEC;
+}
+
+template <int VEC, int OP, int COEF, int U>
+__device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0, int64_t e1,
+                                                   int col, bool active, float er_v, int lane,
+                                                   Vec<VEC> &acc, float &m, float &den) {
+    constexpr int D = TLP_DEPTH;
+    constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);
+    const float *__restrict__ Xc = a.X + col;
+    const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
+    const unsigned ldx = (unsigned)a.ldx;
+    const int32_t *__restrict__ ci = a.colidx + e0;
+    const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
+    const int len = (int)(e1 - e0);
+    if (len <= 0) return;
+    float *ring = warp_ring<VEC>() + lane * VEC;
+    int off = 0;
+    int n0 = min(32, len);
+    int n1 = min(32, len - 32);
+    int u0 = 0, u1 = 0;
+    float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
+    if (lane < n0) {
+        u0 = __ldg(ci + lane);
+        if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
+    }
+    if (lane < n1) {
+        u1 = __ldg(ci + 32 + lane);
+        if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
+    }
+    if constexpr (DEP)
+        if (lane < n0) d0 = __ldg(dep + u0);
+    // prologue: edges 0 .. D-2 in flight
+#pragma unroll
+    for (int k = 0; k < D - 1; ++k) {
+        const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
+        cp_async_vec<VEC>(ring + k * 32 * VEC, Xc + (size_t)((unsigned)uk) * ldx, active && k < len);
+        cp_async_commit();
+    }
+    int slot = 0;  // ring slot of edge `off + j`
+    while (true) {
+        const int n2 = min(32, len - off - 64);
+        int u2 = 0;
+        float w2 = 1.f;
+        if (lane < n2) {
+            u2 = __ldg(ci + off + 64 + lane);
+            if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
+        }
+        if constexpr (DEP)
+            if (lane < n1) d1 = __ldg(dep + u1);
+        float c_l = 1.f;
+        if constexpr (OP == OP_GAT) {
+            float s = -INFINITY;
+            if (lane < n0) {
+                const float t = d0 + er_v;
+                s = t >= 0.f ? t : a.slope * t;
+            }
+            const float m_new = fmaxf(m, warp_max(s));
+            const float scale = __expf(m - m_new);
+            c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
+            den = fmaf(den, scale, warp_sum(c_l));
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) acc.v[c] *= scale;
+            m = m_new;
+        } else {
+            if constexpr (COEF & COEF_COUT) c_l = d0;
+            if constexpr (COEF & COEF_W) c_l *= w0;
+        }
+        for (int j = 0; j < n0; ++j) {
+            // issue edge j + D - 1 (in this chunk or the next one)
+            const int jj = j + D - 1;
+            const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
+            const bool valid = (off + jj) < len;
+            int ws = slot + D - 1;
+            if (ws >= D) ws -= D;
+            cp_async_vec<VEC>(ring + ws * 32 * VEC, Xc + (size_t)((unsigned)ui) * ldx, active && valid);
+            cp_async_commit();
+            cp_async_wait<D - 1>();
+            const float cj = __shfl_sync(FULL, c_l, j);
+            const float *src = ring + slot * 32 * VEC;
+            if constexpr (VEC == 4) {
+                const float4 x = *reinterpret_cast<const float4 *>(src);
+                if constexpr (COEF != COEF_NONE || OP == OP_GAT) {
+                    acc.v[0] = fmaf(cj, x.x, acc.v[0]); acc.v[1] = fmaf(cj, x.y, acc.v[1]);
+                    acc.v[2] = fmaf(cj, x.z, acc.v[2]); acc.v[3] = fmaf(cj, x.w, acc.v[3]);
+                } else {
+                    acc.v[0] += x.x; acc.v[1] += x.y; acc.v[2] += x.z; acc.v[3] += x.w;
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < VEC; ++c) {
+                    if constexpr (COEF != COEF_NONE || OP == OP_GAT) acc.v[c] = fmaf(cj, src[c], acc.v[c]);
+                    else acc.v[c] += src[c];
+                }
+            }
+            if (++slot == D) slot = 0;
+        }
+        if (n1 <= 0) break;
+        off += 32;
+        n0 = n1; n1 = n2;
+        u0 = u1; u1 = u2;
+        w0 = w1; w1 = w2;
+        d0 = d1;
+    }
+    cp_async_wait<0>();  // drain the (empty) tail groups before the ring is reused
 }
 
 // Epilogue (a9) for a full row reduction.
@@ -225,9 +439,10 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_
     return y;
 }
 
-// A regular work unit: whole rows [r0, r1).
-template <int VEC, int OP, int COEF, int U>
-__device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int lane) {
+// A regular work unit: whole rows [r0, r1), feature strips [s0, s1).
+template <int VEC, int OP, int COEF, int U, bool ASYNC>
+__device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0, int s1,
+                                        int lane) {
     for (int rb = r0; rb < r1; rb += 31) {
         const int nr = min(31, r1 - rb);
         // lanes fetch the row offsets of up to 31 rows at once (register caching
@@ -243,14 +458,17 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int la
             const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
             const int64_t r = rb + k;
             float *yrow = a.Y + r * a.ldy;
-            for (int s = 0; s < a.n_strips; ++s) {
+            for (int s = s0; s < s1; ++s) {
                 const int col = s * 32 * VEC + lane * VEC;
                 const bool active = col < a.F;
                 Vec<VEC> acc;
 #pragma unroll
                 for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
                 float m = -INFINITY, den = 0.f;
-                reduce_edges<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+                if constexpr (ASYNC)
+                    reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+                else
+                    reduce_edges<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
                 if (active) st_row<VEC>(yrow, col, a.F, y);
             }
@@ -258,10 +476,12 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int la
     }
 }
 
-// One C-edge chunk of hub h (a8).  The last chunk to finish merges all the
-// partials of the hub in chunk order and writes the row.
-template <int VEC, int OP, int COEF, int U>
-__device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int lane) {
+// One C-edge chunk of hub h (a8), feature strips [s0, s1).  The last chunk of
+// the hub to finish these strips merges all its partials in chunk order and
+// writes the row.  Tickets (and GAT (m, den) pairs) are kept per panel s0.
+template <int VEC, int OP, int COEF, int U, bool ASYNC>
+__device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int s0, int s1,
+                                             int lane) {
     const int r = __ldg(a.hub_row + h);
     const int off = __ldg(a.hub_off + h);
     const int nch = __ldg(a.hub_off + h + 1) - off;
@@ -271,39 +491,44 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     float er_v = 0.f;
     if constexpr (OP == OP_GAT) er_v = __ldg(a.er + a.row_offset + r);
     const int slot = off + j;
-    for (int s = 0; s < a.n_strips; ++s) {
+    float *md = a.md + 2 * (int64_t)s0 * a.n_chunks;  // this panel's (m, den) pairs
+    int32_t *ticket = a.hub_ticket + (int64_t)s0 * a.n_hubs + h;
+    for (int s = s0; s < s1; ++s) {
         const int col = s * 32 * VEC + lane * VEC;
         const bool active = col < a.F;
         Vec<VEC> acc;
 #pragma unroll
         for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
         float m = -INFINITY, den = 0.f;
-        reduce_edges<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+        if constexpr (ASYNC)
+                    reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+                else
+                    reduce_edges<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
         if (active) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
         if constexpr (OP == OP_GAT)
-            if (s == 0 && lane == 0) {
-                a.md[2 * (int64_t)slot] = m;
-                a.md[2 * (int64_t)slot + 1] = den;
+            if (s == s0 && lane == 0) {
+                md[2 * (int64_t)slot] = m;
+                md[2 * (int64_t)slot + 1] = den;
             }
     }
     __threadfence();
     __syncwarp();
     int last = 0;
-    if (lane == 0) last = (atomicAdd(a.hub_ticket + h, 1) == nch - 1);
+    if (lane == 0) last = (atomicAdd(ticket, 1) == nch - 1);
     last = __shfl_sync(FULL, last, 0);
     if (!last) return;
     __threadfence();
     float *yrow = a.Y + (int64_t)r * a.ldy;
     float M = -INFINITY, D = 0.f;
     if constexpr (OP == OP_GAT) {
-        for (int q = 0; q < nch; ++q) M = fmaxf(M, __ldcg(a.md + 2 * (int64_t)(off + q)));
+        for (int q = 0; q < nch; ++q) M = fmaxf(M, __ldcg(md + 2 * (int64_t)(off + q)));
         for (int q = 0; q < nch; ++q) {
-            const float mq = __ldcg(a.md + 2 * (int64_t)(off + q));
-            const float dq = __ldcg(a.md + 2 * (int64_t)(off + q) + 1);
+            const float mq = __ldcg(md + 2 * (int64_t)(off + q));
+            const float dq = __ldcg(md + 2 * (int64_t)(off + q) + 1);
             D = fmaf(dq, __expf(mq - M), D);
         }
     }
-    for (int s = 0; s < a.n_strips; ++s) {
+    for (int s = s0; s < s1; ++s) {
         const int col = s * 32 * VEC + lane * VEC;
         const bool active = col < a.F;
         Vec<VEC> acc;
@@ -313,7 +538,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
             for (int q = 0; q < nch; ++q) {
                 Vec<VEC> p = ld_vec_cg<VEC>(a.scratch + (int64_t)(off + q) * a.ldp + col);
                 if constexpr (OP == OP_GAT) {
-                    const float w = __expf(__ldcg(a.md + 2 * (int64_t)(off + q)) - M);
+                    const float w = __expf(__ldcg(md + 2 * (int64_t)(off + q)) - M);
 #pragma unroll
                     for (int c = 0; c < VEC; ++c) acc.v[c] = fmaf(w, p.v[c], acc.v[c]);
                 } else {
@@ -325,32 +550,42 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         Vec<VEC> y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
         if (active) st_row<VEC>(yrow, col, a.F, y);
     }
-    if (lane == 0) a.hub_ticket[h] = 0;  // self-reset for the next launch
+    if (lane == 0) *ticket = 0;  // self-reset for the next launch
 }
 
-template <int VEC, int OP, int COEF, int U>
-__device__ __forceinline__ void do_task(const AggArgs &a, int64_t t, int lane) {
+// Work item i: task-major (all strips of task i) or, in panel mode, strip
+// s = i / n_tasks of task i % n_tasks, so that all warps sweep one L2-resident
+// feature panel of X at a time.
+template <int VEC, int OP, int COEF, int U, bool ASYNC>
+__device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
+    int64_t t = i;
+    int s0 = 0, s1 = a.n_strips;
+    if (a.panel) {
+        s0 = (int)(i / a.n_tasks);
+        t = i - (int64_t)s0 * a.n_tasks;
+        s1 = s0 + 1;
+    }
     const int2 tk = a.tasks[t];
-    if (tk.y >= 0) do_unit<VEC, OP, COEF, U>(a, tk.x, tk.y, lane);
-    else do_hub_chunk<VEC, OP, COEF, U>(a, tk.x, -tk.y - 1, lane);
+    if (tk.y >= 0) do_unit<VEC, OP, COEF, U, ASYNC>(a, tk.x, tk.y, s0, s1, lane);
+    else do_hub_chunk<VEC, OP, COEF, U, ASYNC>(a, tk.x, -tk.y - 1, s0, s1, lane);
 }
 
-template <int VEC, int OP, int COEF, int U>
-__global__ void __launch_bounds__(512, 1) k_agg(const AggArgs a) {
+template <int VEC, int OP, int COEF, int U, bool ASYNC>
+__global__ void __launch_bounds__(TLP_MAXT, ASYNC ? TLP_MINB_ASYNC : TLP_MINB) k_agg(const AggArgs a) {
     const int lane = threadIdx.x & 31;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (a.sched == S_HARDWARE) {  // one warp per task
-        if (wid < a.n_tasks) do_task<VEC, OP, COEF, U>(a, wid, lane);
+    if (a.sched == S_HARDWARE) {  // one warp per item
+        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC>(a, wid, lane);
         return;
     }
     const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int64_t stride = W * a.step;
     int64_t t = wid * a.step;  // static first wave
-    while (t < a.n_tasks) {
+    while (t < a.n_items) {
         unsigned long long v = 0;
         if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned long long)a.step);
-        const int64_t tend = min(t + a.step, a.n_tasks);
-        for (int64_t tt = t; tt < tend; ++tt) do_task<VEC, OP, COEF, U>(a, tt, lane);
+        const int64_t tend = min(t + a.step, a.n_items);
+        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC>(a, tt, lane);
         if (a.sched == S_DYNAMIC) t = stride + (int64_t)__shfl_sync(FULL, v, 0);
         else t += stride;
     }
@@ -367,36 +602,51 @@ __global__ void __launch_bounds__(512, 1) k_agg(const AggArgs a) {
 
 // ------------------------------------------------------------- dispatch --
 
-constexpr int kU = 8;  // source rows in flight per warp
+constexpr int kU = TLP_U;  // source rows per gather group (2 groups in flight)
 
 typedef void (*KernelFn)(const AggArgs);
 
-template <int VEC>
+template <int VEC, bool ASYNC>
 static KernelFn pick(int op, int coef) {
     if (op == OP_GCN) {
         switch (coef) {
-            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU>;
-            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU>;
-            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU>;
-            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU>;
+            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU, ASYNC>;
+            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU, ASYNC>;
+            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU, ASYNC>;
+            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU, ASYNC>;
         }
     }
     if (op == OP_GIN)
-        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU> : k_agg<VEC, OP_GIN, COEF_NONE, kU>;
-    return k_agg<VEC, OP_GAT, COEF_NONE, kU>;
+        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC>
+                             : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC>;
+    return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC>;
 }
 
-static int occupancy_blocks(KernelFn fn, int threads) {
-    // small cache keyed by (kernel, threads)
-    struct Entry { KernelFn fn; int threads; int blocks; };
+template <bool ASYNC>
+static KernelFn pick_vec(int vec, int op, int coef) {
+    return vec == 4 ? pick<4, ASYNC>(op, coef) : vec == 2 ? pick<2, ASYNC>(op, coef) : pick<1, ASYNC>(op, coef);
+}
+
+static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
+    // small cache keyed by (kernel, threads, smem)
+    struct Entry { KernelFn fn; int threads; size_t smem; int blocks; };
     static thread_local Entry cache[64];
     static thread_local int n_cache = 0;
     for (int i = 0; i < n_cache; ++i)
-        if (cache[i].fn == fn && cache[i].threads == threads) return cache[i].blocks;
+        if (cache[i].fn == fn && cache[i].threads == threads && cache[i].smem == smem)
+            return cache[i].blocks;
+    if (smem > 0) {
+        // opt in to the device maximum once per kernel (never lowered afterwards)
+        int dev = 0, mx = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&mx, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
+        cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    }
     int nb = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, 0) != cudaSuccess || nb < 1)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, smem) != cudaSuccess || nb < 1)
         nb = 1;
-    if (n_cache < 64) cache[n_cache++] = {fn, threads, nb};
+    if (n_cache < 64) cache[n_cache++] = {fn, threads, smem, nb};
     return nb;
 }
 
@@ -435,6 +685,42 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) coef |= COEF_COUT;
     if (r.op != OP_GAT && g->ew) coef |= COEF_W;
 
+    // Feature panels: when X is much larger than
+    // L2, sweep the graph once per 32*VEC-column strip so the strip of X being
+    // gathered (n_src * 32*VEC * 4 bytes) stays L2-resident while every edge
+    // pulls from it.  The per-column reduction order is unchanged, so panel
+    // mode and strip width never change a single output bit.
+    int panel = 0;
+    bool panel_off = false;
+    {
+        const double budget = 0.6 * (double)g->l2_bytes;
+        const double xbytes = 4.0 * (double)g->n_src * (double)r.ldx;
+        int mode = -1;  // auto
+        if (const char *e = getenv("TLP_PANEL")) mode = atoi(e);
+        if (mode == 0) {
+            panel = 0;
+            panel_off = true;
+        } else if (mode == 128 && vec == 4) {
+            panel = 1;
+        } else if (mode == 64 && vec >= 2) {
+            panel = 1;
+            vec = 2;
+        } else if (mode == 32) {
+            panel = 1;
+            vec = 1;
+        } else if (xbytes > budget) {
+            // measured on B200: a 128-column strip still wins when its
+            // slice of X is as large as the whole L2; narrower strips lose more to
+            // halved bytes per load than they gain in hit rate
+            if (vec == 4 && 512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
+        }
+    }
+    const int n_strips = (int)((r.F + 32 * vec - 1) / (32 * vec));
+    // Few tasks for the resident warps (small graphs): split every task into its
+    // strips as separate work items too, so all SMs get work.
+    if (!panel && !panel_off && n_strips > 1 && g->n_tasks < (int64_t)g->num_sms * 32 * 4) panel = 1;
+    if (n_strips < 2) panel = 0;
+
     AggArgs a;
     a.rowptr = g->rowptr;
     a.colidx = g->colidx;
@@ -447,7 +733,6 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.tasks = g->tasks;
     a.hub_row = g->hub_row;
     a.hub_off = g->hub_off;
-    a.hub_ticket = g->hub_ticket;
     a.ctr = reinterpret_cast<unsigned long long *>(g->ctr);
     a.done = g->ctr + 2;
     a.ldx = r.ldx;
@@ -455,20 +740,40 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.ldp = (r.F + 3) / 4 * 4;
     a.row_offset = g->row_offset;
     a.n_tasks = g->n_tasks;
+    a.n_hubs = g->n_hubs;
+    a.n_chunks = g->n_chunks;
     a.C = g->C;
     a.F = (int)r.F;
-    a.n_strips = (int)((r.F + 32 * vec - 1) / (32 * vec));
+    a.n_strips = n_strips;
+    a.panel = panel;
+    a.n_items = panel ? g->n_tasks * n_strips : g->n_tasks;
     a.norm = r.norm;
     a.eps1 = 1.0f + r.eps;
     a.slope = r.slope;
     a.scratch = nullptr;
     a.md = nullptr;
+    a.hub_ticket = nullptr;
     if (g->n_chunks > 0) {
-        size_t need = sizeof(float) * (size_t)g->n_chunks * (a.ldp + 2) + 64;
+        // scratch = [partials n_chunks x ldp][(m,den) 2 x n_chunks x panels][tickets n_hubs x panels]
+        const int np = panel ? n_strips : 1;
+        const size_t part = (size_t)g->n_chunks * a.ldp;
+        const size_t mdn = 2 * (size_t)g->n_chunks * np;
+        const size_t tick_off = (part + mdn) * sizeof(float);
+        const size_t tick_n = (size_t)g->n_hubs * np;
+        const size_t need = tick_off + tick_n * sizeof(int32_t) + 64;
+        const bool realloc_ = need > g->scratch_bytes;
         tlp_status st = ensure_scratch(g, need, s);
         if (st != TLP_OK) return st;
+        if (realloc_ || g->ticket_off != tick_off || g->ticket_n < tick_n) {
+            cudaError_t e = cudaMemsetAsync((char *)g->scratch + tick_off, 0,
+                                            tick_n * sizeof(int32_t), s);
+            if (e != cudaSuccess) return cuda_error(e, "cudaMemsetAsync(tickets)");
+            g->ticket_off = tick_off;
+            g->ticket_n = tick_n;
+        }
         a.scratch = g->scratch;
-        a.md = g->scratch + (size_t)g->n_chunks * a.ldp;
+        a.md = g->scratch + part;
+        a.hub_ticket = reinterpret_cast<int32_t *>((char *)g->scratch + tick_off);
     }
     // scheduler
     int sched = g->sched;
@@ -479,28 +784,41 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     }
     int step = g->step;
     if (step <= 0) {
-        // Alg. 1's step: enough tasks per atomic for ~32 KB of gathered rows
+        // Alg. 1's step: enough work items per atomic for ~32 KB of gathered rows
         double edges_per_task = g->n_tasks ? (double)g->nnz / (double)g->n_tasks : 1.0;
-        double bytes = edges_per_task * 4.0 * (double)r.F;
+        double width = panel ? 32.0 * vec : (double)r.F;
+        double bytes = edges_per_task * 4.0 * width;
         step = (int)std::min(32.0, std::max(1.0, std::ceil(32768.0 / std::max(bytes, 1.0))));
     }
     a.step = step;
     a.sched = sched;
 
-    KernelFn fn = vec == 4 ? pick<4>(r.op, coef) : vec == 2 ? pick<2>(r.op, coef) : pick<1>(r.op, coef);
-    const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, 16) : 8;
+    // Gather path: gathers served from an
+    // L2-resident panel are latency-light and instruction-bound -> register
+    // double buffering; gathers that stream from HBM need more bytes in flight
+    // than registers can hold -> cp.async shared-memory ring.  TLP_GATHER
+    // (reg|async) overrides the choice.
+    bool async_path = !panel && (4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes);
+    if (const char *e = getenv("TLP_GATHER")) {
+        if (!strcmp(e, "reg")) async_path = false;
+        else if (!strcmp(e, "async")) async_path = true;
+    }
+    KernelFn fn = async_path ? pick_vec<true>(vec, r.op, coef) : pick_vec<false>(vec, r.op, coef);
+    const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
+    const size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;
+    if (smem > 0 && sched == S_HARDWARE) occupancy_blocks(fn, threads, smem);  // sets attributes
     int64_t blocks;
     if (sched == S_HARDWARE) {
-        blocks = (g->n_tasks + wpc - 1) / wpc;
+        blocks = (a.n_items + wpc - 1) / wpc;
     } else {
-        blocks = (int64_t)occupancy_blocks(fn, threads) * g->num_sms;
-        int64_t need = (g->n_tasks + (int64_t)wpc * step - 1) / ((int64_t)wpc * step);
+        blocks = (int64_t)occupancy_blocks(fn, threads, smem) * g->num_sms;
+        int64_t need = (a.n_items + (int64_t)wpc * step - 1) / ((int64_t)wpc * step);
         if (blocks > need) blocks = need;  // tiny graphs: do not launch idle warps
     }
     if (blocks < 1) blocks = 1;
     if (blocks > 0x7fffffff) return set_error(TLP_ERR_UNSUPPORTED, "grid too large");
-    fn<<<(unsigned)blocks, threads, 0, s>>>(a);
+    fn<<<(unsigned)blocks, threads, smem, s>>>(a);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_agg launch");
     g->last_stream = s;

@@ -6,6 +6,7 @@
 // building beyond a row-range plan.
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <chrono>
 #include <cstring>
 #include <string>
@@ -166,7 +167,7 @@ static tlp_status dmalloc(void **p, size_t bytes, tlp_graph g) {
 static void graph_free(tlp_graph g) {
     if (!g) return;
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out,
-                    g->tasks, g->hub_row, g->hub_off, g->hub_ticket, g->ctr,
+                    g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)
         if (p) cudaFree(p);
@@ -206,13 +207,26 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
     tlp_graph g = new tlp_graph_s();
     CTRY(cudaGetDevice(&g->device));
     CTRY(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
+    {
+        int l2 = 0;
+        CTRY(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, g->device));
+        g->l2_bytes = (size_t)l2;
+    }
     g->n_dst = n_dst;
     g->n_src = n_src;
     g->nnz = nnz;
     g->row_offset = row_offset;
     g->H = (opts && opts->hub_threshold > 0) ? opts->hub_threshold : kDefaultHubThreshold;
     g->C = (opts && opts->hub_chunk > 0) ? opts->hub_chunk : kDefaultHubChunk;
-    g->K = (opts && opts->unit_edges > 0) ? opts->unit_edges : kDefaultUnitEdges;
+    if (opts && opts->unit_edges > 0) {
+        g->K = opts->unit_edges;
+    } else {
+        // enough units to give every resident warp (~SMs x 32) about four of
+        // them, at most kDefaultUnitEdges edges each.  K only groups whole rows
+        // into tasks; it never changes any row's reduction order.
+        const int64_t target = (int64_t)std::max(g->num_sms, 1) * 32 * 4;
+        g->K = std::max<int64_t>(1, std::min<int64_t>(kDefaultUnitEdges, nnz / target));
+    }
     g->last_stream = s;
     const int nsm = g->num_sms;
 
@@ -344,8 +358,6 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         g->n_hubs = n_hubs;
         TRY(dmalloc((void **)&g->hub_row, sizeof(int32_t) * n_hubs, g));
         TRY(dmalloc((void **)&g->hub_off, sizeof(int32_t) * (n_hubs + 1), g));
-        TRY(dmalloc((void **)&g->hub_ticket, sizeof(int32_t) * n_hubs, g));
-        CTRY(cudaMemsetAsync(g->hub_ticket, 0, sizeof(int32_t) * (n_hubs ? n_hubs : 1), s));
         CTRY(cudaMemsetAsync(g->hub_off, 0, sizeof(int32_t) * (n_hubs + 1), s));
         int64_t n_chunks = 0;
         if (n_hubs > 0) {

@@ -47,13 +47,14 @@ struct tlp_graph_s {
     int2 *tasks = nullptr;       // [n_tasks]
     int32_t *hub_row = nullptr;  // [n_hubs]
     int32_t *hub_off = nullptr;  // [n_hubs+1]
-    int32_t *hub_ticket = nullptr;  // [n_hubs], zero between calls
     unsigned int *ctr = nullptr;    // [2]: next task, finished warps
     int64_t n_tasks = 0, n_units = 0, n_hubs = 0, n_chunks = 0;
     int64_t regular_edges = 0;
 
-    float *scratch = nullptr;    // hub partials
+    float *scratch = nullptr;    // hub partials, GAT (m, den), hub tickets
     size_t scratch_bytes = 0;
+    size_t ticket_off = 0, ticket_n = 0;  // ticket region inside scratch (zeroed)
+    size_t l2_bytes = 0;
     size_t device_bytes = 0;
     double create_ms = 0.0;
 

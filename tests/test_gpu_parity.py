@@ -411,3 +411,45 @@ def test_config_products_gat_sampled(tlp):
     Y = g.gat(_t(X), _t(el), _t(er), synth.SLOPE, F=F)
     _check("products gat", Y[_t(rows)], oracle.gat(rp, ci, X, el, er, synth.SLOPE, rows=rows, F=F))
     g.close()
+
+
+def test_panel_modes_bitwise(tlp, monkeypatch):
+    """Feature-panel sweeps (any strip width) give bitwise the task-major result."""
+    n = 3000
+    rp, ci = synth.chung_lu(n, 80000, 0.5, 13, device="cpu")
+    F, ld = 300, 300
+    Xh = synth.features(n, F, ld, seed=5)
+    X = _t(Xh)
+    el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    outs = {}
+    for mode in ("0", "32", "64", "128", "-1"):
+        monkeypatch.setenv("TLP_PANEL", mode)
+        outs[mode] = (g.gcn(X, "both").clone(), g.gin(X, 0.1).clone(), g.gat(X, el, er, 0.2).clone())
+    for mode in outs:
+        for a, b in zip(outs[mode], outs["0"]):
+            assert torch.equal(a, b), mode
+    _check("panel gcn", outs["64"][0], oracle.gcn(rp, ci, Xh, "both"))
+    g.close()
+
+
+@pytest.mark.parametrize("F,ld", [(100, 100), (300, 300), (37, 40), (5, 6)])
+def test_gather_paths_bitwise(tlp, monkeypatch, F, ld):
+    """Register double-buffered and cp.async shared-memory gathers agree bit for bit."""
+    n = 2500
+    rp, ci = synth.chung_lu(n, 60000, 0.5, 17, device="cpu")
+    Xh = synth.features(n, F, ld, seed=6)
+    X = _t(Xh)
+    el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
+    ew = _t(synth.edge_weights(len(ci), 4))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=80, hub_chunk=40))
+    gw = tlp.Graph(_t(rp), _t(ci), edge_weight=ew, opts=dict(hub_threshold=80, hub_chunk=40))
+    outs = {}
+    for path in ("reg", "async"):
+        monkeypatch.setenv("TLP_GATHER", path)
+        outs[path] = [g.gcn(X, "both", F=F).clone(), g.gin(X, 0.1, F=F).clone(),
+                      g.gat(X, el, er, 0.2, F=F).clone(), gw.gcn(X, "right", F=F).clone()]
+    for a, b in zip(outs["reg"], outs["async"]):
+        assert torch.equal(a, b)
+    _check("async gat", outs["async"][2], oracle.gat(rp, ci, Xh, synth.normal(n, 1), synth.normal(n, 2), 0.2, F=F))
+    g.close(); gw.close()
