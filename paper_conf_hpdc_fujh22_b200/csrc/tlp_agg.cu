@@ -51,7 +51,7 @@ constexpr unsigned FULL = 0xffffffffu;
 #define TLP_MAXT 256   // threads per CTA at most (8 warps)
 #endif
 #ifndef TLP_MINB
-#define TLP_MINB 4     // register path: 4 CTAs/SM -> 64 registers, 32 warps/SM
+#define TLP_MINB 3     // register path: 3 CTAs/SM -> <= 85 registers, 24 warps/SM
 #endif
 #ifndef TLP_MINB_ASYNC
 #define TLP_MINB_ASYNC 3  // async path: 3 CTAs/SM (ring = 3 x 64 KB of shared memory)
@@ -151,133 +151,183 @@ __device__ __forceinline__ float warp_sum(float v) {
     return v;
 }
 
-// Issue the gathers of edges [j, j+U) of the current 32-edge chunk (lane k of
-// the chunk holds source u and coefficient c of edge k).
-template <int VEC, int U, bool HASC>
-__device__ __forceinline__ void issue_group(const float *__restrict__ Xc, unsigned ldx, int j, int n,
-                                            bool active, int u_l, float c_l, Vec<VEC> (&xv)[U],
+// Gather address of source row u: base + u * row_bytes, one IMAD.WIDE.U32
+// (32x32 -> 64-bit multiply-add); base = X + column (a byte pointer).
+__device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, unsigned row_bytes) {
+    return reinterpret_cast<const float *>(base + (unsigned long long)u * row_bytes);
+}
+
+// ---- canonical reduction order ---------------------------------------------
+// Every path reduces a row (or a hub chunk) as TWO interleaved chains: the
+// edges at even and at odd positions (relative to the row / chunk start, in
+// CSR order), each accumulated sequentially with fmaf, then added as
+// even + odd.  Hub chunks start at even offsets (C is even) and are merged in
+// chunk order.  The register path (full warp or half-warp PAIR), the cp.async
+// path, every strip width, scheduler and partition produce exactly this
+// order, hence bitwise-identical results.
+//
+// Lane -> edge mapping inside a 32-edge chunk, for step j, group slot k:
+//   full warp: every lane gathers edge j+k for its 4 columns (chain (j+k)&1)
+//   PAIR     : lanes 0-15 gather edge 2(j+k), lanes 16-31 edge 2(j+k)+1, over
+//              64 columns, so a warp-wide LDG.128 still moves 512 bytes while
+//              the strip of X is half as wide (each half-warp is one chain).
+
+template <int VEC, int U, bool HASC, bool PAIR, bool CLAMP>
+__device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes, int j, int n,
+                                            int half, int u_l, float c_l, Vec<VEC> (&xv)[U],
                                             float (&ck)[U]) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-        const int jj = j + k;
-        const int u = __shfl_sync(FULL, u_l, jj & 31);
-        if constexpr (HASC) ck[k] = __shfl_sync(FULL, c_l, jj & 31);
-        if (jj < n && active) {
-            xv[k] = ld_vec<VEC>(Xc + (size_t)((unsigned)u) * ldx);  // IMAD.WIDE.U32
-        } else {
-#pragma unroll
-            for (int c = 0; c < VEC; ++c) xv[k].v[c] = 0.f;
-        }
+        int p = PAIR ? 2 * (j + k) + half : j + k;
+        if constexpr (CLAMP) p = min(p, n - 1);  // duplicate of a line in flight
+        const unsigned u = (unsigned)__shfl_sync(FULL, u_l, p);
+        if constexpr (HASC) ck[k] = __shfl_sync(FULL, c_l, p);
+        xv[k] = ld_vec<VEC>(row_ptr(base, u, row_bytes));
     }
 }
 
-// Accumulate a gathered group in CSR order.
-template <int VEC, int U, bool HASC>
-__device__ __forceinline__ void consume_group(int j, int n, const Vec<VEC> (&xv)[U],
-                                              const float (&ck)[U], Vec<VEC> &acc) {
+// PHASE: parity of the group's first step (the caller's j is a multiple of 2U).
+template <int VEC, int U, bool HASC, bool PAIR, bool GUARD, int PHASE>
+__device__ __forceinline__ void consume_group(int j, int n, int half, const Vec<VEC> (&xv)[U],
+                                              const float (&ck)[U], Vec<VEC> (&ac)[2]) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-        if (j + k < n) {
+        const int p = PAIR ? 2 * (j + k) + half : j + k;
+        constexpr int dummy = 0;
+        (void)dummy;
+        const int ch = PAIR ? 0 : ((PHASE + k) & 1);
+        if (!GUARD || p < n) {
 #pragma unroll
             for (int c = 0; c < VEC; ++c) {
-                if constexpr (HASC) acc.v[c] = fmaf(ck[k], xv[k].v[c], acc.v[c]);
-                else acc.v[c] += xv[k].v[c];
+                if constexpr (HASC) ac[ch].v[c] = fmaf(ck[k], xv[k].v[c], ac[ch].v[c]);
+                else ac[ch].v[c] += xv[k].v[c];
             }
         }
     }
 }
 
 // Reduce the edges [e0, e1) of one destination row for the feature vector at
-// `col` (a6 / a7).  GCN/GIN: acc = sum_e c_e X[u_e] in CSR order.  GAT: online
-// softmax state (m, den, acc = sum_e exp(s_e - m) X[u_e]).
+// `col` (a6 / a7).  GCN/GIN: acc = sum_e c_e X[u_e] (two-chain order above).
+// GAT: online softmax state (m, den, acc = sum_e exp(s_e - m) X[u_e]).
 //
 // Latency hiding (the kernel is bound by bytes in flight, not by arithmetic):
 //  * edge indices are loaded 32 at a time by the lanes two chunks ahead, and
 //    the index-dependent values (c_out[u] or el[u]) one chunk ahead, so the
 //    gathers of a chunk never wait on an index load;
 //  * the gathers of a chunk are issued in double-buffered groups of U source
-//    rows: the next group is in flight while the current one is accumulated.
-template <int VEC, int OP, int COEF, int U>
+//    rows: the next group is in flight while the current one is accumulated;
+//    full 32-edge chunks are fully unrolled (compile-time shuffle lanes).
+template <int VEC, int OP, int COEF, int U, bool PAIR>
 __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64_t e1,
                                              int col, bool active, float er_v, int lane,
                                              Vec<VEC> &acc, float &m, float &den) {
     constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT);
     constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);  // index-dependent value
-    const float *__restrict__ Xc = a.X + col;
+    constexpr int STEPS = PAIR ? 16 : 32;  // gather steps of a full chunk
+    // lanes past F read column 0 (a valid address); their results are never stored
+    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
+    const unsigned row_bytes = (unsigned)a.ldx * 4u;
     const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
-    const unsigned ldx = (unsigned)a.ldx;
     // 32-bit edge offsets relative to e0 (a row or hub chunk has < 2^31 edges)
     const int32_t *__restrict__ ci = a.colidx + e0;
     const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
     const int len = (int)(e1 - e0);
-    if (len <= 0) return;
-    int off = 0;
-    int n0 = min(32, len);
-    int n1 = min(32, len - 32);
-    int u0 = 0, u1 = 0;
-    float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
-    if (lane < n0) {
-        u0 = __ldg(ci + lane);
-        if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
-    }
-    if (lane < n1) {
-        u1 = __ldg(ci + 32 + lane);
-        if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
-    }
-    if constexpr (DEP)
-        if (lane < n0) d0 = __ldg(dep + u0);
-    while (true) {
-        // two chunks ahead: indices; one chunk ahead: index-dependent values
-        const int n2 = min(32, len - off - 64);
-        int u2 = 0;
-        float w2 = 1.f;
-        if (lane < n2) {
-            u2 = __ldg(ci + off + 64 + lane);
-            if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
+    const int half = PAIR ? (lane >> 4) : 0;
+    Vec<VEC> ac[2];
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) ac[0].v[c] = ac[1].v[c] = 0.f;
+    if (len > 0) {
+        int off = 0;
+        int n0 = min(32, len);
+        int n1 = min(32, len - 32);
+        int u0 = 0, u1 = 0;
+        float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
+        if (lane < n0) {
+            u0 = __ldg(ci + lane);
+            if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
+        }
+        if (lane < n1) {
+            u1 = __ldg(ci + 32 + lane);
+            if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
         }
         if constexpr (DEP)
-            if (lane < n1) d1 = __ldg(dep + u1);
-        // coefficients of the current chunk
-        float c_l = 1.f;
-        if constexpr (OP == OP_GAT) {
-            float s = -INFINITY;
-            if (lane < n0) {
-                const float t = d0 + er_v;
-                s = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
+            if (lane < n0) d0 = __ldg(dep + u0);
+        while (true) {
+            // two chunks ahead: indices; one chunk ahead: index-dependent values
+            const int n2 = min(32, len - off - 64);
+            int u2 = 0;
+            float w2 = 1.f;
+            if (lane < n2) {
+                u2 = __ldg(ci + off + 64 + lane);
+                if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
             }
-            const float m_new = fmaxf(m, warp_max(s));
-            const float scale = __expf(m - m_new);  // m = -inf -> 0
-            c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
-            den = fmaf(den, scale, warp_sum(c_l));
+            if constexpr (DEP)
+                if (lane < n1) d1 = __ldg(dep + u1);
+            // coefficients of the current chunk
+            float c_l = 1.f;
+            if constexpr (OP == OP_GAT) {
+                float s = -INFINITY;
+                if (lane < n0) {
+                    const float t = d0 + er_v;
+                    s = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
+                }
+                const float m_new = fmaxf(m, warp_max(s));
+                const float scale = __expf(m - m_new);  // m = -inf -> 0
+                c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
+                den = fmaf(den, scale, warp_sum(c_l));
 #pragma unroll
-            for (int c = 0; c < VEC; ++c) acc.v[c] *= scale;
-            m = m_new;
-        } else {
-            if constexpr (COEF & COEF_COUT) c_l = d0;
-            if constexpr (COEF & COEF_W) c_l *= w0;
-        }
-        // gathers: double-buffered groups of U rows
-        {
+                for (int c = 0; c < VEC; ++c) {
+                    ac[0].v[c] *= scale;
+                    ac[1].v[c] *= scale;
+                }
+                m = m_new;
+            } else {
+                if constexpr (COEF & COEF_COUT) c_l = d0;
+                if constexpr (COEF & COEF_W) c_l *= w0;
+            }
             Vec<VEC> xa[U], xb[U];
             float ca[U], cb[U];
-            issue_group<VEC, U, HASC>(Xc, ldx, 0, n0, active, u0, c_l, xa, ca);
-            for (int j = 0; j < n0; j += 2 * U) {
-                issue_group<VEC, U, HASC>(Xc, ldx, j + U, n0, active, u0, c_l, xb, cb);
-                consume_group<VEC, U, HASC>(j, n0, xa, ca, acc);
-                issue_group<VEC, U, HASC>(Xc, ldx, j + 2 * U, n0, active, u0, c_l, xa, ca);
-                consume_group<VEC, U, HASC>(j + U, n0, xb, cb, acc);
+            if (n0 == 32) {
+                // full chunk: fully unrolled, compile-time shuffle lanes, no guards
+                issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, 0, 32, half, u0, c_l, xa, ca);
+#pragma unroll
+                for (int j = 0; j < STEPS; j += 2 * U) {
+                    issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, j + U, 32, half, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, PAIR, false, 0>(j, 32, half, xa, ca, ac);
+                    if (j + 2 * U < STEPS)
+                        issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, j + 2 * U, 32, half, u0, c_l, xa, ca);
+                    consume_group<VEC, U, HASC, PAIR, false, U>(j + U, 32, half, xb, cb, ac);
+                }
+            } else {
+                // partial chunk (n0 is warp-uniform: the guards never diverge)
+                const int steps = PAIR ? (n0 + 1) >> 1 : n0;
+                issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, 0, n0, half, u0, c_l, xa, ca);
+                for (int j = 0; j < steps; j += 2 * U) {
+                    const bool more = j + U < steps;
+                    if (more) issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, j + U, n0, half, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, PAIR, true, 0>(j, n0, half, xa, ca, ac);
+                    if (j + 2 * U < steps)
+                        issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, j + 2 * U, n0, half, u0, c_l, xa, ca);
+                    if (more) consume_group<VEC, U, HASC, PAIR, true, U>(j + U, n0, half, xb, cb, ac);
+                }
             }
+            if (n1 <= 0) break;
+            off += 32;
+            n0 = n1; n1 = n2;
+            u0 = u1; u1 = u2;
+            w0 = w1; w1 = w2;
+            d0 = d1;
         }
-        if (n1 <= 0) break;
-        off += 32;
-        n0 = n1; n1 = n2;
-        u0 = u1; u1 = u2;
-        w0 = w1; w1 = w2;
-        d0 = d1;
+    }
+    // even + odd (in PAIR mode the odd chain lives in the other half-warp)
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) {
+        if constexpr (PAIR) acc.v[c] = ac[0].v[c] + __shfl_xor_sync(FULL, ac[0].v[c], 16);
+        else acc.v[c] = ac[0].v[c] + ac[1].v[c];
     }
 }
 
-// ---- asynchronous-copy variant (TLP_ASYNC) --------------------------------
+// ---- asynchronous-copy path ------------------------------------------------
 // The gathered rows land in a per-warp shared-memory ring through cp.async
 // (LDGSTS, L2 -> SMEM, bypassing L1 and the register file), D edges deep.  Bytes
 // in flight then cost no registers, so occupancy and depth are decoupled.
@@ -307,108 +357,124 @@ __device__ __forceinline__ float *warp_ring() {
     return tlp_smem + (size_t)w * TLP_DEPTH * 32 * VEC;
 }
 
+template <int VEC, bool HASC>
+__device__ __forceinline__ void acc_from_smem(const float *src, float cj, Vec<VEC> &acc) {
+    if constexpr (VEC == 4) {
+        const float4 x = *reinterpret_cast<const float4 *>(src);
+        if constexpr (HASC) {
+            acc.v[0] = fmaf(cj, x.x, acc.v[0]); acc.v[1] = fmaf(cj, x.y, acc.v[1]);
+            acc.v[2] = fmaf(cj, x.z, acc.v[2]); acc.v[3] = fmaf(cj, x.w, acc.v[3]);
+        } else {
+            acc.v[0] += x.x; acc.v[1] += x.y; acc.v[2] += x.z; acc.v[3] += x.w;
+        }
+    } else {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) {
+            if constexpr (HASC) acc.v[c] = fmaf(cj, src[c], acc.v[c]);
+            else acc.v[c] += src[c];
+        }
+    }
+}
+
 template <int VEC, int OP, int COEF, int U>
 __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0, int64_t e1,
                                                    int col, bool active, float er_v, int lane,
                                                    Vec<VEC> &acc, float &m, float &den) {
     constexpr int D = TLP_DEPTH;
+    constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT);
     constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);
-    const float *__restrict__ Xc = a.X + col;
+    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
+    const unsigned row_bytes = (unsigned)a.ldx * 4u;
     const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
-    const unsigned ldx = (unsigned)a.ldx;
     const int32_t *__restrict__ ci = a.colidx + e0;
     const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
     const int len = (int)(e1 - e0);
-    if (len <= 0) return;
-    float *ring = warp_ring<VEC>() + lane * VEC;
-    int off = 0;
-    int n0 = min(32, len);
-    int n1 = min(32, len - 32);
-    int u0 = 0, u1 = 0;
-    float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
-    if (lane < n0) {
-        u0 = __ldg(ci + lane);
-        if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
-    }
-    if (lane < n1) {
-        u1 = __ldg(ci + 32 + lane);
-        if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
-    }
-    if constexpr (DEP)
-        if (lane < n0) d0 = __ldg(dep + u0);
-    // prologue: edges 0 .. D-2 in flight
+    Vec<VEC> ae, ao;  // even / odd chains (canonical order)
 #pragma unroll
-    for (int k = 0; k < D - 1; ++k) {
-        const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
-        cp_async_vec<VEC>(ring + k * 32 * VEC, Xc + (size_t)((unsigned)uk) * ldx, active && k < len);
-        cp_async_commit();
-    }
-    int slot = 0;  // ring slot of edge `off + j`
-    while (true) {
-        const int n2 = min(32, len - off - 64);
-        int u2 = 0;
-        float w2 = 1.f;
-        if (lane < n2) {
-            u2 = __ldg(ci + off + 64 + lane);
-            if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
+    for (int c = 0; c < VEC; ++c) ae.v[c] = ao.v[c] = 0.f;
+    if (len > 0) {
+        float *ring = warp_ring<VEC>() + lane * VEC;
+        int off = 0;
+        int n0 = min(32, len);
+        int n1 = min(32, len - 32);
+        int u0 = 0, u1 = 0;
+        float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
+        if (lane < n0) {
+            u0 = __ldg(ci + lane);
+            if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
+        }
+        if (lane < n1) {
+            u1 = __ldg(ci + 32 + lane);
+            if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
         }
         if constexpr (DEP)
-            if (lane < n1) d1 = __ldg(dep + u1);
-        float c_l = 1.f;
-        if constexpr (OP == OP_GAT) {
-            float s = -INFINITY;
-            if (lane < n0) {
-                const float t = d0 + er_v;
-                s = t >= 0.f ? t : a.slope * t;
-            }
-            const float m_new = fmaxf(m, warp_max(s));
-            const float scale = __expf(m - m_new);
-            c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
-            den = fmaf(den, scale, warp_sum(c_l));
+            if (lane < n0) d0 = __ldg(dep + u0);
+        // prologue: edges 0 .. D-2 in flight
 #pragma unroll
-            for (int c = 0; c < VEC; ++c) acc.v[c] *= scale;
-            m = m_new;
-        } else {
-            if constexpr (COEF & COEF_COUT) c_l = d0;
-            if constexpr (COEF & COEF_W) c_l *= w0;
-        }
-        for (int j = 0; j < n0; ++j) {
-            // issue edge j + D - 1 (in this chunk or the next one)
-            const int jj = j + D - 1;
-            const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
-            const bool valid = (off + jj) < len;
-            int ws = slot + D - 1;
-            if (ws >= D) ws -= D;
-            cp_async_vec<VEC>(ring + ws * 32 * VEC, Xc + (size_t)((unsigned)ui) * ldx, active && valid);
+        for (int k = 0; k < D - 1; ++k) {
+            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
+            cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
             cp_async_commit();
-            cp_async_wait<D - 1>();
-            const float cj = __shfl_sync(FULL, c_l, j);
-            const float *src = ring + slot * 32 * VEC;
-            if constexpr (VEC == 4) {
-                const float4 x = *reinterpret_cast<const float4 *>(src);
-                if constexpr (COEF != COEF_NONE || OP == OP_GAT) {
-                    acc.v[0] = fmaf(cj, x.x, acc.v[0]); acc.v[1] = fmaf(cj, x.y, acc.v[1]);
-                    acc.v[2] = fmaf(cj, x.z, acc.v[2]); acc.v[3] = fmaf(cj, x.w, acc.v[3]);
-                } else {
-                    acc.v[0] += x.x; acc.v[1] += x.y; acc.v[2] += x.z; acc.v[3] += x.w;
+        }
+        int slot = 0;  // ring slot of edge `off + j`
+        while (true) {
+            const int n2 = min(32, len - off - 64);
+            int u2 = 0;
+            float w2 = 1.f;
+            if (lane < n2) {
+                u2 = __ldg(ci + off + 64 + lane);
+                if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
+            }
+            if constexpr (DEP)
+                if (lane < n1) d1 = __ldg(dep + u1);
+            float c_l = 1.f;
+            if constexpr (OP == OP_GAT) {
+                float s = -INFINITY;
+                if (lane < n0) {
+                    const float t = d0 + er_v;
+                    s = t >= 0.f ? t : a.slope * t;
                 }
-            } else {
+                const float m_new = fmaxf(m, warp_max(s));
+                const float scale = __expf(m - m_new);
+                c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
+                den = fmaf(den, scale, warp_sum(c_l));
 #pragma unroll
                 for (int c = 0; c < VEC; ++c) {
-                    if constexpr (COEF != COEF_NONE || OP == OP_GAT) acc.v[c] = fmaf(cj, src[c], acc.v[c]);
-                    else acc.v[c] += src[c];
+                    ae.v[c] *= scale;
+                    ao.v[c] *= scale;
                 }
+                m = m_new;
+            } else {
+                if constexpr (COEF & COEF_COUT) c_l = d0;
+                if constexpr (COEF & COEF_W) c_l *= w0;
             }
-            if (++slot == D) slot = 0;
+            for (int j = 0; j < n0; ++j) {
+                // issue edge j + D - 1 (in this chunk or the next one)
+                const int jj = j + D - 1;
+                const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
+                const bool valid = (off + jj) < len;
+                int ws = slot + D - 1;
+                if (ws >= D) ws -= D;
+                cp_async_vec<VEC>(ring + ws * 32 * VEC, row_ptr(base, (unsigned)ui, row_bytes), active && valid);
+                cp_async_commit();
+                cp_async_wait<D - 1>();
+                const float cj = __shfl_sync(FULL, c_l, j);
+                // chunks start at even offsets: the parity of j is the edge's parity
+                if (j & 1) acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, cj, ao);
+                else acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, cj, ae);
+                if (++slot == D) slot = 0;
+            }
+            if (n1 <= 0) break;
+            off += 32;
+            n0 = n1; n1 = n2;
+            u0 = u1; u1 = u2;
+            w0 = w1; w1 = w2;
+            d0 = d1;
         }
-        if (n1 <= 0) break;
-        off += 32;
-        n0 = n1; n1 = n2;
-        u0 = u1; u1 = u2;
-        w0 = w1; w1 = w2;
-        d0 = d1;
+        cp_async_wait<0>();  // drain the (empty) tail groups before the ring is reused
     }
-    cp_async_wait<0>();  // drain the (empty) tail groups before the ring is reused
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
 }
 
 // Epilogue (a9) for a full row reduction.
@@ -439,8 +505,19 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_
     return y;
 }
 
+// Column of this lane's 4-float vector in strip s (PAIR: 64-column strips,
+// lanes l and l+16 share a column), and whether this lane stores it.
+template <int VEC, bool PAIR>
+__device__ __forceinline__ int strip_col(int s, int lane) {
+    return PAIR ? s * 64 + (lane & 15) * 4 : s * 32 * VEC + lane * VEC;
+}
+template <bool PAIR>
+__device__ __forceinline__ bool stores(int lane) {
+    return !PAIR || lane < 16;
+}
+
 // A regular work unit: whole rows [r0, r1), feature strips [s0, s1).
-template <int VEC, int OP, int COEF, int U, bool ASYNC>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
 __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0, int s1,
                                         int lane) {
     for (int rb = r0; rb < r1; rb += 31) {
@@ -459,7 +536,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
             const int64_t r = rb + k;
             float *yrow = a.Y + r * a.ldy;
             for (int s = s0; s < s1; ++s) {
-                const int col = s * 32 * VEC + lane * VEC;
+                const int col = strip_col<VEC, PAIR>(s, lane);
                 const bool active = col < a.F;
                 Vec<VEC> acc;
 #pragma unroll
@@ -468,9 +545,9 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                 if constexpr (ASYNC)
                     reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
                 else
-                    reduce_edges<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+                    reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den);
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
-                if (active) st_row<VEC>(yrow, col, a.F, y);
+                if (active && stores<PAIR>(lane)) st_row<VEC>(yrow, col, a.F, y);
             }
         }
     }
@@ -479,7 +556,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
 // One C-edge chunk of hub h (a8), feature strips [s0, s1).  The last chunk of
 // the hub to finish these strips merges all its partials in chunk order and
 // writes the row.  Tickets (and GAT (m, den) pairs) are kept per panel s0.
-template <int VEC, int OP, int COEF, int U, bool ASYNC>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
 __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int s0, int s1,
                                              int lane) {
     const int r = __ldg(a.hub_row + h);
@@ -494,7 +571,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     float *md = a.md + 2 * (int64_t)s0 * a.n_chunks;  // this panel's (m, den) pairs
     int32_t *ticket = a.hub_ticket + (int64_t)s0 * a.n_hubs + h;
     for (int s = s0; s < s1; ++s) {
-        const int col = s * 32 * VEC + lane * VEC;
+        const int col = strip_col<VEC, PAIR>(s, lane);
         const bool active = col < a.F;
         Vec<VEC> acc;
 #pragma unroll
@@ -503,8 +580,8 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         if constexpr (ASYNC)
                     reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
                 else
-                    reduce_edges<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
-        if (active) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
+                    reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+        if (active && stores<PAIR>(lane)) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
         if constexpr (OP == OP_GAT)
             if (s == s0 && lane == 0) {
                 md[2 * (int64_t)slot] = m;
@@ -529,7 +606,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         }
     }
     for (int s = s0; s < s1; ++s) {
-        const int col = s * 32 * VEC + lane * VEC;
+        const int col = strip_col<VEC, PAIR>(s, lane);
         const bool active = col < a.F;
         Vec<VEC> acc;
 #pragma unroll
@@ -548,7 +625,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
             }
         }
         Vec<VEC> y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
-        if (active) st_row<VEC>(yrow, col, a.F, y);
+        if (active && stores<PAIR>(lane)) st_row<VEC>(yrow, col, a.F, y);
     }
     if (lane == 0) *ticket = 0;  // self-reset for the next launch
 }
@@ -556,7 +633,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
 // Work item i: task-major (all strips of task i) or, in panel mode, strip
 // s = i / n_tasks of task i % n_tasks, so that all warps sweep one L2-resident
 // feature panel of X at a time.
-template <int VEC, int OP, int COEF, int U, bool ASYNC>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
 __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
     int64_t t = i;
     int s0 = 0, s1 = a.n_strips;
@@ -566,16 +643,16 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
         s1 = s0 + 1;
     }
     const int2 tk = a.tasks[t];
-    if (tk.y >= 0) do_unit<VEC, OP, COEF, U, ASYNC>(a, tk.x, tk.y, s0, s1, lane);
-    else do_hub_chunk<VEC, OP, COEF, U, ASYNC>(a, tk.x, -tk.y - 1, s0, s1, lane);
+    if (tk.y >= 0) do_unit<VEC, OP, COEF, U, ASYNC, PAIR>(a, tk.x, tk.y, s0, s1, lane);
+    else do_hub_chunk<VEC, OP, COEF, U, ASYNC, PAIR>(a, tk.x, -tk.y - 1, s0, s1, lane);
 }
 
-template <int VEC, int OP, int COEF, int U, bool ASYNC>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
 __global__ void __launch_bounds__(TLP_MAXT, ASYNC ? TLP_MINB_ASYNC : TLP_MINB) k_agg(const AggArgs a) {
     const int lane = threadIdx.x & 31;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (a.sched == S_HARDWARE) {  // one warp per item
-        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC>(a, wid, lane);
+        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC, PAIR>(a, wid, lane);
         return;
     }
     const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -585,7 +662,7 @@ __global__ void __launch_bounds__(TLP_MAXT, ASYNC ? TLP_MINB_ASYNC : TLP_MINB) k
         unsigned long long v = 0;
         if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned long long)a.step);
         const int64_t tend = min(t + a.step, a.n_items);
-        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC>(a, tt, lane);
+        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, PAIR>(a, tt, lane);
         if (a.sched == S_DYNAMIC) t = stride + (int64_t)__shfl_sync(FULL, v, 0);
         else t += stride;
     }
@@ -606,25 +683,30 @@ constexpr int kU = TLP_U;  // source rows per gather group (2 groups in flight)
 
 typedef void (*KernelFn)(const AggArgs);
 
-template <int VEC, bool ASYNC>
+template <int VEC, bool ASYNC, bool PAIR>
 static KernelFn pick(int op, int coef) {
     if (op == OP_GCN) {
         switch (coef) {
-            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU, ASYNC>;
-            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU, ASYNC>;
-            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU, ASYNC>;
-            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU, ASYNC>;
+            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU, ASYNC, PAIR>;
+            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU, ASYNC, PAIR>;
+            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU, ASYNC, PAIR>;
+            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU, ASYNC, PAIR>;
         }
     }
     if (op == OP_GIN)
-        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC>
-                             : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC>;
-    return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC>;
+        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC, PAIR>
+                             : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC, PAIR>;
+    return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC, PAIR>;
 }
 
-template <bool ASYNC>
-static KernelFn pick_vec(int vec, int op, int coef) {
-    return vec == 4 ? pick<4, ASYNC>(op, coef) : vec == 2 ? pick<2, ASYNC>(op, coef) : pick<1, ASYNC>(op, coef);
+// gather path: 0 register (full warp), 1 cp.async ring, 2 register half-warp PAIR (VEC = 4)
+static KernelFn pick_kernel(int path, int vec, int op, int coef) {
+    if (path == 2) return pick<4, false, true>(op, coef);
+    if (path == 1)
+        return vec == 4 ? pick<4, true, false>(op, coef) : vec == 2 ? pick<2, true, false>(op, coef)
+                                                                   : pick<1, true, false>(op, coef);
+    return vec == 4 ? pick<4, false, false>(op, coef) : vec == 2 ? pick<2, false, false>(op, coef)
+                                                                 : pick<1, false, false>(op, coef);
 }
 
 static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
@@ -681,16 +763,27 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (r.ldx % 4 == 0 && r.ldy % 4 == 0 && aligned(r.X, 16) && aligned(r.Y, 16)) vec = 4;
     else if (r.ldx % 2 == 0 && r.ldy % 2 == 0 && aligned(r.X, 8) && aligned(r.Y, 8)) vec = 2;
 
+    // Edge coefficients.  GCN BOTH streams the per-edge product
+    // c_out[colidx[e]] * w_e precomputed at create (the same fp32 value the
+    // kernel would form, so bitwise identical), instead of a dependent gather.
     int coef = COEF_NONE;
-    if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) coef |= COEF_COUT;
-    if (r.op != OP_GAT && g->ew) coef |= COEF_W;
+    const float *ew = g->ew;
+    if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) {
+        if (g->ew_both) { ew = g->ew_both; coef |= COEF_W; }
+        else { coef |= COEF_COUT; if (g->ew) coef |= COEF_W; }
+    } else if (r.op != OP_GAT && g->ew) {
+        coef |= COEF_W;
+    }
 
     // Feature panels: when X is much larger than
-    // L2, sweep the graph once per 32*VEC-column strip so the strip of X being
-    // gathered (n_src * 32*VEC * 4 bytes) stays L2-resident while every edge
-    // pulls from it.  The per-column reduction order is unchanged, so panel
+    // L2, sweep the graph once per column strip so the strip of X being
+    // gathered (n_src x strip width x 4 bytes) stays L2-resident while every
+    // edge pulls from it.  Strips are 64 columns gathered by half-warps (PAIR:
+    // lanes 0-15 and 16-31 take consecutive edges, LDG.128 each) when that
+    // slice fits in 60% of L2, else 128 columns (full warp, LDG.128).  The
+    // reduction order is the canonical two-chain order in every case, so panel
     // mode and strip width never change a single output bit.
-    int panel = 0;
+    int panel = 0, pair = 0;
     bool panel_off = false;
     {
         const double budget = 0.6 * (double)g->l2_bytes;
@@ -698,24 +791,26 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         int mode = -1;  // auto
         if (const char *e = getenv("TLP_PANEL")) mode = atoi(e);
         if (mode == 0) {
-            panel = 0;
             panel_off = true;
         } else if (mode == 128 && vec == 4) {
             panel = 1;
-        } else if (mode == 64 && vec >= 2) {
+        } else if (mode == 64 && vec == 4) {
             panel = 1;
-            vec = 2;
+            pair = 1;
+        } else if (mode == 64 && vec == 2) {
+            panel = 1;
         } else if (mode == 32) {
             panel = 1;
             vec = 1;
-        } else if (xbytes > budget) {
-            // measured on B200: a 128-column strip still wins when its
-            // slice of X is as large as the whole L2; narrower strips lose more to
-            // halved bytes per load than they gain in hit rate
-            if (vec == 4 && 512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
+        } else if (xbytes > budget && vec == 4) {
+            // GAT recomputes its scores and online-softmax state per strip, so it
+            // keeps the wider 128-column strips (measured)
+            if (r.op != OP_GAT && 256.0 * g->n_src <= budget) { panel = 1; pair = 1; }
+            else if (512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
         }
     }
-    const int n_strips = (int)((r.F + 32 * vec - 1) / (32 * vec));
+    const int strip_w = pair ? 64 : 32 * vec;
+    const int n_strips = (int)((r.F + strip_w - 1) / strip_w);
     // Few tasks for the resident warps (small graphs): split every task into its
     // strips as separate work items too, so all SMs get work.
     if (!panel && !panel_off && n_strips > 1 && g->n_tasks < (int64_t)g->num_sms * 32 * 4) panel = 1;
@@ -724,7 +819,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     AggArgs a;
     a.rowptr = g->rowptr;
     a.colidx = g->colidx;
-    a.ew = g->ew;
+    a.ew = ew;
     a.c_out = g->c_out;
     a.X = r.X;
     a.Y = r.Y;
@@ -786,24 +881,26 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (step <= 0) {
         // Alg. 1's step: enough work items per atomic for ~32 KB of gathered rows
         double edges_per_task = g->n_tasks ? (double)g->nnz / (double)g->n_tasks : 1.0;
-        double width = panel ? 32.0 * vec : (double)r.F;
+        double width = panel ? (double)strip_w : (double)r.F;
         double bytes = edges_per_task * 4.0 * width;
         step = (int)std::min(32.0, std::max(1.0, std::ceil(32768.0 / std::max(bytes, 1.0))));
     }
     a.step = step;
     a.sched = sched;
 
-    // Gather path (DESIGN.md "Two gather paths"): gathers served from an
+    // Gather path (DESIGN.md "Gather paths"): gathers served from an
     // L2-resident panel are latency-light and instruction-bound -> register
-    // double buffering; gathers that stream from HBM need more bytes in flight
-    // than registers can hold -> cp.async shared-memory ring.  TLP_GATHER
-    // (reg|async) overrides the choice.
+    // double buffering (full warp, or PAIR half-warps for 64-column strips);
+    // gathers that stream from HBM need more bytes in flight than registers can
+    // hold -> cp.async shared-memory ring.  TLP_GATHER (reg|async) overrides.
     bool async_path = !panel && (4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes);
     if (const char *e = getenv("TLP_GATHER")) {
         if (!strcmp(e, "reg")) async_path = false;
         else if (!strcmp(e, "async")) async_path = true;
     }
-    KernelFn fn = async_path ? pick_vec<true>(vec, r.op, coef) : pick_vec<false>(vec, r.op, coef);
+    if (pair) async_path = false;
+    const int path = pair ? 2 : (async_path ? 1 : 0);
+    KernelFn fn = pick_kernel(path, vec, r.op, coef);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
     const size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;

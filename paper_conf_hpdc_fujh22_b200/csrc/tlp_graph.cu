@@ -81,6 +81,18 @@ __global__ void k_norm(const int32_t *__restrict__ out_deg, int64_t n,
     }
 }
 
+// Per-edge GCN-BOTH coefficient c_out[colidx[e]] * w_e (a2): a coalesced
+// stream for the aggregation instead of a dependent gather of c_out.
+__global__ void k_edge_both(const int32_t *__restrict__ colidx, const float *__restrict__ ew,
+                            const float *__restrict__ c_out, int64_t nnz, float *__restrict__ out) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        float c = c_out[colidx[e]];
+        if (ew) c *= ew[e];
+        out[e] = c;
+    }
+}
+
 // Plan flags (a3).  Row r starts a work unit iff it is row 0, a hub, follows a
 // hub, or a multiple of K edges falls in (rowptr[r-1], rowptr[r]] -- i.e. r is
 // lower_bound(rowptr, u*K) for some u.  Hubs (deg > H) become chunk tasks.
@@ -166,7 +178,7 @@ static tlp_status dmalloc(void **p, size_t bytes, tlp_graph g) {
 
 static void graph_free(tlp_graph g) {
     if (!g) return;
-    void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out,
+    void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)
@@ -295,6 +307,11 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         }
         if (n_src) {
             k_norm<<<grid_for(n_src, nsm), 256, 0, s>>>(g->out_deg, n_src, g->c_out);
+            CTRY(cudaGetLastError());
+        }
+        if (nnz) {
+            TRY(dmalloc((void **)&g->ew_both, sizeof(float) * nnz + 16, g));
+            k_edge_both<<<grid_for(nnz, nsm), 256, 0, s>>>(g->colidx, g->ew, g->c_out, nnz, g->ew_both);
             CTRY(cudaGetLastError());
         }
     }

@@ -43,6 +43,7 @@ struct tlp_graph_s {
     int32_t *in_deg = nullptr;   // [n_dst]
     int32_t *out_deg = nullptr;  // [n_src] (global for a dist slice)
     float *c_out = nullptr;      // [n_src] 1/sqrt(max(out_deg,1))
+    float *ew_both = nullptr;    // [nnz] c_out[colidx[e]] * w_e (GCN BOTH coefficient)
 
     int2 *tasks = nullptr;       // [n_tasks]
     int32_t *hub_row = nullptr;  // [n_hubs]
