@@ -53,6 +53,9 @@ constexpr unsigned FULL = 0xffffffffu;
 #ifndef TLP_MINB
 #define TLP_MINB 3     // register path: 3 CTAs/SM -> <= 85 registers, 24 warps/SM
 #endif
+#ifndef TLP_HINTS
+#define TLP_HINTS 0    // 1: L2 evict_first policy on per-edge streams and Y stores (measured: no gain)
+#endif
 #ifndef TLP_MINB_ASYNC
 #define TLP_MINB_ASYNC 3  // async path: 3 CTAs/SM (ring = 3 x 64 KB of shared memory)
 #endif
@@ -118,7 +121,14 @@ __device__ __forceinline__ Vec<VEC> ld_vec_cg(const float *p) {
 template <int VEC>
 __device__ __forceinline__ void st_vec(float *p, const Vec<VEC> &x) {
     if constexpr (VEC == 4) {
+#if TLP_HINTS
+        unsigned long long pol;
+        asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
+                     ::"l"(p), "f"(x.v[0]), "f"(x.v[1]), "f"(x.v[2]), "f"(x.v[3]), "l"(pol) : "memory");
+#else
         *reinterpret_cast<float4 *>(p) = make_float4(x.v[0], x.v[1], x.v[2], x.v[3]);
+#endif
     } else if constexpr (VEC == 2) {
         *reinterpret_cast<float2 *>(p) = make_float2(x.v[0], x.v[1]);
     } else {
@@ -206,6 +216,36 @@ __device__ __forceinline__ void consume_group(int j, int n, int half, const Vec<
     }
 }
 
+// ---- L2 residency hints -------------------------------------------------------
+// Per-edge streams (colidx, edge coefficients) and Y are touched once per strip:
+// with TLP_HINTS they are loaded / stored with an L2 evict_first policy so they
+// do not evict the L2-resident panel of X that every edge gathers from.
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+    unsigned long long p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ int ld_stream(const int32_t *ptr) {
+#if TLP_HINTS
+    int v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
+                 : "=r"(v) : "l"(ptr), "l"(policy_evict_first()));
+    return v;
+#else
+    return __ldg(ptr);
+#endif
+}
+__device__ __forceinline__ float ld_stream(const float *ptr) {
+#if TLP_HINTS
+    float v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
+                 : "=f"(v) : "l"(ptr), "l"(policy_evict_first()));
+    return v;
+#else
+    return __ldg(ptr);
+#endif
+}
+
 // Reduce the edges [e0, e1) of one destination row for the feature vector at
 // `col` (a6 / a7).  GCN/GIN: acc = sum_e c_e X[u_e] (two-chain order above).
 // GAT: online softmax state (m, den, acc = sum_e exp(s_e - m) X[u_e]).
@@ -243,12 +283,12 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
         int u0 = 0, u1 = 0;
         float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
         if (lane < n0) {
-            u0 = __ldg(ci + lane);
-            if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
+            u0 = ld_stream(ci + lane);
+            if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane);
         }
         if (lane < n1) {
-            u1 = __ldg(ci + 32 + lane);
-            if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
+            u1 = ld_stream(ci + 32 + lane);
+            if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
         }
         if constexpr (DEP)
             if (lane < n0) d0 = __ldg(dep + u0);
@@ -258,8 +298,8 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             int u2 = 0;
             float w2 = 1.f;
             if (lane < n2) {
-                u2 = __ldg(ci + off + 64 + lane);
-                if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
+                u2 = ld_stream(ci + off + 64 + lane);
+                if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
             }
             if constexpr (DEP)
                 if (lane < n1) d1 = __ldg(dep + u1);
@@ -400,12 +440,12 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
         int u0 = 0, u1 = 0;
         float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
         if (lane < n0) {
-            u0 = __ldg(ci + lane);
-            if constexpr (COEF & COEF_W) w0 = __ldg(wp + lane);
+            u0 = ld_stream(ci + lane);
+            if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane);
         }
         if (lane < n1) {
-            u1 = __ldg(ci + 32 + lane);
-            if constexpr (COEF & COEF_W) w1 = __ldg(wp + 32 + lane);
+            u1 = ld_stream(ci + 32 + lane);
+            if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
         }
         if constexpr (DEP)
             if (lane < n0) d0 = __ldg(dep + u0);
@@ -422,8 +462,8 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
             int u2 = 0;
             float w2 = 1.f;
             if (lane < n2) {
-                u2 = __ldg(ci + off + 64 + lane);
-                if constexpr (COEF & COEF_W) w2 = __ldg(wp + off + 64 + lane);
+                u2 = ld_stream(ci + off + 64 + lane);
+                if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
             }
             if constexpr (DEP)
                 if (lane < n1) d1 = __ldg(dep + u1);
