@@ -40,6 +40,7 @@ METRIC = "GCN/GAT aggregation ms & HBM GB/s vs 8 TB/s, Reddit-shaped, 1/2/4/8 B2
 NOMINAL_HBM_GBS = 8000.0
 FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
 OPS = ("gcn", "gin", "gat")
+# "gcn2": two GCN(BOTH) layers, Y1 = A X, Y2 = A Y1 (the R-MAT config; X.W is out of scope)
 
 
 # ------------------------------------------------------------------ bytes --
@@ -52,6 +53,8 @@ def gather_bytes(op, n_rows, n_edges, F):
         return n_edges * (4 * F + 4) + n_rows * (8 * F + 8)
     if op == "gat":
         return n_edges * (4 * F + 8) + n_rows * (4 * F + 12)
+    if op == "gcn2":
+        return 2 * gather_bytes("gcn", n_rows, n_edges, F)
     raise ValueError(op)
 
 
@@ -145,20 +148,26 @@ WORKLOADS = {
     "products": dict(graph="products", ops=("gat",)),
     "pubmed": dict(graph="pubmed", ops=("gat",)),
     "cora": dict(graph="cora", ops=("gcn",)),
+    "rmat24": dict(graph="rmat24", ops=("gcn2",)),
 }
+LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2}
 
 
 def workload_desc(name, cfg, E):
-    ops = "+".join({"gcn": "GCN(both)", "gin": "GIN(eps=0.1)", "gat": "GAT(slope=0.2)"}[o]
-                   for o in WORKLOADS[name]["ops"])
-    return f"{name}-shaped {ops}: N={cfg['n']} E={E} F={cfg['F']} ld={cfg['ld']}"
+    ops = "+".join({"gcn": "GCN(both)", "gin": "GIN(eps=0.1)", "gat": "GAT(slope=0.2)",
+                    "gcn2": "2-layer GCN(both)"}[o] for o in WORKLOADS[name]["ops"])
+    return f"{name}-shaped {ops}: N={cfg_n(cfg)} E={E} F={cfg['F']} ld={cfg['ld']}"
+
+
+def cfg_n(cfg):
+    return cfg["n"] if "n" in cfg else 1 << cfg["scale"]
 
 
 def make_inputs(name, device):
     import synth
     cfg = synth.CONFIGS[WORKLOADS[name]["graph"]]
     rp, ci = synth.dataset_graph(WORKLOADS[name]["graph"], device=device)
-    n = cfg["n"]
+    n = cfg_n(cfg)
     X = synth.dataset_features(WORKLOADS[name]["graph"], n)
     el = synth.normal(n, 1000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
     er = synth.normal(n, 2000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
@@ -178,12 +187,16 @@ def run_tlp(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+    # the dist path (NCCL comm + tlp_dist_*) also at world = 1 with --dist
+    use_dist = world > 1 or args.dist
+    if use_dist:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", str(29500 + os.getpid() % 1000))
+        dist.init_process_group("nccl", device_id=dev, rank=rank, world_size=world)
     name = args.workload
     ops = WORKLOADS[name]["ops"]
     cfg, rp, ci, Xh, elh, erh = make_inputs(name, dev)
-    n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+    n, F, ld = cfg_n(cfg), cfg["F"], cfg["ld"]
     E = len(ci)
     stream = torch.cuda.current_stream(dev)
 
@@ -191,7 +204,7 @@ def run_tlp(args):
     ci_d = torch.from_numpy(ci).to(dev)
     comm = None
     t0 = time.perf_counter()
-    if world > 1:
+    if use_dist:
         comm = tlp.comm_from_torch()
         g = tlp.Graph.dist(comm, rp_d, ci_d)
     else:
@@ -204,22 +217,29 @@ def run_tlp(args):
     el = torch.from_numpy(elh).to(dev)
     er = torch.from_numpy(erh).to(dev)
     Y = {op: torch.empty((n, ld), dtype=torch.float32, device=dev) for op in ops}
+    Y1 = torch.empty((n, ld), dtype=torch.float32, device=dev) if "gcn2" in ops else None
+
+    def gcn_to(Xin, out):
+        if use_dist:
+            tlp.tlp_dist_gcn_aggregate(g.handle, comm, Xin, out, "both", F=F)
+        else:
+            g.gcn(Xin, "both", Y=out, F=F)
 
     def launch(op, Xin=X, elv=el, erv=er):
-        if world > 1:
-            if op == "gcn":
-                tlp.tlp_dist_gcn_aggregate(g.handle, comm, Xin, Y[op], "both", F=F)
-            elif op == "gin":
+        if op == "gcn2":  # layer 1, then layer 2 on its output (all-gather between in dist mode)
+            gcn_to(Xin, Y1)
+            gcn_to(Y1, Y[op])
+        elif op == "gcn":
+            gcn_to(Xin, Y[op])
+        elif use_dist:
+            if op == "gin":
                 tlp.tlp_dist_gin_aggregate(g.handle, comm, Xin, Y[op], synth.EPS, F=F)
             else:
                 tlp.tlp_dist_gat_aggregate(g.handle, comm, Xin, Y[op], elv, erv, synth.SLOPE, F=F)
+        elif op == "gin":
+            g.gin(Xin, synth.EPS, Y=Y[op], F=F)
         else:
-            if op == "gcn":
-                g.gcn(Xin, "both", Y=Y[op], F=F)
-            elif op == "gin":
-                g.gin(Xin, synth.EPS, Y=Y[op], F=F)
-            else:
-                g.gat(Xin, elv, erv, synth.SLOPE, Y=Y[op], F=F)
+            g.gat(Xin, elv, erv, synth.SLOPE, Y=Y[op], F=F)
 
     for _ in range(args.warmup):
         for op in ops:
@@ -229,7 +249,7 @@ def run_tlp(args):
     # ---- device-resident timed region ----
     ev = {op: [] for op in ops}
     start, stop = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    if world > 1:
+    if use_dist:
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
@@ -243,12 +263,12 @@ def run_tlp(args):
                 ev[op].append((a, b))
         stop.record(stream)
         torch.cuda.synchronize()
-    if world > 1:
+    if use_dist:
         dist.barrier()
     total_ms = start.elapsed_time(stop)
     op_ms = {op: [a.elapsed_time(b) for a, b in ev[op]] for op in ops}
     t = torch.tensor([total_ms], device=dev)
-    if world > 1:
+    if use_dist:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         for op in ops:
             tt = torch.tensor(op_ms[op], device=dev)
@@ -264,8 +284,10 @@ def run_tlp(args):
     if not args.no_e2e:
         Xp = torch.from_numpy(Xh).pin_memory()
         elp, erp = torch.from_numpy(elh).pin_memory(), torch.from_numpy(erh).pin_memory()
-        Yp = {op: torch.empty((n, ld), dtype=torch.float32).pin_memory() for op in ops}
-        if world > 1:
+        # every rank uploads its (replicated) inputs; rank 0 reads the result back
+        read_back = rank == 0
+        Yp = {op: torch.empty((n, ld), dtype=torch.float32).pin_memory() for op in ops} if read_back else {}
+        if use_dist:
             dist.barrier()
         torch.cuda.synchronize()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -276,21 +298,23 @@ def run_tlp(args):
             er.copy_(erp, non_blocking=True)
             for op in ops:
                 launch(op)
-                Yp[op].copy_(Y[op], non_blocking=True)
+                if read_back:
+                    Yp[op].copy_(Y[op], non_blocking=True)
         b.record(stream)
         torch.cuda.synchronize()
         te = torch.tensor([a.elapsed_time(b)], device=dev)
-        if world > 1:
+        if use_dist:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e2e_ms = float(te.item()) / args.steps
         h2d = Xp.numel() * 4 + elp.numel() * 4 + erp.numel() * 4
-        d2h = sum(Yp[op].numel() * 4 for op in ops)
+        d2h = sum(Yp[op].numel() * 4 for op in ops) if read_back else 0
         e2e = {"value": round(step_bytes / (e2e_ms * 1e-3) / 1e9, 2), "unit": "GB/s",
                "ms_per_step": round(e2e_ms, 3), "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h),
-               "note": "pinned host X/el/er -> device, 3 aggregations, Y -> pinned host, per step"}
+               "note": "per step: pinned host X/el/er -> device (every rank), the step's "
+                       "aggregations, Y -> pinned host (rank 0); max over ranks"}
         # parity spot check of the end-to-end outputs (device copy vs host copy)
-        for op in ops:
+        for op in Yp:
             assert torch.equal(Yp[op][:64].to(dev), Y[op][:64])
 
     # ---- roofline of the dominant kernel ----
@@ -318,25 +342,26 @@ def run_tlp(args):
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
         "config": {"workload": workload_desc(name, cfg, E),
-                   "graph": "Chung-Lu G1 (SURVEY 8(d) d1), seed %d" % cfg["seed"],
+                   "graph": ("R-MAT G2 (0.57,0.19,0.19,0.05), seed %d" if name == "rmat24"
+                             else "Chung-Lu G1 (SURVEY 8(d) d1), seed %d") % cfg["seed"],
                    "l2": "inputs larger than L2 (X = %.0f MB, colidx = %.0f MB vs 126 MB L2); no flush"
                          % (n * ld * 4 / 1e6, E * 4 / 1e6),
-                   "parallelism": "rows%d" % world if world > 1 else "single",
+                   "parallelism": ("rows%d (edge-balanced row ranges, X replicated, grouped-broadcast all-gather of Y)" % world) if use_dist else "single",
                    "frac_of_8TBs": round(value / NOMINAL_HBM_GBS, 4)},
         "ops": per_op, "create_ms": round(create_ms, 1),
         "plan": {k: info[k] for k in ("n_hubs", "n_hub_chunks", "n_units", "n_tasks",
                                       "hub_threshold", "hub_chunk", "max_in_degree")},
-        "roofline": roofline, "gpu_launches": args.steps * len(ops) * 1,
+        "roofline": roofline, "gpu_launches": args.steps * sum(LAUNCHES[o] for o in ops),
         "clocks": clk.summary(), "e2e": e2e,
     }
-    if world > 1:
-        result["gpu_launches_note"] = "per rank: 1 k_agg + NCCL broadcasts per aggregation"
+    if use_dist:
+        result["gpu_launches_note"] = "per rank: 1 k_agg per aggregation, plus NCCL's broadcast kernels"
     if rank == 0 and not args.no_cpu_baseline and world == 1:
         result["cpu_baseline"] = cpu_baseline(name, cfg, rp, ci, Xh, elh, erh, args.cpu_seconds)
     g.close()
     if comm is not None:
         tlp.tlp_comm_destroy(comm)
-    if world > 1:
+    if use_dist:
         dist.destroy_process_group()
     if rank == 0:
         print(json.dumps(result))
@@ -353,6 +378,11 @@ def _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows):
     for op in WORKLOADS[name]["ops"]:
         if op == "gcn":
             oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F)
+        elif op == "gcn2":
+            # layer 2 of a row needs layer 1 at its in-neighbours: the bounded sample
+            # times layer 1 on the sampled rows twice (same work per row as layer 2)
+            oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F)
+            oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F)
         elif op == "gin":
             oracle.gin(rp, ci, Xh, synth.EPS, rows=rows, F=F)
         else:
@@ -364,10 +394,10 @@ def _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows):
 
 def _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds, seed=0):
     rng = np.random.default_rng(seed)
-    perm = rng.permutation(cfg["n"])
+    perm = rng.permutation(cfg_n(cfg))
     probe = np.sort(perm[:64])
     by, dt = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, probe)
-    k = int(max(64, min(cfg["n"], 64 * seconds / max(dt, 1e-3))))
+    k = int(max(64, min(cfg_n(cfg), 64 * seconds / max(dt, 1e-3))))
     return np.sort(perm[:k])
 
 
@@ -375,7 +405,7 @@ def cpu_baseline(name, cfg, rp, ci, Xh, elh, erh, seconds):
     rows = _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds)
     by, dt = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows)
     return {"value": round(by / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{len(rows)} of {cfg['n']} destination rows (uniform random, seed 0), "
+            "sample": f"{len(rows)} of {cfg_n(cfg)} destination rows (uniform random, seed 0), "
                       f"all ops of the step, {dt:.1f} s single-threaded fp64",
             "host_cores_available": len(os.sched_getaffinity(0))}
 
@@ -399,7 +429,7 @@ def run_reference(args):
         tot_b += b
         tot_t += t
     value = tot_b / tot_t / 1e9
-    sample = (f"{len(rows)} of {cfg['n']} destination rows per step (uniform random, seed 0), "
+    sample = (f"{len(rows)} of {cfg_n(cfg)} destination rows per step (uniform random, seed 0), "
               f"all ops of the step, single-threaded fp64 oracle")
     out = {"impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -424,6 +454,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--dist", action="store_true",
+                    help="use the NCCL dist API even at world size 1 (exercises the N>1 path)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: the contract wants >= 3 warm-up steps", file=sys.stderr)

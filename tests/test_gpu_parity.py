@@ -453,3 +453,43 @@ def test_gather_paths_bitwise(tlp, monkeypatch, F, ld):
         assert torch.equal(a, b)
     _check("async gat", outs["async"][2], oracle.gat(rp, ci, Xh, synth.normal(n, 1), synth.normal(n, 2), 0.2, F=F))
     g.close(); gw.close()
+
+
+def test_config_rmat24_two_layer_sampled(tlp):
+    """R-MAT scale 24 (E = 2^29), F = 128, two GCN(BOTH) layers.  Layer 1 is checked
+    against the oracle on sampled rows (incl. the largest hubs); layer 2 against the
+    oracle applied to the GPU's fp32 layer-1 output (R22)."""
+    cfg = synth.CONFIGS["rmat24"]
+    n = 1 << cfg["scale"]
+    F = cfg["F"]
+    rp, ci = synth.dataset_graph("rmat24")
+    assert len(ci) == 2 * cfg["edge_factor"] * n
+    Xh = synth.features(n, F, F, seed=105)
+    g = tlp.Graph(_t(rp), _t(ci))
+    X = _t(Xh)
+    Y1 = g.gcn(X, "both")
+    Y2 = g.gcn(Y1, "both")
+    rows = _sample_rows(rp, 2000, 8, 5)
+    _check("rmat layer 1", Y1[_t(rows)], oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F))
+    Y1h = Y1.cpu().numpy()
+    _check("rmat layer 2", Y2[_t(rows)], oracle.gcn(rp, ci, Y1h, "both", rows=rows, F=F))
+    g.close()
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck", "initcheck"])
+def test_compute_sanitizer(tool):
+    """T5: compute-sanitizer over both gather paths, hub merges and panels."""
+    import os, shutil, subprocess, sys
+    cs = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(cs):
+        pytest.skip("compute-sanitizer not available")
+    tgt = os.path.join(os.path.dirname(__file__), "sanitize_target.py")
+    args = [cs, "--tool", tool, "--error-exitcode", "9"]
+    if tool == "memcheck":
+        args += ["--leak-check", "no"]
+    # restrict to our kernels (torch's own kernels are not under test); initcheck
+    # must see every kernel, since a filtered-out writer looks like missing init
+    if tool != "initcheck":
+        args += ["--kernel-name", "kns=k_"]
+    r = subprocess.run(args + [sys.executable, tgt], capture_output=True, text=True, timeout=1500)
+    assert r.returncode == 0 and "sanitize target ok" in r.stdout, r.stdout[-3000:] + r.stderr[-3000:]
