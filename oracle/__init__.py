@@ -66,6 +66,11 @@ def _load():
         lib.oracle_gat.argtypes = [I64, I64, P, P, P, I64, I64, P, P,
                                    ctypes.c_double, I64, I64, P, P, P, P]
         lib.oracle_gat.restype = ctypes.c_int
+        lib.oracle_sage.argtypes = [I64, I64, P, P, P, I64, I64, ctypes.c_int, I64, I64, P, P, P]
+        lib.oracle_sage.restype = ctypes.c_int
+        lib.oracle_gat_mh.argtypes = [I64, I64, P, P, P, I64, I64, I64, P, P, ctypes.c_double,
+                                      I64, I64, P, P, P]
+        lib.oracle_gat_mh.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -181,6 +186,44 @@ def gat(rowptr, colidx, X, el, er, slope, rows=None, row_offset=0, F=None,
     if rc:
         raise ValueError("oracle_gat: bad arguments")
     return (Y, A, S) if return_alpha_sum else (Y, A)
+
+
+def sage(rowptr, colidx, X, include_self=False, rows=None, row_offset=0, F=None):
+    """GraphSage mean (optionally including the self row).  Returns (Y, A)."""
+    rowptr, colidx = _csr(rowptr, colidx)
+    X = _feat(X)
+    n_dst = rowptr.shape[0] - 1
+    F = X.shape[1] if F is None else F
+    ldx = X.strides[0] // 4
+    rows, nr = _rows(rows, n_dst)
+    Y = np.empty((nr, F)); A = np.empty((nr, F))
+    rc = _load().oracle_sage(n_dst, X.shape[0], _ptr(rowptr), _ptr(colidx), _ptr(X), F, ldx,
+                             int(bool(include_self)), int(row_offset), nr, _ptr(rows), _ptr(Y),
+                             _ptr(A))
+    if rc:
+        raise ValueError("oracle_sage: bad arguments")
+    return Y, A
+
+
+def gat_mh(rowptr, colidx, X, el, er, heads, slope, rows=None, row_offset=0, Fh=None):
+    """Multi-head GAT: el, er are [n, heads] (row-major); head h owns columns
+    [h*Fh, (h+1)*Fh).  Returns (Y, A) of width heads*Fh."""
+    rowptr, colidx = _csr(rowptr, colidx)
+    X = _feat(X)
+    n_dst = rowptr.shape[0] - 1
+    H = int(heads)
+    Fh = X.shape[1] // H if Fh is None else int(Fh)
+    ldx = X.strides[0] // 4
+    el = np.ascontiguousarray(el, dtype=np.float32).reshape(-1)
+    er = np.ascontiguousarray(er, dtype=np.float32).reshape(-1)
+    rows, nr = _rows(rows, n_dst)
+    Y = np.empty((nr, H * Fh)); A = np.empty((nr, H * Fh))
+    rc = _load().oracle_gat_mh(n_dst, X.shape[0], _ptr(rowptr), _ptr(colidx), _ptr(X), H, Fh, ldx,
+                               _ptr(el), _ptr(er), float(slope), int(row_offset), nr, _ptr(rows),
+                               _ptr(Y), _ptr(A))
+    if rc:
+        raise ValueError("oracle_gat_mh: bad arguments")
+    return Y, A
 
 
 def within_tolerance(Y_test, Y_ref, A_ref, rel=1e-5, abs_=1e-6):

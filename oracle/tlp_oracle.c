@@ -264,3 +264,97 @@ int oracle_gat(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
     }
     return 0;
 }
+
+/* ---- NEXT-1: GraphSage mean, multi-head GAT ------------------ */
+
+/* GraphSage mean aggregator (Hamilton et al. [15]):
+ *   include_self = 0:  Y[v,f] = (1/max(d,1)) * sum_e X[u,f]            (mean of N(v))
+ *   include_self = 1:  Y[v,f] = (X[row_offset+v,f] + sum_e X[u,f]) / (d+1)
+ *                      (the "GCN" aggregator variant of [15]: mean over N(v) + v)
+ * Edge weights are not an input (the mean is unweighted).  A = sum |terms| / count. */
+int oracle_sage(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+                const int32_t *colidx, const float *X, int64_t F, int64_t ldx,
+                int include_self, int64_t row_offset, int64_t n_rows,
+                const int64_t *rows, double *Y, double *A)
+{
+    if (F < 0 || ldx < F || row_offset < 0 ||
+        (include_self && row_offset + n_dst > n_src))
+        return -1;
+    for (int64_t i = 0; i < n_rows; ++i) {
+        int64_t v = pick_row(rows, i);
+        int64_t d = rowptr[v + 1] - rowptr[v];
+        int64_t cnt = d + (include_self ? 1 : 0);
+        double inv = 1.0 / (double)(cnt > 1 ? cnt : 1);
+        for (int64_t f = 0; f < F; ++f) {
+            double s = 0.0, a = 0.0;
+            if (include_self) {
+                double x = (double)X[(row_offset + v) * ldx + f];
+                s += x;
+                a += fabs(x);
+            }
+            for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e) {
+                double x = (double)X[(int64_t)colidx[e] * ldx + f];
+                s += x;
+                a += fabs(x);
+            }
+            Y[i * F + f] = inv * s;
+            if (A)
+                A[i * F + f] = inv * a;
+        }
+    }
+    return 0;
+}
+
+/* Multi-head GAT (Velickovic [43]): H heads, head h owns the
+ * feature columns [h*Fh, (h+1)*Fh) of X and Y (F = H*Fh), with its own scores
+ *   s_e,h = LeakyReLU(el[u*H + h] + er[(row_offset+v)*H + h], slope)
+ * and its own softmax over the in-edges of v.  Each head is exactly the
+ * single-head oracle_gat on its column block (computed here the same way). */
+int oracle_gat_mh(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+                  const int32_t *colidx, const float *X, int64_t H, int64_t Fh,
+                  int64_t ldx, const float *el, const float *er, double slope,
+                  int64_t row_offset, int64_t n_rows, const int64_t *rows,
+                  double *Y, double *A)
+{
+    if (H < 1 || Fh < 0 || ldx < H * Fh || row_offset < 0)
+        return -1;
+    int64_t F = H * Fh;
+    for (int64_t i = 0; i < n_rows; ++i) {
+        int64_t v = pick_row(rows, i);
+        int64_t e0 = rowptr[v], e1 = rowptr[v + 1];
+        int64_t d = e1 - e0;
+        double *alpha = (double *)malloc(sizeof(double) * (size_t)(d > 0 ? d : 1));
+        if (!alpha)
+            return -1;
+        for (int64_t h = 0; h < H; ++h) {
+            if (d > 0) {
+                double er_v = (double)er[(row_offset + v) * H + h];
+                double m = -INFINITY;
+                for (int64_t e = e0; e < e1; ++e) {
+                    double s = leaky_relu((double)el[(int64_t)colidx[e] * H + h] + er_v, slope);
+                    alpha[e - e0] = s;
+                    if (s > m)
+                        m = s;
+                }
+                double z = 0.0;
+                for (int64_t k = 0; k < d; ++k)
+                    z += exp(alpha[k] - m);
+                for (int64_t k = 0; k < d; ++k)
+                    alpha[k] = exp(alpha[k] - m) / z;
+            }
+            for (int64_t f = h * Fh; f < (h + 1) * Fh; ++f) {
+                double s = 0.0, a = 0.0;
+                for (int64_t e = e0; e < e1; ++e) {
+                    double x = (double)X[(int64_t)colidx[e] * ldx + f];
+                    s += alpha[e - e0] * x;
+                    a += alpha[e - e0] * fabs(x);
+                }
+                Y[i * F + f] = s;
+                if (A)
+                    A[i * F + f] = a;
+            }
+        }
+        free(alpha);
+    }
+    return 0;
+}

@@ -388,3 +388,68 @@ def test_p6_partition_edge_cases():
     rp0 = np.zeros(4, np.int64)  # E = 0
     assert oracle.partition(rp0, 3).tolist() == [0, 0, 0, 3]
     assert oracle.partition(np.zeros(1, np.int64), 2).tolist() == [0, 0, 0]
+
+
+# ---------------------------------------------------- NEXT-1: Sage, multi-head GAT --
+
+def test_p1_star_sage():
+    g = _star()
+    s = g["without_self_loops"]
+    rp, ci = synth.figure1_star(self_loops=False)
+    X = np.array(g["x"], np.float32).reshape(-1, 1)
+    np.testing.assert_allclose(oracle.sage(rp, ci, X)[0].ravel(), s["sage_mean"], rtol=1e-15)
+    np.testing.assert_allclose(oracle.sage(rp, ci, X, include_self=True)[0].ravel(),
+                               s["sage_mean_with_self"], rtol=1e-15)
+
+
+@pytest.mark.parametrize("case", range(6))
+@pytest.mark.parametrize("include_self", [False, True])
+def test_p2_brute_sage(case, include_self):
+    rp, ci, n_src = _small_cases()[case]
+    n_dst = len(rp) - 1
+    if include_self and n_dst > n_src:
+        pytest.skip("self row needs n_dst <= n_src")
+    X = synth.features(n_src, 5, 6, seed=case)
+    Y, _ = oracle.sage(rp, ci, X, include_self=include_self, F=5)
+    _, C = _dense_adj(rp, ci, n_dst, n_src)
+    if include_self:
+        C[np.arange(n_dst), np.arange(n_dst)] += 1
+    cnt = np.maximum(C.sum(1, keepdims=True), 1)
+    np.testing.assert_allclose(Y, (C / cnt) @ X[:, :5].astype(np.float64), rtol=1e-12, atol=1e-13)
+
+
+def test_p4_sage_without_self_is_gcn_right(pub):
+    rp, ci, n = pub
+    X = synth.features(n, 6, seed=8)
+    np.testing.assert_allclose(oracle.sage(rp, ci, X)[0], oracle.gcn(rp, ci, X, "right")[0],
+                               rtol=1e-14, atol=1e-15)
+
+
+@pytest.mark.parametrize("case", range(6))
+@pytest.mark.parametrize("H,Fh", [(1, 3), (2, 2), (4, 1), (3, 5)])
+def test_p2_brute_gat_mh(case, H, Fh):
+    rp, ci, n_src = _small_cases()[case]
+    n_dst = len(rp) - 1
+    X = synth.features(n_src, H * Fh, H * Fh + 1, seed=case)
+    el = (synth.normal(n_src * H, case + 70) * 2).reshape(n_src, H)
+    er = (synth.normal(max(n_dst, n_src) * H, case + 80) * 2).reshape(-1, H)
+    Y, _ = oracle.gat_mh(rp, ci, X, el, er, H, 0.2, Fh=Fh)
+    for h in range(H):
+        ref = _brute_gat(rp, ci, X[:, h * Fh:(h + 1) * Fh], el[:, h].copy(), er[:, h].copy(), 0.2, n_src)
+        np.testing.assert_allclose(Y[:, h * Fh:(h + 1) * Fh], ref, rtol=1e-11, atol=1e-13)
+
+
+def test_p4_gat_mh_one_head_and_head_permutation(pub):
+    rp, ci, n = pub
+    X = synth.features(n, 12, seed=4)
+    el1, er1 = synth.normal(n, 1), synth.normal(n, 2)
+    np.testing.assert_array_equal(oracle.gat_mh(rp, ci, X, el1, er1, 1, 0.2)[0],
+                                  oracle.gat(rp, ci, X, el1, er1, 0.2)[0])
+    H, Fh = 3, 4
+    el = synth.normal(n * H, 5).reshape(n, H)
+    er = synth.normal(n * H, 6).reshape(n, H)
+    Y = oracle.gat_mh(rp, ci, X, el, er, H, 0.2)[0]
+    perm = [2, 0, 1]
+    Xp = np.concatenate([X[:, p * Fh:(p + 1) * Fh] for p in perm], axis=1)
+    Yp = oracle.gat_mh(rp, ci, Xp, el[:, perm], er[:, perm], H, 0.2)[0]
+    np.testing.assert_array_equal(Yp, np.concatenate([Y[:, p * Fh:(p + 1) * Fh] for p in perm], axis=1))
