@@ -55,6 +55,11 @@ def gather_bytes(op, n_rows, n_edges, F):
         return n_edges * (4 * F + 8) + n_rows * (4 * F + 12)
     if op == "gcn2":
         return 2 * gather_bytes("gcn", n_rows, n_edges, F)
+    if op == "sage":  # mean over N(v)+v: per edge 4F + 4; per row self + Y + rowptr
+        return n_edges * (4 * F + 4) + n_rows * (8 * F + 8)
+    if op.startswith("gat") and op[3:].isdigit():  # H heads: el/er per head
+        H = int(op[3:])
+        return n_edges * (4 * F + 4 + 4 * H) + n_rows * (4 * F + 8 + 4 * H)
     raise ValueError(op)
 
 
@@ -149,13 +154,17 @@ WORKLOADS = {
     "pubmed": dict(graph="pubmed", ops=("gat",)),
     "cora": dict(graph="cora", ops=("gcn",)),
     "rmat24": dict(graph="rmat24", ops=("gcn2",)),
+    # NEXT-1 rows: GraphSage mean (+self) and 4-head GAT
+    "reddit_sage": dict(graph="reddit", ops=("sage",)),
+    "products_gat4": dict(graph="products", ops=("gat4",)),
 }
-LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2}
+LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2, "sage": 1, "gat4": 1}
 
 
 def workload_desc(name, cfg, E):
     ops = "+".join({"gcn": "GCN(both)", "gin": "GIN(eps=0.1)", "gat": "GAT(slope=0.2)",
-                    "gcn2": "2-layer GCN(both)"}[o] for o in WORKLOADS[name]["ops"])
+                    "gcn2": "2-layer GCN(both)", "sage": "GraphSage-mean(+self)",
+                    "gat4": "4-head GAT(slope=0.2)"}[o] for o in WORKLOADS[name]["ops"])
     return f"{name}-shaped {ops}: N={cfg_n(cfg)} E={E} F={cfg['F']} ld={cfg['ld']}"
 
 
@@ -169,8 +178,10 @@ def make_inputs(name, device):
     rp, ci = synth.dataset_graph(WORKLOADS[name]["graph"], device=device)
     n = cfg_n(cfg)
     X = synth.dataset_features(WORKLOADS[name]["graph"], n)
-    el = synth.normal(n, 1000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
-    er = synth.normal(n, 2000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
+    H = max([int(o[3:]) for o in WORKLOADS[name]["ops"] if o.startswith("gat") and o[3:].isdigit()]
+            or [1])
+    el = synth.normal(n * H, 1000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
+    er = synth.normal(n * H, 2000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
     return cfg, rp, ci, X, el, er
 
 
@@ -234,12 +245,21 @@ def run_tlp(args):
         elif use_dist:
             if op == "gin":
                 tlp.tlp_dist_gin_aggregate(g.handle, comm, Xin, Yo[op], synth.EPS, F=F)
-            else:
+            elif op == "sage":
+                tlp.tlp_dist_sage_aggregate(g.handle, comm, Xin, Yo[op], True, F=F)
+            elif op == "gat":
                 tlp.tlp_dist_gat_aggregate(g.handle, comm, Xin, Yo[op], elv, erv, synth.SLOPE, F=F)
+            else:
+                tlp.tlp_dist_gat_mh_aggregate(g.handle, comm, Xin, Yo[op], elv, erv, int(op[3:]),
+                                              synth.SLOPE, F=F)
         elif op == "gin":
             g.gin(Xin, synth.EPS, Y=Yo[op], F=F)
-        else:
+        elif op == "sage":
+            g.sage(Xin, True, Y=Yo[op], F=F)
+        elif op == "gat":
             g.gat(Xin, elv, erv, synth.SLOPE, Y=Yo[op], F=F)
+        else:
+            g.gat_mh(Xin, elv, erv, int(op[3:]), synth.SLOPE, Y=Yo[op], F=F)
 
     for _ in range(args.warmup):
         for op in ops:
@@ -425,8 +445,13 @@ def _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows):
             oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F)
         elif op == "gin":
             oracle.gin(rp, ci, Xh, synth.EPS, rows=rows, F=F)
-        else:
+        elif op == "sage":
+            oracle.sage(rp, ci, Xh, include_self=True, rows=rows, F=F)
+        elif op == "gat":
             oracle.gat(rp, ci, Xh, elh, erh, synth.SLOPE, rows=rows, F=F)
+        else:
+            H = int(op[3:])
+            oracle.gat_mh(rp, ci, Xh, elh, erh, H, synth.SLOPE, rows=rows, Fh=F // H)
         e = int((rp[rows + 1] - rp[rows]).sum())
         by += gather_bytes(op, len(rows), e, F)
     return by, time.perf_counter() - t0

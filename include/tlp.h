@@ -199,6 +199,29 @@ tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F,
                              int64_t ldx, const float *el, const float *er,
                              float slope, float *Y, int64_t ldy, void *stream);
 
+/* ---- NEXT-1: GraphSage mean, multi-head GAT ------------------ */
+
+/* GraphSage mean aggregator (Hamilton et al. [15]):
+ *   include_self = 0: Y[v] = (1/max(d,1)) * sum_e X[u]            (mean over N(v))
+ *   include_self = 1: Y[v] = (X[row_offset+v] + sum_e X[u]) / (d+1) (mean over N(v)+v)
+ * Unweighted (edge weights ignored).  The concatenation / linear layer of
+ * GraphSage is dense and out of scope.  Same layouts and errors as GCN;
+ * include_self requires row_offset + n_dst <= n_src. */
+tlp_status tlp_sage_aggregate(tlp_graph g, const float *X, int64_t F,
+                              int64_t ldx, int include_self, float *Y,
+                              int64_t ldy, void *stream);
+
+/* Multi-head GAT (Velickovic [43]): `heads` independent attention heads; head
+ * h owns feature columns [h*F/heads, (h+1)*F/heads) of X and Y (F must be a
+ * multiple of heads) and has its own scores and softmax:
+ *   s_e,h = LeakyReLU(el[u*heads + h] + er[(row_offset+v)*heads + h], slope)
+ * el: fp32 device [n_src x heads], er: fp32 device [(row_offset+n_dst) x heads]
+ * (row-major).  heads = 1 equals tlp_gat_aggregate. */
+tlp_status tlp_gat_mh_aggregate(tlp_graph g, const float *X, int64_t heads,
+                                int64_t F, int64_t ldx, const float *el,
+                                const float *er, float slope, float *Y,
+                                int64_t ldy, void *stream);
+
 /* ---- multi-GPU (destination-row ranges balanced by edge count) ------------ */
 
 /* Pure host function: bounds[0] = 0, bounds[parts] = n, and for 0 < k < parts
@@ -260,6 +283,15 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph local, tlp_comm c,
                                   const float *X_full, int64_t F, int64_t ldx,
                                   const float *el, const float *er, float slope,
                                   float *Y_full, int64_t ldy, void *stream);
+tlp_status tlp_dist_sage_aggregate(tlp_graph local, tlp_comm c,
+                                   const float *X_full, int64_t F, int64_t ldx,
+                                   int include_self, float *Y_full, int64_t ldy,
+                                   void *stream);
+tlp_status tlp_dist_gat_mh_aggregate(tlp_graph local, tlp_comm c,
+                                     const float *X_full, int64_t heads,
+                                     int64_t F, int64_t ldx, const float *el,
+                                     const float *er, float slope,
+                                     float *Y_full, int64_t ldy, void *stream);
 
 #ifdef __cplusplus
 }

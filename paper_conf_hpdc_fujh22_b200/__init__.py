@@ -70,6 +70,8 @@ _sig = {
     "tlp_gcn_aggregate": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_gin_aggregate": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
     "tlp_gat_aggregate": ([_P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
+    "tlp_sage_aggregate": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
+    "tlp_gat_mh_aggregate": ([_P, _P, _I64, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
     "tlp_graph_create_rows": ([_I64, _I64, _P, _P, _P, _I64, _I64, ctypes.POINTER(tlp_create_opts),
                                _P, ctypes.POINTER(_P)], _I),
     "tlp_partition_rows": ([_P, _I64, _I, _P], _I),
@@ -83,6 +85,8 @@ _sig = {
     "tlp_dist_gcn_aggregate": ([_P, _P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_dist_gin_aggregate": ([_P, _P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
     "tlp_dist_gat_aggregate": ([_P, _P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
+    "tlp_dist_sage_aggregate": ([_P, _P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
+    "tlp_dist_gat_mh_aggregate": ([_P, _P, _P, _I64, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
 }
 for _name, (_args, _res) in _sig.items():
     _fn = getattr(_lib, _name)
@@ -301,6 +305,29 @@ def tlp_gat_aggregate(g, X, el, er, slope=0.2, Y=None, F=None, stream=None, n_ds
     return Y
 
 
+def tlp_sage_aggregate(g, X, include_self=False, Y=None, F=None, stream=None, n_dst=None):
+    """GraphSage mean over N(v) (or N(v) + v with include_self)."""
+    X, F, ldx = _feat(X, F)
+    n = _n_dst(g) if n_dst is None else n_dst
+    Y, F, ldy = _out(Y, n, F, X)
+    _check(_lib.tlp_sage_aggregate(g, _ptr(X), F, ldx, int(bool(include_self)), _ptr(Y), ldy,
+                                   _stream(stream, X.device)), "tlp_sage_aggregate")
+    return Y
+
+
+def tlp_gat_mh_aggregate(g, X, el, er, heads, slope=0.2, Y=None, F=None, stream=None, n_dst=None):
+    """Multi-head GAT; el: [n_src, heads], er: [n_dst (+row_offset), heads] CUDA fp32."""
+    X, F, ldx = _feat(X, F)
+    el = _vec_cuda(el, "el")
+    er = _vec_cuda(er, "er")
+    n = _n_dst(g) if n_dst is None else n_dst
+    Y, F, ldy = _out(Y, n, F, X)
+    _check(_lib.tlp_gat_mh_aggregate(g, _ptr(X), int(heads), F, ldx, _ptr(el), _ptr(er),
+                                     float(slope), _ptr(Y), ldy, _stream(stream, X.device)),
+           "tlp_gat_mh_aggregate")
+    return Y
+
+
 # -------------------------------------------------------------- multi-GPU ----
 
 def tlp_partition_rows(rowptr, parts):
@@ -399,6 +426,26 @@ def tlp_dist_gat_aggregate(g, comm, X_full, Y_full, el, er, slope=0.2, F=None, s
     return Y_full
 
 
+def tlp_dist_sage_aggregate(g, comm, X_full, Y_full, include_self=False, F=None, stream=None):
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_full, F)
+    _check(_lib.tlp_dist_sage_aggregate(g, comm, _ptr(X), F, ldx, int(bool(include_self)), _ptr(Y),
+                                        ldy, _stream(stream, X.device)), "tlp_dist_sage_aggregate")
+    return Y_full
+
+
+def tlp_dist_gat_mh_aggregate(g, comm, X_full, Y_full, el, er, heads, slope=0.2, F=None,
+                              stream=None):
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_full, F)
+    el = _vec_cuda(el, "el")
+    er = _vec_cuda(er, "er")
+    _check(_lib.tlp_dist_gat_mh_aggregate(g, comm, _ptr(X), int(heads), F, ldx, _ptr(el), _ptr(er),
+                                          float(slope), _ptr(Y), ldy, _stream(stream, X.device)),
+           "tlp_dist_gat_mh_aggregate")
+    return Y_full
+
+
 # ------------------------------------------------------------ convenience ---
 
 class Graph:
@@ -428,6 +475,13 @@ class Graph:
 
     def gat(self, X, el, er, slope=0.2, Y=None, F=None, stream=None):
         return tlp_gat_aggregate(self.handle, X, el, er, slope, Y, F, stream, n_dst=self.n_dst)
+
+    def sage(self, X, include_self=False, Y=None, F=None, stream=None):
+        return tlp_sage_aggregate(self.handle, X, include_self, Y, F, stream, n_dst=self.n_dst)
+
+    def gat_mh(self, X, el, er, heads, slope=0.2, Y=None, F=None, stream=None):
+        return tlp_gat_mh_aggregate(self.handle, X, el, er, heads, slope, Y, F, stream,
+                                    n_dst=self.n_dst)
 
     def degrees(self):
         return tlp_graph_degrees(self.handle)

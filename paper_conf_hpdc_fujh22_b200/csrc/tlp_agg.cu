@@ -36,7 +36,9 @@
 
 namespace tlp {
 
-enum Op : int { OP_GCN = 0, OP_GIN = 1, OP_GAT = 2 };
+// OP_SAGE: GraphSage mean (optionally with the self row); OP_GATH: multi-head
+// GAT.
+enum Op : int { OP_GCN = 0, OP_GIN = 1, OP_GAT = 2, OP_SAGE = 3, OP_GATH = 4 };
 enum Coef : int { COEF_NONE = 0, COEF_COUT = 1, COEF_W = 2, COEF_W_COUT = 3 };
 enum Sched : int { S_DYNAMIC = 0, S_STATIC = 1, S_HARDWARE = 2 };
 
@@ -52,6 +54,9 @@ constexpr unsigned FULL = 0xffffffffu;
 #endif
 #ifndef TLP_MINB
 #define TLP_MINB 3     // register path: 3 CTAs/SM -> <= 85 registers, 24 warps/SM
+#endif
+#ifndef TLP_MHB
+#define TLP_MHB 4      // multi-head GAT: heads scored together per pass
 #endif
 #ifndef TLP_HINTS
 #define TLP_HINTS 0    // 1: L2 evict_first policy on per-edge streams and Y stores (measured: no gain)
@@ -80,6 +85,8 @@ struct AggArgs {
     int64_t ldx, ldy, ldp, row_offset, n_tasks, n_items, n_hubs, n_chunks, C;
     int F, n_strips, norm, step, sched, panel;
     float eps1, slope;
+    int sage_self;  // OP_SAGE: include X[v] in the mean
+    int heads, fh;  // OP_GATH: H heads of fh columns each (F = heads * fh)
 };
 
 template <int VEC>
@@ -517,6 +524,241 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
     for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
 }
 
+// ---- multi-head GAT (NEXT-1) -----------------------------------------------
+// Head h owns columns [h*fh, (h+1)*fh) (fh a multiple of VEC, so a lane's
+// vector lies in one head).  A strip of 32*VEC columns spans heads
+// [h_lo, h_lo+nh).  Per 32-edge chunk the warp computes, head by head, the
+// LeakyReLU scores, the online-softmax update (running max M, denominator D,
+// rescale S) and the weights p[j], kept in a per-warp shared-memory block;
+// each lane then gathers with the weights of its own head.  Scores never
+// leave the SM.  Reduction order: the canonical two chains per head.
+constexpr int kMhMaxHeads = 33;  // heads one strip can touch (fh >= VEC)
+constexpr int kMhWarpFloats = kMhMaxHeads * 32 + 3 * kMhMaxHeads + 1;  // P, M, D, S (+pad)
+
+__device__ __forceinline__ float *mh_warp_smem() {
+    extern __shared__ __align__(16) float tlp_smem[];
+    return tlp_smem + (size_t)(threadIdx.x >> 5) * kMhWarpFloats;
+}
+
+// Scores, online-softmax update and weights of one 32-edge chunk for the heads
+// [h_lo, h_lo+nh) of a strip (lane j holds edge j with source u_l).  Heads are
+// processed TLP_MHB at a time so their el loads and warp reductions overlap.
+__device__ __forceinline__ void mh_chunk_scores(const AggArgs &a, int u_l, int n0, int H, int h_lo,
+                                                int nh, const float *__restrict__ erv, int lane,
+                                                float *P, float *M, float *D, float *S) {
+    constexpr int B = TLP_MHB;
+    const float *__restrict__ elu = a.el + (size_t)((unsigned)u_l) * H + h_lo;
+    for (int hb = 0; hb < nh; hb += B) {
+        float sv[B], mo[B], mn[B], sm[B];
+#pragma unroll
+        for (int k = 0; k < B; ++k) {
+            sv[k] = -INFINITY;
+            if (hb + k < nh && lane < n0) {
+                const float t = __ldg(elu + hb + k) + __ldg(erv + hb + k);
+                sv[k] = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < B; ++k) {
+            if (hb + k < nh) {  // warp-uniform
+                mo[k] = M[hb + k];
+                mn[k] = fmaxf(mo[k], warp_max(sv[k]));
+                const float p = (lane < n0) ? __expf(sv[k] - mn[k]) : 0.f;
+                sm[k] = warp_sum(p);
+                P[(hb + k) * 32 + lane] = p;
+            }
+        }
+        __syncwarp();
+        if (lane == 0) {
+#pragma unroll
+            for (int k = 0; k < B; ++k)
+                if (hb + k < nh) {
+                    const float scale = __expf(mo[k] - mn[k]);
+                    M[hb + k] = mn[k];
+                    D[hb + k] = fmaf(D[hb + k], scale, sm[k]);
+                    S[hb + k] = scale;
+                }
+        }
+        __syncwarp();
+    }
+}
+
+// A lane's VEC columns [col, col+VEC) lie in at most two heads (fh >= VEC):
+// head slot hl for components c < split, hl + 1 for the rest.
+template <int VEC, int U>
+__device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, int64_t e1, int s,
+                                                int col, bool active, int64_t rglob, int lane,
+                                                Vec<VEC> &acc, float *&Mh, float *&Dh, int &h_lo,
+                                                int &nh, int &hl, int &split) {
+    float *P = mh_warp_smem();
+    float *M = P + kMhMaxHeads * 32;
+    float *D = M + kMhMaxHeads;
+    float *S = D + kMhMaxHeads;
+    Mh = M;
+    Dh = D;
+    const int H = a.heads, fh = a.fh;
+    const int c_lo = s * 32 * VEC;
+    const int c_hi = min(a.F, c_lo + 32 * VEC) - 1;
+    h_lo = c_lo / fh;
+    nh = c_hi / fh - h_lo + 1;
+    const int cc = active ? col : c_lo;
+    hl = cc / fh - h_lo;
+    split = (hl + h_lo + 1) * fh - cc;                 // components in head hl
+    const int hl2 = min(hl + (split < VEC ? 1 : 0), nh - 1);
+    for (int hh = lane; hh < nh; hh += 32) {
+        M[hh] = -INFINITY;
+        D[hh] = 0.f;
+    }
+    __syncwarp();
+    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
+    const unsigned row_bytes = (unsigned)a.ldx * 4u;
+    const int32_t *__restrict__ ci = a.colidx + e0;
+    const float *__restrict__ erv = a.er + rglob * H + h_lo;
+    const int len = (int)(e1 - e0);
+    Vec<VEC> ac[2];
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) ac[0].v[c] = ac[1].v[c] = 0.f;
+    for (int off = 0; off < len; off += 32) {
+        const int n0 = min(32, len - off);
+        const int u_l = (lane < n0) ? __ldg(ci + off + lane) : 0;
+        mh_chunk_scores(a, u_l, n0, H, h_lo, nh, erv, lane, P, M, D, S);
+        const float sA = S[hl], sB = S[hl2];
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) {
+            const float sc = (c < split) ? sA : sB;
+            ac[0].v[c] *= sc;
+            ac[1].v[c] *= sc;
+        }
+        const float *pa = P + hl * 32;
+        const float *pb = P + hl2 * 32;
+        for (int j = 0; j < n0; j += 2 * U) {
+            Vec<VEC> xv[2 * U];
+            float ca[2 * U], cb[2 * U];
+#pragma unroll
+            for (int k = 0; k < 2 * U; ++k) {
+                const int jj = min(j + k, n0 - 1);
+                const unsigned u = (unsigned)__shfl_sync(FULL, u_l, jj);
+                ca[k] = pa[jj];
+                cb[k] = pb[jj];
+                xv[k] = ld_vec<VEC>(row_ptr(base, u, row_bytes));
+            }
+#pragma unroll
+            for (int k = 0; k < 2 * U; ++k)
+                if (j + k < n0) {
+#pragma unroll
+                    for (int c = 0; c < VEC; ++c)
+                        ac[k & 1].v[c] = fmaf(c < split ? ca[k] : cb[k], xv[k].v[c], ac[k & 1].v[c]);
+                }
+        }
+        __syncwarp();  // P, S are rewritten by the next chunk
+    }
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) acc.v[c] = ac[0].v[c] + ac[1].v[c];
+}
+
+// Multi-head GAT with the cp.async ring (gathers that stream from HBM): the
+// per-warp shared memory holds the head block followed by a D-deep ring.
+template <int VEC>
+__device__ __forceinline__ float *mh_warp_ring() {
+    extern __shared__ __align__(16) float tlp_smem[];
+    constexpr int stride = kMhWarpFloats + TLP_DEPTH * 32 * VEC;
+    return tlp_smem + (size_t)(threadIdx.x >> 5) * stride + kMhWarpFloats;
+}
+template <int VEC>
+__device__ __forceinline__ float *mh_warp_smem_async() {
+    extern __shared__ __align__(16) float tlp_smem[];
+    constexpr int stride = kMhWarpFloats + TLP_DEPTH * 32 * VEC;
+    return tlp_smem + (size_t)(threadIdx.x >> 5) * stride;
+}
+
+template <int VEC>
+__device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t e0, int64_t e1,
+                                                      int s, int col, bool active, int64_t rglob,
+                                                      int lane, Vec<VEC> &acc, float *&Mh,
+                                                      float *&Dh, int &h_lo, int &nh, int &hl,
+                                                      int &split) {
+    constexpr int DD = TLP_DEPTH;
+    float *P = mh_warp_smem_async<VEC>();
+    float *M = P + kMhMaxHeads * 32;
+    float *Dn = M + kMhMaxHeads;
+    float *S = Dn + kMhMaxHeads;
+    Mh = M;
+    Dh = Dn;
+    const int H = a.heads, fh = a.fh;
+    const int c_lo = s * 32 * VEC;
+    const int c_hi = min(a.F, c_lo + 32 * VEC) - 1;
+    h_lo = c_lo / fh;
+    nh = c_hi / fh - h_lo + 1;
+    const int cc = active ? col : c_lo;
+    hl = cc / fh - h_lo;
+    split = (hl + h_lo + 1) * fh - cc;
+    const int hl2 = min(hl + (split < VEC ? 1 : 0), nh - 1);
+    for (int hh = lane; hh < nh; hh += 32) {
+        M[hh] = -INFINITY;
+        Dn[hh] = 0.f;
+    }
+    __syncwarp();
+    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
+    const unsigned row_bytes = (unsigned)a.ldx * 4u;
+    const int32_t *__restrict__ ci = a.colidx + e0;
+    const float *__restrict__ erv = a.er + rglob * H + h_lo;
+    const int len = (int)(e1 - e0);
+    Vec<VEC> ae, ao;
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) ae.v[c] = ao.v[c] = 0.f;
+    if (len > 0) {
+        float *ring = mh_warp_ring<VEC>() + lane * VEC;
+        int n0 = min(32, len), n1 = min(32, len - 32);
+        int u0 = (lane < n0) ? __ldg(ci + lane) : 0;
+        int u1 = (lane < n1) ? __ldg(ci + 32 + lane) : 0;
+#pragma unroll
+        for (int k = 0; k < DD - 1; ++k) {
+            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
+            cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
+            cp_async_commit();
+        }
+        int slot = 0, off = 0;
+        while (true) {
+            const int n2 = min(32, len - off - 64);
+            const int u2 = (lane < n2) ? __ldg(ci + off + 64 + lane) : 0;
+            mh_chunk_scores(a, u0, n0, H, h_lo, nh, erv, lane, P, M, Dn, S);
+            const float sA = S[hl], sB = S[hl2];
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) {
+                const float sc = (c < split) ? sA : sB;
+                ae.v[c] *= sc;
+                ao.v[c] *= sc;
+            }
+            const float *pa = P + hl * 32;
+            const float *pb = P + hl2 * 32;
+            for (int j = 0; j < n0; ++j) {
+                const int jj = j + DD - 1;
+                const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
+                int ws = slot + DD - 1;
+                if (ws >= DD) ws -= DD;
+                cp_async_vec<VEC>(ring + ws * 32 * VEC, row_ptr(base, (unsigned)ui, row_bytes),
+                                  active && (off + jj) < len);
+                cp_async_commit();
+                cp_async_wait<DD - 1>();
+                const float ca = pa[j], cb = pb[j];
+                const float *src = ring + slot * 32 * VEC;
+                Vec<VEC> &ac = (j & 1) ? ao : ae;
+#pragma unroll
+                for (int c = 0; c < VEC; ++c) ac.v[c] = fmaf(c < split ? ca : cb, src[c], ac.v[c]);
+                if (++slot == DD) slot = 0;
+            }
+            __syncwarp();  // P, S are rewritten by the next chunk
+            if (n1 <= 0) break;
+            off += 32;
+            n0 = n1; n1 = n2;
+            u0 = u1; u1 = u2;
+        }
+        cp_async_wait<0>();
+    }
+#pragma unroll
+    for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
+}
+
 // Epilogue (a9) for a full row reduction.
 template <int VEC, int OP>
 __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_t deg, int col,
@@ -538,6 +780,16 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_
         }
 #pragma unroll
         for (int c = 0; c < VEC; ++c) y.v[c] = fmaf(a.eps1, xs.v[c], acc.v[c]);
+    } else if constexpr (OP == OP_SAGE) {
+        // mean over N(v) (+ v itself when sage_self): (X[v] + sum) / (deg + 1)
+        const int64_t cnt = deg + a.sage_self;
+        const float inv = 1.0f / (float)(cnt > 1 ? cnt : 1);
+        Vec<VEC> xs;
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) xs.v[c] = 0.f;
+        if (a.sage_self && active) xs = ld_vec<VEC>(a.X + (a.row_offset + r) * a.ldx + col);
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) y.v[c] = (xs.v[c] + acc.v[c]) * inv;
     } else {
 #pragma unroll
         for (int c = 0; c < VEC; ++c) y.v[c] = deg > 0 ? acc.v[c] / den : 0.f;
@@ -582,10 +834,28 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
 #pragma unroll
                 for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
                 float m = -INFINITY, den = 0.f;
-                if constexpr (ASYNC)
+                if constexpr (OP == OP_GATH) {
+                    float *Mh, *Dh;
+                    int h_lo, nh, hl, split;
+                    if constexpr (ASYNC)
+                        reduce_edges_mh_async<VEC>(a, e0, e1, s, col, active, a.row_offset + r, lane,
+                                                   acc, Mh, Dh, h_lo, nh, hl, split);
+                    else
+                        reduce_edges_mh<VEC, U>(a, e0, e1, s, col, active, a.row_offset + r, lane, acc,
+                                                Mh, Dh, h_lo, nh, hl, split);
+                    const float dA = Dh[hl], dB = Dh[min(hl + 1, nh - 1)];
+                    __syncwarp();  // the head state is reset by the next strip / row
+                    Vec<VEC> y;
+#pragma unroll
+                    for (int c = 0; c < VEC; ++c)
+                        y.v[c] = (e1 > e0) ? acc.v[c] / (c < split ? dA : dB) : 0.f;
+                    if (active) st_row<VEC>(yrow, col, a.F, y);
+                    continue;
+                } else if constexpr (ASYNC) {
                     reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
-                else
+                } else {
                     reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+                }
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
                 if (active && stores<PAIR>(lane)) st_row<VEC>(yrow, col, a.F, y);
             }
@@ -608,7 +878,9 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     float er_v = 0.f;
     if constexpr (OP == OP_GAT) er_v = __ldg(a.er + a.row_offset + r);
     const int slot = off + j;
-    float *md = a.md + 2 * (int64_t)s0 * a.n_chunks;  // this panel's (m, den) pairs
+    // this panel's (m, den) pairs: [n_chunks][heads] (heads = 1 unless OP_GATH)
+    const int mdh = (OP == OP_GATH) ? a.heads : 1;
+    float *md = a.md + 2 * (int64_t)s0 * a.n_chunks * mdh;
     int32_t *ticket = a.hub_ticket + (int64_t)s0 * a.n_hubs + h;
     for (int s = s0; s < s1; ++s) {
         const int col = strip_col<VEC, PAIR>(s, lane);
@@ -617,10 +889,25 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
 #pragma unroll
         for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
         float m = -INFINITY, den = 0.f;
-        if constexpr (ASYNC)
-                    reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
-                else
-                    reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+        if constexpr (OP == OP_GATH) {
+            float *Mh, *Dh;
+            int h_lo, nh, hl, split;
+            if constexpr (ASYNC)
+                reduce_edges_mh_async<VEC>(a, e0, e1, s, col, active, a.row_offset + r, lane, acc, Mh,
+                                           Dh, h_lo, nh, hl, split);
+            else
+                reduce_edges_mh<VEC, U>(a, e0, e1, s, col, active, a.row_offset + r, lane, acc, Mh, Dh,
+                                        h_lo, nh, hl, split);
+            for (int hh = lane; hh < nh; hh += 32) {
+                md[2 * ((int64_t)slot * mdh + h_lo + hh)] = Mh[hh];
+                md[2 * ((int64_t)slot * mdh + h_lo + hh) + 1] = Dh[hh];
+            }
+            __syncwarp();
+        } else if constexpr (ASYNC) {
+            reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+        } else {
+            reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den);
+        }
         if (active && stores<PAIR>(lane)) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
         if constexpr (OP == OP_GAT)
             if (s == s0 && lane == 0) {
@@ -648,13 +935,38 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     for (int s = s0; s < s1; ++s) {
         const int col = strip_col<VEC, PAIR>(s, lane);
         const bool active = col < a.F;
+        // OP_GATH: the lane's (up to two) heads and their merged softmax states
+        int64_t mA = 0, mB = 0;
+        int split = VEC;
+        float MA = -INFINITY, DA = 0.f, MB = -INFINITY, DB = 0.f;
+        if constexpr (OP == OP_GATH) {
+            const int cc = active ? col : s * 32 * VEC;
+            mA = cc / a.fh;
+            split = (int)((mA + 1) * a.fh - cc);
+            mB = min(mA + (split < VEC ? 1 : 0), (int64_t)a.heads - 1);
+            for (int q = 0; q < nch; ++q) {
+                MA = fmaxf(MA, __ldcg(md + 2 * ((int64_t)(off + q) * mdh + mA)));
+                MB = fmaxf(MB, __ldcg(md + 2 * ((int64_t)(off + q) * mdh + mB)));
+            }
+            for (int q = 0; q < nch; ++q) {
+                const float *pa = md + 2 * ((int64_t)(off + q) * mdh + mA);
+                const float *pb = md + 2 * ((int64_t)(off + q) * mdh + mB);
+                DA = fmaf(__ldcg(pa + 1), __expf(__ldcg(pa) - MA), DA);
+                DB = fmaf(__ldcg(pb + 1), __expf(__ldcg(pb) - MB), DB);
+            }
+        }
         Vec<VEC> acc;
 #pragma unroll
         for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
         if (active) {
             for (int q = 0; q < nch; ++q) {
                 Vec<VEC> p = ld_vec_cg<VEC>(a.scratch + (int64_t)(off + q) * a.ldp + col);
-                if constexpr (OP == OP_GAT) {
+                if constexpr (OP == OP_GATH) {
+                    const float wA = __expf(__ldcg(md + 2 * ((int64_t)(off + q) * mdh + mA)) - MA);
+                    const float wB = __expf(__ldcg(md + 2 * ((int64_t)(off + q) * mdh + mB)) - MB);
+#pragma unroll
+                    for (int c = 0; c < VEC; ++c) acc.v[c] = fmaf(c < split ? wA : wB, p.v[c], acc.v[c]);
+                } else if constexpr (OP == OP_GAT) {
                     const float w = __expf(__ldcg(md + 2 * (int64_t)(off + q)) - M);
 #pragma unroll
                     for (int c = 0; c < VEC; ++c) acc.v[c] = fmaf(w, p.v[c], acc.v[c]);
@@ -664,7 +976,13 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
                 }
             }
         }
-        Vec<VEC> y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
+        Vec<VEC> y;
+        if constexpr (OP == OP_GATH) {
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] / (c < split ? DA : DB);
+        } else {
+            y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
+        }
         if (active && stores<PAIR>(lane)) st_row<VEC>(yrow, col, a.F, y);
     }
     if (lane == 0) *ticket = 0;  // self-reset for the next launch
@@ -736,7 +1054,19 @@ static KernelFn pick(int op, int coef) {
     if (op == OP_GIN)
         return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC, PAIR>
                              : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC, PAIR>;
+    if (op == OP_SAGE) return k_agg<VEC, OP_SAGE, COEF_NONE, kU, ASYNC, PAIR>;
     return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC, PAIR>;
+}
+
+// multi-head GAT: full-warp register path or cp.async ring
+static KernelFn pick_mh(int vec, bool async_path) {
+    if (async_path)
+        return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, true, false>
+                        : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, true, false>
+                                   : k_agg<1, OP_GATH, COEF_NONE, kU, true, false>;
+    return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, false, false>
+                    : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, false, false>
+                               : k_agg<1, OP_GATH, COEF_NONE, kU, false, false>;
 }
 
 // gather path: 0 register (full warp), 1 cp.async ring, 2 register half-warp PAIR (VEC = 4)
@@ -786,10 +1116,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         return set_error(TLP_ERR_INVALID_ARGUMENT, "X and Y must be 4-byte aligned");
     if (r.op == OP_GCN && (r.norm < TLP_NORM_NONE || r.norm > TLP_NORM_BOTH))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown norm");
-    if (r.op == OP_GIN && g->row_offset + g->n_dst > g->n_src)
-        return set_error(TLP_ERR_INVALID_ARGUMENT, "GIN needs row_offset + n_dst <= n_src");
-    if (r.op == OP_GAT && (!r.el || !r.er))
+    if ((r.op == OP_GIN || (r.op == OP_SAGE && r.sage_self)) && g->row_offset + g->n_dst > g->n_src)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "the self term needs row_offset + n_dst <= n_src");
+    if ((r.op == OP_GAT || r.op == OP_GATH) && (!r.el || !r.er))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "GAT needs el and er");
+    if (r.op == OP_GATH && (r.heads < 1 || r.F % r.heads != 0))
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "multi-head GAT needs F = heads * head_dim");
     {
         const char *x0 = (const char *)r.X;
         const char *x1 = x0 + sizeof(float) * ((g->n_src ? g->n_src - 1 : 0) * r.ldx + r.F);
@@ -802,6 +1134,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     int vec = 1;
     if (r.ldx % 4 == 0 && r.ldy % 4 == 0 && aligned(r.X, 16) && aligned(r.Y, 16)) vec = 4;
     else if (r.ldx % 2 == 0 && r.ldy % 2 == 0 && aligned(r.X, 8) && aligned(r.Y, 8)) vec = 2;
+    const int fh = (r.op == OP_GATH) ? (int)(r.F / r.heads) : 0;
+    if (r.op == OP_GATH)  // a lane's vector may straddle at most two heads
+        while (vec > fh) vec >>= 1;
 
     // Edge coefficients.  GCN BOTH streams the per-edge product
     // c_out[colidx[e]] * w_e precomputed at create (the same fp32 value the
@@ -834,7 +1169,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             panel_off = true;
         } else if (mode == 128 && vec == 4) {
             panel = 1;
-        } else if (mode == 64 && vec == 4) {
+        } else if (mode == 64 && vec == 4 && r.op != OP_GATH) {
             panel = 1;
             pair = 1;
         } else if (mode == 64 && vec == 2) {
@@ -845,7 +1180,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         } else if (xbytes > budget && vec == 4) {
             // GAT recomputes its scores and online-softmax state per strip, so it
             // keeps the wider 128-column strips (measured)
-            if (r.op != OP_GAT && 256.0 * g->n_src <= budget) { panel = 1; pair = 1; }
+            if (r.op != OP_GAT && r.op != OP_GATH && 256.0 * g->n_src <= budget) { panel = 1; pair = 1; }
             else if (512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
         }
     }
@@ -885,6 +1220,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.norm = r.norm;
     a.eps1 = 1.0f + r.eps;
     a.slope = r.slope;
+    a.sage_self = r.sage_self;
+    a.heads = (int)r.heads;
+    a.fh = fh;
     a.scratch = nullptr;
     a.md = nullptr;
     a.hub_ticket = nullptr;
@@ -892,7 +1230,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         // scratch = [partials n_chunks x ldp][(m,den) 2 x n_chunks x panels][tickets n_hubs x panels]
         const int np = panel ? n_strips : 1;
         const size_t part = (size_t)g->n_chunks * a.ldp;
-        const size_t mdn = 2 * (size_t)g->n_chunks * np;
+        const size_t mdn = 2 * (size_t)g->n_chunks * np * (r.op == OP_GATH ? (size_t)r.heads : 1);
         const size_t tick_off = (part + mdn) * sizeof(float);
         const size_t tick_n = (size_t)g->n_hubs * np;
         const size_t need = tick_off + tick_n * sizeof(int32_t) + 64;
@@ -940,10 +1278,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     }
     if (pair) async_path = false;
     const int path = pair ? 2 : (async_path ? 1 : 0);
-    KernelFn fn = pick_kernel(path, vec, r.op, coef);
+    KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, r.op, coef);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
-    const size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;
+    size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;
+    if (r.op == OP_GATH)
+        smem = (size_t)wpc * (kMhWarpFloats + (async_path ? TLP_DEPTH * 32 * vec : 0)) * sizeof(float);
     if (smem > 0 && sched == S_HARDWARE) occupancy_blocks(fn, threads, smem);  // sets attributes
     int64_t blocks;
     if (sched == S_HARDWARE) {
@@ -990,6 +1330,24 @@ tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F, int64_t ldx
     r.op = OP_GAT;
     r.X = X; r.F = F; r.ldx = ldx; r.Y = Y; r.ldy = ldy;
     r.el = el; r.er = er; r.slope = slope;
+    return aggregate(g, r, (cudaStream_t)stream);
+}
+
+tlp_status tlp_sage_aggregate(tlp_graph g, const float *X, int64_t F, int64_t ldx, int include_self,
+                              float *Y, int64_t ldy, void *stream) {
+    AggRequest r;
+    r.op = OP_SAGE;
+    r.X = X; r.F = F; r.ldx = ldx; r.Y = Y; r.ldy = ldy; r.sage_self = include_self ? 1 : 0;
+    return aggregate(g, r, (cudaStream_t)stream);
+}
+
+tlp_status tlp_gat_mh_aggregate(tlp_graph g, const float *X, int64_t heads, int64_t F, int64_t ldx,
+                                const float *el, const float *er, float slope, float *Y, int64_t ldy,
+                                void *stream) {
+    AggRequest r;
+    r.op = OP_GATH;
+    r.X = X; r.F = F; r.ldx = ldx; r.Y = Y; r.ldy = ldy;
+    r.el = el; r.er = er; r.slope = slope; r.heads = heads;
     return aggregate(g, r, (cudaStream_t)stream);
 }
 

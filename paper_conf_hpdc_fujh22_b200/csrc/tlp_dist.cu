@@ -242,4 +242,22 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph g, tlp_comm c, const float *X_full, 
     return dist_local(g, c, r, stream);
 }
 
+tlp_status tlp_dist_sage_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t F,
+                                   int64_t ldx, int include_self, float *Y_full, int64_t ldy,
+                                   void *stream) {
+    AggRequest r;
+    r.op = 3; r.X = X_full; r.F = F; r.ldx = ldx; r.Y = Y_full; r.ldy = ldy;
+    r.sage_self = include_self ? 1 : 0;
+    return dist_local(g, c, r, stream);
+}
+
+tlp_status tlp_dist_gat_mh_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t heads,
+                                     int64_t F, int64_t ldx, const float *el, const float *er,
+                                     float slope, float *Y_full, int64_t ldy, void *stream) {
+    AggRequest r;
+    r.op = 4; r.X = X_full; r.F = F; r.ldx = ldx; r.Y = Y_full; r.ldy = ldy;
+    r.el = el; r.er = er; r.slope = slope; r.heads = heads;
+    return dist_local(g, c, r, stream);
+}
+
 }  // extern "C"

@@ -87,7 +87,8 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
 
 tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s);
 
-// Enqueue one aggregation kernel; op: 0 GCN, 1 GIN, 2 GAT.
+// Enqueue one aggregation kernel; op: 0 GCN, 1 GIN, 2 GAT, 3 GraphSage mean,
+// 4 multi-head GAT.
 struct AggRequest {
     int op = 0;
     const float *X = nullptr;
@@ -98,6 +99,8 @@ struct AggRequest {
     float eps = 0.f;
     const float *el = nullptr, *er = nullptr;
     float slope = 0.f;
+    int sage_self = 0;  // op 3 (GraphSage mean): include the self row
+    int64_t heads = 1;  // op 4 (multi-head GAT)
 };
 tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s);
 

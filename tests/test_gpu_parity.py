@@ -493,3 +493,92 @@ def test_compute_sanitizer(tool):
         args += ["--kernel-name", "kns=k_"]
     r = subprocess.run(args + [sys.executable, tgt], capture_output=True, text=True, timeout=1500)
     assert r.returncode == 0 and "sanitize target ok" in r.stdout, r.stdout[-3000:] + r.stderr[-3000:]
+
+
+# ------------------------------------------------------------ NEXT-1 ---------
+
+@pytest.mark.parametrize("name", ["random64", "powerlaw_hubs", "selfloops_multi", "isolated_last", "e0_n5"])
+@pytest.mark.parametrize("include_self", [False, True])
+def test_sage_edge_cases(tlp, name, include_self):
+    rp, ci, n_src = _edge_graphs()[name]
+    F, ld = 37, 40
+    Xh = synth.features(n_src, F, ld, seed=2)
+    g = tlp.Graph(_t(rp), _t(ci), n_src=n_src, opts=dict(hub_threshold=64, hub_chunk=32))
+    Y = torch.full((len(rp) - 1, ld), float("nan"), device=DEV)
+    g.sage(_t(Xh), include_self, Y=Y, F=F)
+    _check("sage", Y[:, :F], oracle.sage(rp, ci, Xh, include_self=include_self, F=F))
+    assert torch.isnan(Y[:, F:]).all()
+    g.close()
+
+
+def test_sage_reddit_sampled_and_equals_gcn_right(tlp, reddit):
+    cfg = synth.CONFIGS["reddit"]
+    n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+    rp, ci = reddit
+    Xh = synth.features(n, F, ld, seed=103)
+    g = tlp.Graph(_t(rp), _t(ci))
+    X = _t(Xh)
+    rows = _sample_rows(rp, 300, 40, 9)
+    Ys = g.sage(X, True, F=F)
+    _check("reddit sage+self", Ys[_t(rows)], oracle.sage(rp, ci, Xh, include_self=True, rows=rows, F=F))
+    # mean without self is the RIGHT-normalised GCN: same canonical sum, same scaling
+    assert torch.equal(g.sage(X, False, F=F), g.gcn(X, "right", F=F))
+    g.close()
+
+
+@pytest.mark.parametrize("path", ["reg", "async"])
+@pytest.mark.parametrize("H,Fh,ld", [(1, 37, 40), (2, 16, 32), (4, 8, 32), (8, 4, 32),
+                                     (3, 5, 15), (4, 50, 200), (6, 100, 600), (33, 4, 132),
+                                     (4, 25, 100), (3, 3, 9), (5, 6, 30)])
+def test_gat_mh_parity(tlp, monkeypatch, H, Fh, ld, path):
+    monkeypatch.setenv("TLP_GATHER", path)
+    n = 700
+    rp, ci = synth.chung_lu(n, 14000, 0.55, 21, device="cpu")
+    F = H * Fh
+    Xh = synth.features(n, F, ld, seed=H)
+    el = (synth.normal(n * H, 31) * 1.5).reshape(n, H)
+    er = (synth.normal(n * H, 32) * 1.5).reshape(n, H)
+    for opts in (dict(hub_threshold=64, hub_chunk=32), None):
+        g = tlp.Graph(_t(rp), _t(ci), opts=opts)
+        Y = torch.full((n, ld), float("nan"), device=DEV)
+        g.gat_mh(_t(Xh), _t(el), _t(er), H, 0.2, Y=Y, F=F)
+        _check(f"gat_mh H={H}", Y[:, :F], oracle.gat_mh(rp, ci, Xh, el, er, H, 0.2, Fh=Fh))
+        if ld > F:
+            assert torch.isnan(Y[:, F:]).all()
+        g.close()
+
+
+def test_gat_mh_one_head_equals_gat_and_panels(tlp, monkeypatch):
+    n = 3000
+    rp, ci = synth.chung_lu(n, 80000, 0.5, 23, device="cpu")
+    F = 256
+    X = _t(synth.features(n, F, F, seed=3))
+    el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    y1 = g.gat(X, el, er, 0.2)
+    assert torch.equal(g.gat_mh(X, el.view(n, 1), er.view(n, 1), 1, 0.2), y1)
+    H = 4
+    elh = _t(synth.normal(n * H, 5).reshape(n, H))
+    erh = _t(synth.normal(n * H, 6).reshape(n, H))
+    outs = []
+    for mode in ("0", "128", "-1"):
+        monkeypatch.setenv("TLP_PANEL", mode)
+        outs.append(g.gat_mh(X, elh, erh, H, 0.2).clone())
+    assert torch.equal(outs[0], outs[1]) and torch.equal(outs[0], outs[2])
+    g.close()
+
+
+def test_products_gat_mh_sampled(tlp):
+    """ogbn-products-shaped graph, 4 heads of 25 columns (F = 100)."""
+    cfg = synth.CONFIGS["products"]
+    n, F = cfg["n"], cfg["F"]
+    H = 4
+    rp, ci = synth.dataset_graph("products")
+    Xh = synth.dataset_features("products", n)
+    el = synth.normal(n * H, 501).reshape(n, H)
+    er = synth.normal(n * H, 502).reshape(n, H)
+    g = tlp.Graph(_t(rp), _t(ci))
+    rows = _sample_rows(rp, 2000, 40, 7)
+    Y = g.gat_mh(_t(Xh), _t(el), _t(er), H, synth.SLOPE, F=F)
+    _check("products gat_mh", Y[_t(rows)], oracle.gat_mh(rp, ci, Xh, el, er, H, synth.SLOPE, rows=rows, Fh=F // H))
+    g.close()
