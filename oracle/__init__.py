@@ -71,6 +71,8 @@ def _load():
         lib.oracle_gat_mh.argtypes = [I64, I64, P, P, P, I64, I64, I64, P, P, ctypes.c_double,
                                       I64, I64, P, P, P]
         lib.oracle_gat_mh.restype = ctypes.c_int
+        lib.oracle_epilogue.argtypes = [I64, I64, P, P, P, ctypes.c_int, ctypes.c_double]
+        lib.oracle_epilogue.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -223,6 +225,21 @@ def gat_mh(rowptr, colidx, X, el, er, heads, slope, rows=None, row_offset=0, Fh=
                                _ptr(Y), _ptr(A))
     if rc:
         raise ValueError("oracle_gat_mh: bad arguments")
+    return Y, A
+
+
+ACTS = {"none": 0, "relu": 1, "leaky_relu": 2, "elu": 3}
+
+
+def epilogue(Y, A, bias=None, act="none", param=0.0):
+    """Layer epilogue h' = act(Y + bias) applied to oracle outputs (returns copies)."""
+    Y = np.ascontiguousarray(Y, dtype=np.float64).copy()
+    A = np.ascontiguousarray(A, dtype=np.float64).copy()
+    n, F = Y.shape
+    b = None if bias is None else np.ascontiguousarray(bias, dtype=np.float32)
+    rc = _load().oracle_epilogue(n, F, _ptr(Y), _ptr(A), _ptr(b), ACTS.get(act, act), float(param))
+    if rc:
+        raise ValueError("oracle_epilogue: bad arguments")
     return Y, A
 
 

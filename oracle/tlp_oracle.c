@@ -358,3 +358,35 @@ int oracle_gat_mh(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
     }
     return 0;
 }
+
+/* ---- NEXT-3: the layer epilogue of Eq. 2 ---------------------- */
+
+/* h' = sigma(a + b) (Eq. 2; bias and activation of the layer).
+ * act: 0 identity, 1 ReLU max(x,0), 2 LeakyReLU (x >= 0 ? x : p*x),
+ *      3 ELU (x > 0 ? x : p*(exp(x)-1)).  bias may be NULL.  In place on Y
+ * [n_rows x F]; the bound term A gains the bias as one more term (|b|), and the
+ * activations used here are 1-Lipschitz for 0 <= p <= 1, so A bounds them too. */
+int oracle_epilogue(int64_t n_rows, int64_t F, double *Y, double *A,
+                    const float *bias, int act, double p)
+{
+    if (act < 0 || act > 3 || F < 0)
+        return -1;
+    for (int64_t i = 0; i < n_rows; ++i) {
+        for (int64_t f = 0; f < F; ++f) {
+            double x = Y[i * F + f];
+            if (bias) {
+                x += (double)bias[f];
+                if (A)
+                    A[i * F + f] += fabs((double)bias[f]);
+            }
+            if (act == 1)
+                x = x > 0.0 ? x : 0.0;
+            else if (act == 2)
+                x = x >= 0.0 ? x : p * x;
+            else if (act == 3)
+                x = x > 0.0 ? x : p * (exp(x) - 1.0);
+            Y[i * F + f] = x;
+        }
+    }
+    return 0;
+}

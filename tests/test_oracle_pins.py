@@ -453,3 +453,36 @@ def test_p4_gat_mh_one_head_and_head_permutation(pub):
     Xp = np.concatenate([X[:, p * Fh:(p + 1) * Fh] for p in perm], axis=1)
     Yp = oracle.gat_mh(rp, ci, Xp, el[:, perm], er[:, perm], H, 0.2)[0]
     np.testing.assert_array_equal(Yp, np.concatenate([Y[:, p * Fh:(p + 1) * Fh] for p in perm], axis=1))
+
+
+# ---------------------------------------------------- NEXT-3: layer epilogue ---
+
+def test_epilogue_closed_forms():
+    Y = np.array([[-2.0, -0.5, 0.0, 0.5, 3.0]])
+    A = np.abs(Y)
+    b = np.array([0.5, 0.5, 0.0, -1.0, 0.0], np.float32)
+    # identity without bias is a no-op
+    Yi, Ai = oracle.epilogue(Y, A)
+    assert np.array_equal(Yi, Y) and np.array_equal(Ai, A)
+    # bias only: y + b, bound gains |b|
+    Yb, Ab = oracle.epilogue(Y, A, bias=b)
+    assert Yb.tolist() == [[-1.5, 0.0, 0.0, -0.5, 3.0]]
+    assert Ab.tolist() == [[2.5, 1.0, 0.0, 1.5, 3.0]]
+    # ReLU, LeakyReLU(0.1), ELU(1.0) worked by hand on y + b
+    assert oracle.epilogue(Y, A, b, "relu")[0].tolist() == [[0.0, 0.0, 0.0, 0.0, 3.0]]
+    np.testing.assert_allclose(oracle.epilogue(Y, A, b, "leaky_relu", 0.1)[0],
+                               [[-0.15, 0.0, 0.0, -0.05, 3.0]], rtol=1e-15)
+    np.testing.assert_allclose(oracle.epilogue(Y, A, b, "elu", 1.0)[0],
+                               [[math.exp(-1.5) - 1, 0.0, 0.0, math.exp(-0.5) - 1, 3.0]], rtol=1e-15)
+
+
+def test_epilogue_matches_numpy_definitions():
+    rng = np.random.default_rng(3)
+    Y = rng.standard_normal((50, 7))
+    A = np.abs(Y) + 1
+    b = rng.standard_normal(7).astype(np.float32)
+    x = Y + b.astype(np.float64)
+    np.testing.assert_array_equal(oracle.epilogue(Y, A, b, "relu")[0], np.maximum(x, 0))
+    np.testing.assert_array_equal(oracle.epilogue(Y, A, b, "leaky_relu", 0.2)[0], np.where(x >= 0, x, 0.2 * x))
+    np.testing.assert_allclose(oracle.epilogue(Y, A, b, "elu", 0.7)[0], np.where(x > 0, x, 0.7 * np.expm1(x)),
+                               rtol=1e-14, atol=1e-16)
