@@ -83,6 +83,44 @@ typedef enum tlp_sched {
     TLP_SCHED_PAPER = 3
 } tlp_sched;
 
+/* Aggregation kinds of the descriptor API (tlp_aggregate). */
+typedef enum tlp_op {
+    TLP_OP_GCN = 0,
+    TLP_OP_GIN = 1,
+    TLP_OP_GAT = 2,
+    TLP_OP_SAGE = 3,   /* GraphSage mean (NEXT-1)      */
+    TLP_OP_GAT_MH = 4  /* multi-head GAT (NEXT-1)      */
+} tlp_op;
+
+/* Layer activation of the fused epilogue (Eq. 2's sigma; NEXT-3). */
+typedef enum tlp_act {
+    TLP_ACT_NONE = 0,
+    TLP_ACT_RELU = 1,       /* max(x, 0)                         */
+    TLP_ACT_LEAKY_RELU = 2, /* x >= 0 ? x : act_param * x        */
+    TLP_ACT_ELU = 3         /* x > 0 ? x : act_param * (e^x - 1) */
+} tlp_act;
+
+/* One aggregation, fully described (tlp_aggregate / tlp_dist_aggregate).  The
+ * fields an op does not use are ignored.  After the reduction the epilogue
+ * Y = act(Y + bias) is applied per element in the same kernel (NEXT-3: the
+ * "activation" phase of the layer, fused into the store). */
+typedef struct tlp_agg_desc {
+    int op;                   /* tlp_op                                        */
+    const float *X;           /* device [n_src x ldx]                          */
+    int64_t F, ldx;
+    float *Y;                 /* device [n_dst x ldy] (dist: the full Y)       */
+    int64_t ldy;
+    int norm;                 /* GCN: tlp_norm                                 */
+    float eps;                /* GIN                                           */
+    const float *el, *er;     /* GAT: [n_src], [row_offset+n_dst]; GAT_MH: x heads */
+    float slope;              /* GAT LeakyReLU slope                           */
+    int64_t heads;            /* GAT_MH (0 or 1 = one head)                    */
+    int include_self;         /* SAGE                                          */
+    const float *bias;        /* epilogue: fp32 device [F] or NULL             */
+    int act;                  /* epilogue: tlp_act                             */
+    float act_param;          /* LeakyReLU slope / ELU alpha                   */
+} tlp_agg_desc;
+
 typedef struct tlp_graph_s *tlp_graph;
 typedef struct tlp_comm_s *tlp_comm;
 
@@ -199,6 +237,11 @@ tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F,
                              int64_t ldx, const float *el, const float *er,
                              float slope, float *Y, int64_t ldy, void *stream);
 
+/* Any aggregation from a descriptor, with the fused layer epilogue
+ * act(Y + bias).  Same errors as the specific calls, plus
+ * TLP_ERR_INVALID_ARGUMENT for an unknown op or activation. */
+tlp_status tlp_aggregate(tlp_graph g, const tlp_agg_desc *desc, void *stream);
+
 /* ---- NEXT-1: GraphSage mean, multi-head GAT ------------------ */
 
 /* GraphSage mean aggregator (Hamilton et al. [15]):
@@ -283,6 +326,9 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph local, tlp_comm c,
                                   const float *X_full, int64_t F, int64_t ldx,
                                   const float *el, const float *er, float slope,
                                   float *Y_full, int64_t ldy, void *stream);
+/* Descriptor form of the dist calls (desc->Y is Y_full). */
+tlp_status tlp_dist_aggregate(tlp_graph local, tlp_comm c,
+                              const tlp_agg_desc *desc, void *stream);
 tlp_status tlp_dist_sage_aggregate(tlp_graph local, tlp_comm c,
                                    const float *X_full, int64_t F, int64_t ldx,
                                    int include_self, float *Y_full, int64_t ldy,

@@ -51,6 +51,18 @@ class tlp_graph_info(ctypes.Structure):
         "device_bytes", "scratch_bytes")] + [("create_ms", ctypes.c_double)]
 
 
+class tlp_agg_desc(ctypes.Structure):
+    _fields_ = [("op", ctypes.c_int), ("X", ctypes.c_void_p), ("F", ctypes.c_int64),
+                ("ldx", ctypes.c_int64), ("Y", ctypes.c_void_p), ("ldy", ctypes.c_int64),
+                ("norm", ctypes.c_int), ("eps", ctypes.c_float), ("el", ctypes.c_void_p),
+                ("er", ctypes.c_void_p), ("slope", ctypes.c_float), ("heads", ctypes.c_int64),
+                ("include_self", ctypes.c_int), ("bias", ctypes.c_void_p), ("act", ctypes.c_int),
+                ("act_param", ctypes.c_float)]
+
+
+OPS = {"gcn": 0, "gin": 1, "gat": 2, "sage": 3, "gat_mh": 4}
+ACTS = {"none": 0, "relu": 1, "leaky_relu": 2, "elu": 3}
+
 _P = ctypes.c_void_p
 _I64 = ctypes.c_int64
 _I = ctypes.c_int
@@ -71,6 +83,8 @@ _sig = {
     "tlp_gin_aggregate": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
     "tlp_gat_aggregate": ([_P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
     "tlp_sage_aggregate": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
+    "tlp_aggregate": ([_P, ctypes.POINTER(tlp_agg_desc), _P], _I),
+    "tlp_dist_aggregate": ([_P, _P, ctypes.POINTER(tlp_agg_desc), _P], _I),
     "tlp_gat_mh_aggregate": ([_P, _P, _I64, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
     "tlp_graph_create_rows": ([_I64, _I64, _P, _P, _P, _I64, _I64, ctypes.POINTER(tlp_create_opts),
                                _P, ctypes.POINTER(_P)], _I),
@@ -305,6 +319,39 @@ def tlp_gat_aggregate(g, X, el, er, slope=0.2, Y=None, F=None, stream=None, n_ds
     return Y
 
 
+def _desc(op, X, Y, F, ldx, ldy, norm="both", eps=0.0, el=None, er=None, slope=0.2, heads=1,
+          include_self=False, bias=None, act="none", act_param=0.0):
+    d = tlp_agg_desc()
+    d.op = OPS[op] if isinstance(op, str) else int(op)
+    d.X, d.F, d.ldx, d.Y, d.ldy = _ptr(X), int(F), int(ldx), _ptr(Y), int(ldy)
+    d.norm = NORMS[norm] if isinstance(norm, str) else int(norm)
+    d.eps, d.slope, d.heads = float(eps), float(slope), int(heads)
+    d.el = _ptr(None if el is None else _vec_cuda(el, "el"))
+    d.er = _ptr(None if er is None else _vec_cuda(er, "er"))
+    d.include_self = int(bool(include_self))
+    d.bias = _ptr(None if bias is None else _vec_cuda(bias, "bias"))
+    d.act = ACTS[act] if isinstance(act, str) else int(act)
+    d.act_param = float(act_param)
+    return d
+
+
+def tlp_aggregate(g, op, X, Y=None, F=None, stream=None, n_dst=None, **kw):
+    """Descriptor API: op in {gcn, gin, gat, sage, gat_mh}; keyword arguments of
+    tlp_agg_desc (norm, eps, el, er, slope, heads, include_self) plus the fused
+    layer epilogue bias=[F] tensor, act in {none, relu, leaky_relu, elu}, act_param."""
+    X, F, ldx = _feat(X, F)
+    n = _n_dst(g) if n_dst is None else n_dst
+    Y, F, ldy = _out(Y, n, F, X)
+    keep = [kw.get(k) for k in ("el", "er", "bias")]  # keep contiguous copies alive
+    for k in ("el", "er", "bias"):
+        if kw.get(k) is not None:
+            kw[k] = _vec_cuda(kw[k], k)
+    d = _desc(op, X, Y, F, ldx, ldy, **kw)
+    _check(_lib.tlp_aggregate(g, ctypes.byref(d), _stream(stream, X.device)), "tlp_aggregate")
+    del keep
+    return Y
+
+
 def tlp_sage_aggregate(g, X, include_self=False, Y=None, F=None, stream=None, n_dst=None):
     """GraphSage mean over N(v) (or N(v) + v with include_self)."""
     X, F, ldx = _feat(X, F)
@@ -426,6 +473,18 @@ def tlp_dist_gat_aggregate(g, comm, X_full, Y_full, el, er, slope=0.2, F=None, s
     return Y_full
 
 
+def tlp_dist_aggregate(g, comm, op, X_full, Y_full, F=None, stream=None, **kw):
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_full, F)
+    for k in ("el", "er", "bias"):
+        if kw.get(k) is not None:
+            kw[k] = _vec_cuda(kw[k], k)
+    d = _desc(op, X, Y, F, ldx, ldy, **kw)
+    _check(_lib.tlp_dist_aggregate(g, comm, ctypes.byref(d), _stream(stream, X.device)),
+           "tlp_dist_aggregate")
+    return Y_full
+
+
 def tlp_dist_sage_aggregate(g, comm, X_full, Y_full, include_self=False, F=None, stream=None):
     X, F, ldx = _feat(X_full, F)
     Y, _, ldy = _feat(Y_full, F)
@@ -482,6 +541,9 @@ class Graph:
     def gat_mh(self, X, el, er, heads, slope=0.2, Y=None, F=None, stream=None):
         return tlp_gat_mh_aggregate(self.handle, X, el, er, heads, slope, Y, F, stream,
                                     n_dst=self.n_dst)
+
+    def aggregate(self, op, X, Y=None, F=None, stream=None, **kw):
+        return tlp_aggregate(self.handle, op, X, Y, F, stream, n_dst=self.n_dst, **kw)
 
     def degrees(self):
         return tlp_graph_degrees(self.handle)

@@ -86,6 +86,9 @@ struct AggArgs {
     int F, n_strips, norm, step, sched, panel;
     float eps1, slope;
     int sage_self;  // OP_SAGE: include X[v] in the mean
+    const float *bias;  // layer epilogue (NEXT-3): y = act(y + bias)
+    int act;
+    float act_param;
     int heads, fh;  // OP_GATH: H heads of fh columns each (F = heads * fh)
 };
 
@@ -759,6 +762,27 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
     for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
 }
 
+// Layer epilogue (NEXT-3, Eq. 2): y = act(y + bias), per element, so it never
+// changes with strip width or gather path.
+template <int VEC>
+__device__ __forceinline__ void apply_layer_epilogue(const AggArgs &a, int col, Vec<VEC> &y) {
+    if (a.bias) {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c)
+            if (col + c < a.F) y.v[c] += __ldg(a.bias + col + c);
+    }
+    if (a.act == TLP_ACT_RELU) {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) y.v[c] = y.v[c] > 0.f ? y.v[c] : 0.f;
+    } else if (a.act == TLP_ACT_LEAKY_RELU) {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) y.v[c] = y.v[c] >= 0.f ? y.v[c] : a.act_param * y.v[c];
+    } else if (a.act == TLP_ACT_ELU) {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) y.v[c] = y.v[c] > 0.f ? y.v[c] : a.act_param * expm1f(y.v[c]);
+    }
+}
+
 // Epilogue (a9) for a full row reduction.
 template <int VEC, int OP>
 __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_t deg, int col,
@@ -794,6 +818,7 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_
 #pragma unroll
         for (int c = 0; c < VEC; ++c) y.v[c] = deg > 0 ? acc.v[c] / den : 0.f;
     }
+    apply_layer_epilogue<VEC>(a, col, y);
     return y;
 }
 
@@ -849,6 +874,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
 #pragma unroll
                     for (int c = 0; c < VEC; ++c)
                         y.v[c] = (e1 > e0) ? acc.v[c] / (c < split ? dA : dB) : 0.f;
+                    apply_layer_epilogue<VEC>(a, col, y);
                     if (active) st_row<VEC>(yrow, col, a.F, y);
                     continue;
                 } else if constexpr (ASYNC) {
@@ -980,6 +1006,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         if constexpr (OP == OP_GATH) {
 #pragma unroll
             for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] / (c < split ? DA : DB);
+            apply_layer_epilogue<VEC>(a, col, y);
         } else {
             y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
         }
@@ -1120,6 +1147,10 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         return set_error(TLP_ERR_INVALID_ARGUMENT, "the self term needs row_offset + n_dst <= n_src");
     if ((r.op == OP_GAT || r.op == OP_GATH) && (!r.el || !r.er))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "GAT needs el and er");
+    if (r.act < TLP_ACT_NONE || r.act > TLP_ACT_ELU)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown activation");
+    if (r.op < OP_GCN || r.op > OP_GATH)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown op");
     if (r.op == OP_GATH && (r.heads < 1 || r.F % r.heads != 0))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "multi-head GAT needs F = heads * head_dim");
     {
@@ -1221,6 +1252,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.eps1 = 1.0f + r.eps;
     a.slope = r.slope;
     a.sage_self = r.sage_self;
+    a.bias = r.bias;
+    a.act = r.act;
+    a.act_param = r.act_param;
     a.heads = (int)r.heads;
     a.fh = fh;
     a.scratch = nullptr;
@@ -1331,6 +1365,11 @@ tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F, int64_t ldx
     r.X = X; r.F = F; r.ldx = ldx; r.Y = Y; r.ldy = ldy;
     r.el = el; r.er = er; r.slope = slope;
     return aggregate(g, r, (cudaStream_t)stream);
+}
+
+tlp_status tlp_aggregate(tlp_graph g, const tlp_agg_desc *d, void *stream) {
+    if (!d) return set_error(TLP_ERR_INVALID_ARGUMENT, "null descriptor");
+    return aggregate(g, request_from_desc(*d), (cudaStream_t)stream);
 }
 
 tlp_status tlp_sage_aggregate(tlp_graph g, const float *X, int64_t F, int64_t ldx, int include_self,

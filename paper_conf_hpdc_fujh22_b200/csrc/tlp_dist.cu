@@ -242,6 +242,12 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph g, tlp_comm c, const float *X_full, 
     return dist_local(g, c, r, stream);
 }
 
+tlp_status tlp_dist_aggregate(tlp_graph g, tlp_comm c, const tlp_agg_desc *d, void *stream) {
+    if (!d) return set_error(TLP_ERR_INVALID_ARGUMENT, "null descriptor");
+    AggRequest r = request_from_desc(*d);
+    return dist_local(g, c, r, stream);
+}
+
 tlp_status tlp_dist_sage_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t F,
                                    int64_t ldx, int include_self, float *Y_full, int64_t ldy,
                                    void *stream) {

@@ -101,7 +101,21 @@ struct AggRequest {
     float slope = 0.f;
     int sage_self = 0;  // op 3 (GraphSage mean): include the self row
     int64_t heads = 1;  // op 4 (multi-head GAT)
+    const float *bias = nullptr;  // layer epilogue: y = act(y + bias)
+    int act = 0;
+    float act_param = 0.f;
 };
+
+inline AggRequest request_from_desc(const tlp_agg_desc &d) {
+    AggRequest r;
+    r.op = d.op;
+    r.X = d.X; r.F = d.F; r.ldx = d.ldx; r.Y = d.Y; r.ldy = d.ldy;
+    r.norm = d.norm; r.eps = d.eps;
+    r.el = d.el; r.er = d.er; r.slope = d.slope; r.heads = d.heads > 0 ? d.heads : 1;
+    r.sage_self = d.include_self;
+    r.bias = d.bias; r.act = d.act; r.act_param = d.act_param;
+    return r;
+}
 tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s);
 
 }  // namespace tlp

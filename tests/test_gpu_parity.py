@@ -582,3 +582,51 @@ def test_products_gat_mh_sampled(tlp):
     Y = g.gat_mh(_t(Xh), _t(el), _t(er), H, synth.SLOPE, F=F)
     _check("products gat_mh", Y[_t(rows)], oracle.gat_mh(rp, ci, Xh, el, er, H, synth.SLOPE, rows=rows, Fh=F // H))
     g.close()
+
+
+# ------------------------------------------------------------ NEXT-3 ---------
+
+@pytest.mark.parametrize("op", ["gcn", "gin", "gat", "sage", "gat_mh"])
+@pytest.mark.parametrize("act,param", [("none", 0.0), ("relu", 0.0), ("leaky_relu", 0.1), ("elu", 1.0)])
+def test_layer_epilogue_fused(tlp, op, act, param):
+    """tlp_aggregate with the fused epilogue act(agg + bias) against the oracle's
+    aggregation followed by its plain epilogue."""
+    n = 900
+    rp, ci = synth.chung_lu(n, 20000, 0.55, 31, device="cpu")
+    F, ld, H = 130, 132, 2
+    Xh = synth.features(n, F, ld, seed=5)
+    b = synth.normal(F, 9) * 0.5
+    el = synth.normal(n * H, 10).reshape(n, H)
+    er = synth.normal(n * H, 11).reshape(n, H)
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    kw = dict(bias=_t(b), act=act, act_param=param, F=F)
+    if op == "gcn":
+        Y = g.aggregate("gcn", _t(Xh), norm="both", **kw); ref = oracle.gcn(rp, ci, Xh, "both", F=F)
+    elif op == "gin":
+        Y = g.aggregate("gin", _t(Xh), eps=0.1, **kw); ref = oracle.gin(rp, ci, Xh, 0.1, F=F)
+    elif op == "gat":
+        e1, r1 = el[:, 0].copy(), er[:, 0].copy()
+        Y = g.aggregate("gat", _t(Xh), el=_t(e1), er=_t(r1), slope=0.2, **kw)
+        ref = oracle.gat(rp, ci, Xh, e1, r1, 0.2, F=F)
+    elif op == "sage":
+        Y = g.aggregate("sage", _t(Xh), include_self=True, **kw)
+        ref = oracle.sage(rp, ci, Xh, include_self=True, F=F)
+    else:
+        Y = g.aggregate("gat_mh", _t(Xh), el=_t(el), er=_t(er), heads=H, slope=0.2, **kw)
+        ref = oracle.gat_mh(rp, ci, Xh, el, er, H, 0.2, Fh=F // H)
+    _check(f"{op}+{act}", Y, oracle.epilogue(ref[0], ref[1], b, act, param))
+    # the epilogue is per element: same bits as applying it to the plain output
+    plain = g.aggregate(op, _t(Xh), F=F,
+                        **{k: v for k, v in dict(norm="both", eps=0.1, include_self=True,
+                                                 el=_t(el if op == "gat_mh" else el[:, 0].copy()),
+                                                 er=_t(er if op == "gat_mh" else er[:, 0].copy()),
+                                                 slope=0.2, heads=H if op == "gat_mh" else 1).items()})
+    x = plain + _t(b)
+    if act == "relu":
+        x = torch.relu(x)
+    elif act == "leaky_relu":
+        x = torch.where(x >= 0, x, param * x)
+    elif act == "elu":
+        x = torch.where(x > 0, x, param * torch.expm1(x))
+    assert torch.allclose(Y, x, rtol=0, atol=1e-6)
+    g.close()
