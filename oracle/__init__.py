@@ -73,6 +73,10 @@ def _load():
         lib.oracle_gat_mh.restype = ctypes.c_int
         lib.oracle_epilogue.argtypes = [I64, I64, P, P, P, ctypes.c_int, ctypes.c_double]
         lib.oracle_epilogue.restype = ctypes.c_int
+        lib.oracle_gcn_backward.argtypes = [I64, I64, P, P, P, P, I64, I64, ctypes.c_int, P, P]
+        lib.oracle_gcn_backward.restype = ctypes.c_int
+        lib.oracle_gin_backward.argtypes = [I64, P, P, P, P, I64, I64, ctypes.c_double, P, P]
+        lib.oracle_gin_backward.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -226,6 +230,36 @@ def gat_mh(rowptr, colidx, X, el, er, heads, slope, rows=None, row_offset=0, Fh=
     if rc:
         raise ValueError("oracle_gat_mh: bad arguments")
     return Y, A
+
+
+def gcn_backward(rowptr, colidx, dY, norm="both", ew=None, n_src=None, F=None):
+    """dX = M^T dY for the GCN operator M (returns (dX, A) [n_src, F])."""
+    rowptr, colidx = _csr(rowptr, colidx)
+    dY = _feat(dY)
+    n_dst = rowptr.shape[0] - 1
+    n_src = n_dst if n_src is None else n_src
+    F = dY.shape[1] if F is None else F
+    ew = None if ew is None else np.ascontiguousarray(ew, dtype=np.float32)
+    dX = np.empty((n_src, F)); A = np.empty((n_src, F))
+    rc = _load().oracle_gcn_backward(n_dst, n_src, _ptr(rowptr), _ptr(colidx), _ptr(ew), _ptr(dY), F,
+                                     dY.strides[0] // 4, _NORMS.get(norm, norm), _ptr(dX), _ptr(A))
+    if rc:
+        raise ValueError("oracle_gcn_backward: bad arguments")
+    return dX, A
+
+
+def gin_backward(rowptr, colidx, dY, eps, ew=None, F=None):
+    rowptr, colidx = _csr(rowptr, colidx)
+    dY = _feat(dY)
+    n = rowptr.shape[0] - 1
+    F = dY.shape[1] if F is None else F
+    ew = None if ew is None else np.ascontiguousarray(ew, dtype=np.float32)
+    dX = np.empty((n, F)); A = np.empty((n, F))
+    rc = _load().oracle_gin_backward(n, _ptr(rowptr), _ptr(colidx), _ptr(ew), _ptr(dY), F,
+                                     dY.strides[0] // 4, float(eps), _ptr(dX), _ptr(A))
+    if rc:
+        raise ValueError("oracle_gin_backward: bad arguments")
+    return dX, A
 
 
 ACTS = {"none": 0, "relu": 1, "leaky_relu": 2, "elu": 3}

@@ -390,3 +390,82 @@ int oracle_epilogue(int64_t n_rows, int64_t F, double *Y, double *A,
     }
     return 0;
 }
+
+/* ---- NEXT-4: backward aggregation ----------------------------- */
+
+/* GCN backward (the training workload of Eq. 1): the forward layer
+ * is Y = M X with M[v,u] = sum over edges u->v of c_in(v) w_e c_out(u), so
+ *   dX = M^T dY,  dX[u,f] = sum_{edges e: u -> v} c_in(v) w_e c_out(u) dY[v,f].
+ * Written as the plain scatter over the forward CSR (no transposed CSR), fp64.
+ * dX and A are [n_src x F] (all source rows). */
+int oracle_gcn_backward(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+                        const int32_t *colidx, const float *ew, const float *dY,
+                        int64_t F, int64_t lddy, int norm, double *dX, double *A)
+{
+    if (norm < 0 || norm > 2 || F < 0 || lddy < F)
+        return -1;
+    int64_t nnz = rowptr[n_dst];
+    int32_t *out_deg = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n_src > 0 ? n_src : 1));
+    if (!out_deg)
+        return -1;
+    oracle_out_degree(n_src, nnz, colidx, out_deg);
+    for (int64_t i = 0; i < n_src * F; ++i) {
+        dX[i] = 0.0;
+        if (A)
+            A[i] = 0.0;
+    }
+    for (int64_t v = 0; v < n_dst; ++v) {
+        int64_t deg = rowptr[v + 1] - rowptr[v];
+        double dclamp = (double)(deg > 1 ? deg : 1);
+        double c_in = norm == ORACLE_NORM_RIGHT ? 1.0 / dclamp
+                      : norm == ORACLE_NORM_BOTH ? 1.0 / sqrt(dclamp) : 1.0;
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e) {
+            int64_t u = colidx[e];
+            double w = ew ? (double)ew[e] : 1.0;
+            double c_out = 1.0;
+            if (norm == ORACLE_NORM_BOTH) {
+                int32_t od = out_deg[u];
+                c_out = 1.0 / sqrt((double)(od > 1 ? od : 1));
+            }
+            double coef = c_in * w * c_out;
+            for (int64_t f = 0; f < F; ++f) {
+                double term = coef * (double)dY[v * lddy + f];
+                dX[u * F + f] += term;
+                if (A)
+                    A[u * F + f] += fabs(term);
+            }
+        }
+    }
+    free(out_deg);
+    return 0;
+}
+
+/* GIN backward: Y = (1+eps) X[v] + sum_e w_e X[u]  =>
+ *   dX[u,f] = (1+eps) dY[u,f] + sum_{edges e: u -> v} w_e dY[v,f]
+ * (square graph, n_dst = n_src). */
+int oracle_gin_backward(int64_t n, const int64_t *rowptr, const int32_t *colidx,
+                        const float *ew, const float *dY, int64_t F, int64_t lddy,
+                        double eps, double *dX, double *A)
+{
+    if (F < 0 || lddy < F)
+        return -1;
+    for (int64_t u = 0; u < n; ++u)
+        for (int64_t f = 0; f < F; ++f) {
+            double t = (1.0 + eps) * (double)dY[u * lddy + f];
+            dX[u * F + f] = t;
+            if (A)
+                A[u * F + f] = fabs(t);
+        }
+    for (int64_t v = 0; v < n; ++v)
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; ++e) {
+            int64_t u = colidx[e];
+            double w = ew ? (double)ew[e] : 1.0;
+            for (int64_t f = 0; f < F; ++f) {
+                double term = w * (double)dY[v * lddy + f];
+                dX[u * F + f] += term;
+                if (A)
+                    A[u * F + f] += fabs(term);
+            }
+        }
+    return 0;
+}

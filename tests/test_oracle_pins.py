@@ -486,3 +486,46 @@ def test_epilogue_matches_numpy_definitions():
     np.testing.assert_array_equal(oracle.epilogue(Y, A, b, "leaky_relu", 0.2)[0], np.where(x >= 0, x, 0.2 * x))
     np.testing.assert_allclose(oracle.epilogue(Y, A, b, "elu", 0.7)[0], np.where(x > 0, x, 0.7 * np.expm1(x)),
                                rtol=1e-14, atol=1e-16)
+
+
+# ---------------------------------------------------- NEXT-4: backward ---------
+
+@pytest.mark.parametrize("case", range(6))
+@pytest.mark.parametrize("norm", ["none", "right", "both"])
+@pytest.mark.parametrize("weighted", [False, True])
+def test_p2_brute_gcn_backward(case, norm, weighted):
+    rp, ci, n_src = _small_cases()[case]
+    n_dst = len(rp) - 1
+    dY = synth.features(n_dst, 4, 5, seed=case + 40)
+    ew = synth.edge_weights(len(ci), case + 3) if weighted else None
+    dX, _ = oracle.gcn_backward(rp, ci, dY, norm, ew=ew, n_src=n_src, F=4)
+    # dense operator M from the forward brute force, applied transposed
+    M = _brute_gcn(rp, ci, np.eye(n_src, dtype=np.float32), norm, n_src, ew)
+    np.testing.assert_allclose(dX, M.T @ dY[:, :4].astype(np.float64), rtol=1e-12, atol=1e-13)
+
+
+@pytest.mark.parametrize("norm", ["none", "right", "both"])
+def test_p4_gcn_adjoint_identity(pub, norm):
+    """<M X, G> = <X, M^T G> (exact up to fp64 rounding)."""
+    rp, ci, n = pub
+    X = synth.features(n, 3, seed=1)
+    G = synth.features(n, 3, seed=2)
+    Y, _ = oracle.gcn(rp, ci, X, norm)
+    dX, _ = oracle.gcn_backward(rp, ci, G, norm)
+    lhs = float((Y * G.astype(np.float64)).sum())
+    rhs = float((X.astype(np.float64) * dX).sum())
+    assert abs(lhs - rhs) <= 1e-9 * (abs(lhs) + 1)
+
+
+@pytest.mark.parametrize("case", [1, 2, 3, 5])
+def test_p2_brute_gin_backward(case):
+    rp, ci, n_src = _small_cases()[case]
+    n = len(rp) - 1
+    if n != n_src:
+        pytest.skip("square graphs only")
+    dY = synth.features(n, 4, 4, seed=case)
+    ew = synth.edge_weights(len(ci), 2)
+    dX, _ = oracle.gin_backward(rp, ci, dY, 0.3, ew=ew)
+    A, _ = _dense_adj(rp, ci, n, n, ew)
+    np.testing.assert_allclose(dX, 1.3 * dY.astype(np.float64) + A.T @ dY.astype(np.float64),
+                               rtol=1e-12, atol=1e-13)
