@@ -55,6 +55,8 @@ def gather_bytes(op, n_rows, n_edges, F):
         return n_edges * (4 * F + 8) + n_rows * (4 * F + 12)
     if op == "gcn2":
         return 2 * gather_bytes("gcn", n_rows, n_edges, F)
+    if op == "gcn_bwd":  # dX = M^T dY on the transposed CSR: same byte model as GCN
+        return gather_bytes("gcn", n_rows, n_edges, F)
     if op == "sage":  # mean over N(v)+v: per edge 4F + 4; per row self + Y + rowptr
         return n_edges * (4 * F + 4) + n_rows * (8 * F + 8)
     if op.startswith("gat") and op[3:].isdigit():  # H heads: el/er per head
@@ -157,14 +159,17 @@ WORKLOADS = {
     # NEXT-1 rows: GraphSage mean (+self) and 4-head GAT
     "reddit_sage": dict(graph="reddit", ops=("sage",)),
     "products_gat4": dict(graph="products", ops=("gat4",)),
+    # NEXT-4: the backward aggregation of a GCN(BOTH) layer
+    "reddit_bwd": dict(graph="reddit", ops=("gcn_bwd",)),
 }
-LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2, "sage": 1, "gat4": 1}
+LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2, "sage": 1, "gat4": 1, "gcn_bwd": 1}
 
 
 def workload_desc(name, cfg, E):
     ops = "+".join({"gcn": "GCN(both)", "gin": "GIN(eps=0.1)", "gat": "GAT(slope=0.2)",
                     "gcn2": "2-layer GCN(both)", "sage": "GraphSage-mean(+self)",
-                    "gat4": "4-head GAT(slope=0.2)"}[o] for o in WORKLOADS[name]["ops"])
+                    "gat4": "4-head GAT(slope=0.2)",
+                    "gcn_bwd": "GCN(both) backward dX = M^T dY"}[o] for o in WORKLOADS[name]["ops"])
     return f"{name}-shaped {ops}: N={cfg_n(cfg)} E={E} F={cfg['F']} ld={cfg['ld']}"
 
 
@@ -222,6 +227,8 @@ def run_tlp(args):
         g = tlp.Graph(rp_d, ci_d)
     torch.cuda.synchronize()
     create_ms = (time.perf_counter() - t0) * 1e3
+    if "gcn_bwd" in ops:
+        g.build_transpose()
     info = g.info
     del ci_d
     X = torch.from_numpy(Xh).to(dev)
@@ -242,6 +249,8 @@ def run_tlp(args):
             gcn_to(Y1, Yo[op])
         elif op == "gcn":
             gcn_to(Xin, Yo[op])
+        elif op == "gcn_bwd":
+            g.gcn_backward(Xin, "both", dX=Yo[op], F=F)
         elif use_dist:
             if op == "gin":
                 tlp.tlp_dist_gin_aggregate(g.handle, comm, Xin, Yo[op], synth.EPS, F=F)
@@ -436,7 +445,7 @@ def _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows):
     by = 0
     t0 = time.perf_counter()
     for op in WORKLOADS[name]["ops"]:
-        if op == "gcn":
+        if op in ("gcn", "gcn_bwd"):  # (bwd: the reddit graph is symmetric, same work per row)
             oracle.gcn(rp, ci, Xh, "both", rows=rows, F=F)
         elif op == "gcn2":
             # layer 2 of a row needs layer 1 at its in-neighbours: the bounded sample

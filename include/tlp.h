@@ -265,6 +265,29 @@ tlp_status tlp_gat_mh_aggregate(tlp_graph g, const float *X, int64_t heads,
                                 const float *er, float slope, float *Y,
                                 int64_t ldy, void *stream);
 
+/* ---- NEXT-4: backward aggregation ---------------------------- */
+
+/* Builds (once) the transposed out-edge CSR the backward calls run on (stable
+ * sort of the edges by source; each source's edges stay in destination order)
+ * with its own degrees and plan.  O(nnz) extra device memory; synchronises
+ * `stream`.  Not available for dist row slices (TLP_ERR_UNSUPPORTED). */
+tlp_status tlp_graph_build_transpose(tlp_graph g, void *stream);
+
+/* GCN backward (Eq. 1 training): dX = M^T dY for the forward GCN
+ * operator M of the same norm, i.e.
+ *   dX[u] = sum_{edges e: u -> v} c_in(v) w_e c_out(u) dY[v].
+ * dY: fp32 device [n_dst x lddy], dX: fp32 device [n_src x lddx].  Needs
+ * tlp_graph_build_transpose.  One kernel launch; deterministic. */
+tlp_status tlp_gcn_backward(tlp_graph g, const float *dY, int64_t F,
+                            int64_t lddy, int norm, float *dX, int64_t lddx,
+                            void *stream);
+
+/* GIN backward: dX[u] = (1+eps) dY[u] + sum_{edges e: u -> v} w_e dY[v]
+ * (square graphs). */
+tlp_status tlp_gin_backward(tlp_graph g, const float *dY, int64_t F,
+                            int64_t lddy, float eps, float *dX, int64_t lddx,
+                            void *stream);
+
 /* ---- multi-GPU (destination-row ranges balanced by edge count) ------------ */
 
 /* Pure host function: bounds[0] = 0, bounds[parts] = n, and for 0 < k < parts

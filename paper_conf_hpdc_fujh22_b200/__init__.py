@@ -79,6 +79,9 @@ _sig = {
     "tlp_graph_degrees": ([_P, _P, _P, _P], _I),
     "tlp_graph_plan": ([_P, _P, _P, _P, _P], _I),
     "tlp_graph_set_schedule": ([_P, _I, _I, _I], _I),
+    "tlp_graph_build_transpose": ([_P, _P], _I),
+    "tlp_gcn_backward": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
+    "tlp_gin_backward": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
     "tlp_gcn_aggregate": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_gin_aggregate": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
     "tlp_gat_aggregate": ([_P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
@@ -283,6 +286,10 @@ def tlp_graph_set_schedule(g, sched="dynamic", warps_per_cta=0, step=0):
            "tlp_graph_set_schedule")
 
 
+def tlp_graph_build_transpose(g, stream=None):
+    _check(_lib.tlp_graph_build_transpose(g, _stream(stream)), "tlp_graph_build_transpose")
+
+
 # ------------------------------------------------------------ aggregations ---
 
 def _n_dst(g):
@@ -373,6 +380,26 @@ def tlp_gat_mh_aggregate(g, X, el, er, heads, slope=0.2, Y=None, F=None, stream=
                                      float(slope), _ptr(Y), ldy, _stream(stream, X.device)),
            "tlp_gat_mh_aggregate")
     return Y
+
+
+def tlp_gcn_backward(g, dY, norm="both", dX=None, F=None, stream=None, n_src=None):
+    """dX = M^T dY for the GCN operator of the given norm (needs the transpose)."""
+    dY, F, lddy = _feat(dY, F)
+    n = tlp_graph_info_get(g)["n_src"] if n_src is None else n_src
+    dX, F, lddx = _out(dX, n, F, dY)
+    nm = NORMS[norm] if isinstance(norm, str) else int(norm)
+    _check(_lib.tlp_gcn_backward(g, _ptr(dY), F, lddy, nm, _ptr(dX), lddx, _stream(stream, dY.device)),
+           "tlp_gcn_backward")
+    return dX
+
+
+def tlp_gin_backward(g, dY, eps=0.0, dX=None, F=None, stream=None, n_src=None):
+    dY, F, lddy = _feat(dY, F)
+    n = tlp_graph_info_get(g)["n_src"] if n_src is None else n_src
+    dX, F, lddx = _out(dX, n, F, dY)
+    _check(_lib.tlp_gin_backward(g, _ptr(dY), F, lddy, float(eps), _ptr(dX), lddx,
+                                 _stream(stream, dY.device)), "tlp_gin_backward")
+    return dX
 
 
 # -------------------------------------------------------------- multi-GPU ----
@@ -544,6 +571,15 @@ class Graph:
 
     def aggregate(self, op, X, Y=None, F=None, stream=None, **kw):
         return tlp_aggregate(self.handle, op, X, Y, F, stream, n_dst=self.n_dst, **kw)
+
+    def build_transpose(self, stream=None):
+        tlp_graph_build_transpose(self.handle, stream)
+
+    def gcn_backward(self, dY, norm="both", dX=None, F=None, stream=None):
+        return tlp_gcn_backward(self.handle, dY, norm, dX, F, stream, n_src=self.info["n_src"])
+
+    def gin_backward(self, dY, eps=0.0, dX=None, F=None, stream=None):
+        return tlp_gin_backward(self.handle, dY, eps, dX, F, stream, n_src=self.info["n_src"])
 
     def degrees(self):
         return tlp_graph_degrees(self.handle)

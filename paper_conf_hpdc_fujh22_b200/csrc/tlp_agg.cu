@@ -1141,7 +1141,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         return set_error(TLP_ERR_INVALID_ARGUMENT, "leading dimension smaller than F");
     if (!aligned(r.X, 4) || !aligned(r.Y, 4))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "X and Y must be 4-byte aligned");
-    if (r.op == OP_GCN && (r.norm < TLP_NORM_NONE || r.norm > TLP_NORM_BOTH))
+    if (r.op == OP_GCN && (r.norm < TLP_NORM_NONE || r.norm > kNormLeft))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown norm");
     if ((r.op == OP_GIN || (r.op == OP_SAGE && r.sage_self)) && g->row_offset + g->n_dst > g->n_src)
         return set_error(TLP_ERR_INVALID_ARGUMENT, "the self term needs row_offset + n_dst <= n_src");
@@ -1174,7 +1174,15 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // kernel would form, so bitwise identical), instead of a dependent gather.
     int coef = COEF_NONE;
     const float *ew = g->ew;
-    if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) {
+    const float *cvec = g->c_out;
+    int norm = r.norm;
+    if (r.op == OP_GCN && r.norm == kNormLeft) {
+        // internal: per-source 1/max(d_out,1) gathered per edge, no row scale
+        cvec = g->c_out_left;
+        coef |= COEF_COUT;
+        if (g->ew) coef |= COEF_W;
+        norm = TLP_NORM_NONE;
+    } else if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) {
         if (g->ew_both) { ew = g->ew_both; coef |= COEF_W; }
         else { coef |= COEF_COUT; if (g->ew) coef |= COEF_W; }
     } else if (r.op != OP_GAT && g->ew) {
@@ -1226,7 +1234,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.rowptr = g->rowptr;
     a.colidx = g->colidx;
     a.ew = ew;
-    a.c_out = g->c_out;
+    a.c_out = cvec;
     a.X = r.X;
     a.Y = r.Y;
     a.el = r.el;
@@ -1248,7 +1256,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.n_strips = n_strips;
     a.panel = panel;
     a.n_items = panel ? g->n_tasks * n_strips : g->n_tasks;
-    a.norm = r.norm;
+    a.norm = norm;
     a.eps1 = 1.0f + r.eps;
     a.slope = r.slope;
     a.sage_self = r.sage_self;
@@ -1365,6 +1373,35 @@ tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F, int64_t ldx
     r.X = X; r.F = F; r.ldx = ldx; r.Y = Y; r.ldy = ldy;
     r.el = el; r.er = er; r.slope = slope;
     return aggregate(g, r, (cudaStream_t)stream);
+}
+
+// NEXT-4: backward aggregations on the transposed CSR.  dX = M^T dY:
+//   GCN BOTH  = GCN BOTH forward of the transpose (its c_out is the forward c_in,
+//               its c_in the forward c_out);  NONE = NONE;
+//   GCN RIGHT = per-source 1/max(d_out,1) of the transpose (internal LEFT norm);
+//   GIN       = GIN forward of the transpose (square graphs).
+tlp_status tlp_gcn_backward(tlp_graph g, const float *dY, int64_t F, int64_t lddy, int norm,
+                            float *dX, int64_t lddx, void *stream) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    if (!g->t) return set_error(TLP_ERR_INVALID_ARGUMENT, "call tlp_graph_build_transpose first");
+    if (norm < TLP_NORM_NONE || norm > TLP_NORM_BOTH)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown norm");
+    AggRequest r;
+    r.op = OP_GCN;
+    r.X = dY; r.F = F; r.ldx = lddy; r.Y = dX; r.ldy = lddx;
+    r.norm = (norm == TLP_NORM_RIGHT) ? kNormLeft : norm;
+    return aggregate(g->t, r, (cudaStream_t)stream);
+}
+
+tlp_status tlp_gin_backward(tlp_graph g, const float *dY, int64_t F, int64_t lddy, float eps,
+                            float *dX, int64_t lddx, void *stream) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    if (!g->t) return set_error(TLP_ERR_INVALID_ARGUMENT, "call tlp_graph_build_transpose first");
+    if (g->n_src != g->n_dst) return set_error(TLP_ERR_INVALID_ARGUMENT, "GIN backward needs a square graph");
+    AggRequest r;
+    r.op = OP_GIN;
+    r.X = dY; r.F = F; r.ldx = lddy; r.Y = dX; r.ldy = lddx; r.eps = eps;
+    return aggregate(g->t, r, (cudaStream_t)stream);
 }
 
 tlp_status tlp_aggregate(tlp_graph g, const tlp_agg_desc *d, void *stream) {

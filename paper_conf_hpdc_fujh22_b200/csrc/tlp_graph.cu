@@ -71,14 +71,49 @@ __global__ void k_out_degree(const int32_t *__restrict__ colidx, int64_t nnz,
         atomicAdd(&out_deg[colidx[e]], 1);  // integer: exact in any order
 }
 
-// c_out[u] = 1/sqrt(max(out_deg,1)) (BOTH norm, Kipf [26]; R1).
+// c_out[u] = 1/sqrt(max(out_deg,1)) (BOTH norm, Kipf [26]; R1) and
+// c_out_left[u] = 1/max(out_deg,1) (the backward of the RIGHT norm).
 __global__ void k_norm(const int32_t *__restrict__ out_deg, int64_t n,
-                       float *__restrict__ c_out) {
+                       float *__restrict__ c_out, float *__restrict__ c_out_left) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
          i += (int64_t)gridDim.x * blockDim.x) {
         int32_t d = out_deg[i];
-        c_out[i] = 1.0f / sqrtf((float)(d > 1 ? d : 1));
+        const float dc = (float)(d > 1 ? d : 1);
+        c_out[i] = 1.0f / sqrtf(dc);
+        c_out_left[i] = 1.0f / dc;
     }
+}
+
+// Destination row of every edge (transpose build).
+__global__ void k_edge_rows(const int64_t *__restrict__ rowptr, int64_t n,
+                            int32_t *__restrict__ dst) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n;
+         r += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t e = rowptr[r]; e < rowptr[r + 1]; ++e) dst[e] = (int32_t)r;
+}
+
+__global__ void k_iota(int32_t *__restrict__ v, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        v[i] = (int32_t)i;
+}
+
+__global__ void k_permute_edges(const int32_t *__restrict__ perm, int64_t nnz,
+                                const int32_t *__restrict__ dst, const float *__restrict__ ew,
+                                int32_t *__restrict__ t_col, float *__restrict__ t_ew) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz;
+         k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t e = perm[k];
+        t_col[k] = dst[e];
+        if (ew) t_ew[k] = ew[e];
+    }
+}
+
+__global__ void k_deg_to_rowptr_input(const int32_t *__restrict__ deg, int64_t n,
+                                      int64_t *__restrict__ out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = (i < n) ? (int64_t)deg[i] : 0;
 }
 
 // Per-edge GCN-BOTH coefficient c_out[colidx[e]] * w_e (a2): a coalesced
@@ -178,7 +213,9 @@ static tlp_status dmalloc(void **p, size_t bytes, tlp_graph g) {
 
 static void graph_free(tlp_graph g) {
     if (!g) return;
+    if (g->t) graph_free(g->t);
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
+                    g->c_out_left,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)
@@ -297,6 +334,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
     // ---- a2: degrees and BOTH-norm coefficients --------------------------
     TRY(dmalloc((void **)&g->out_deg, sizeof(int32_t) * n_src, g));
     TRY(dmalloc((void **)&g->c_out, sizeof(float) * n_src, g));
+    TRY(dmalloc((void **)&g->c_out_left, sizeof(float) * n_src, g));
     CTRY(cudaMemsetAsync(g->out_deg, 0, sizeof(int32_t) * n_src, s));
     {
         const int32_t *cols = full_colidx ? full_colidx : g->colidx;
@@ -306,7 +344,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
             CTRY(cudaGetLastError());
         }
         if (n_src) {
-            k_norm<<<grid_for(n_src, nsm), 256, 0, s>>>(g->out_deg, n_src, g->c_out);
+            k_norm<<<grid_for(n_src, nsm), 256, 0, s>>>(g->out_deg, n_src, g->c_out, g->c_out_left);
             CTRY(cudaGetLastError());
         }
         if (nnz) {
@@ -451,6 +489,68 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
     return TLP_OK;
 }
 
+// Transposed (out-edge) CSR for the backward aggregations (NEXT-4): stable sort
+// of the edges by source keeps each source's edges in destination order.
+tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
+    if (g->t) return TLP_OK;
+    if (g->row_offset != 0 || g->bounds_host)
+        return set_error(TLP_ERR_UNSUPPORTED, "transpose of a row slice (dist graph) is not supported");
+    const int64_t nnz = g->nnz, n_dst = g->n_dst, n_src = g->n_src;
+    if (nnz >= (int64_t(1) << 31))
+        return set_error(TLP_ERR_UNSUPPORTED, "transpose needs nnz < 2^31");
+    const int nsm = g->num_sms;
+    DevBuf dst, keys_out, iota, perm, t_col, t_ew, t_rp, deg64, temp;
+    TLP_CUDA_TRY(cudaMalloc(&dst.p, sizeof(int32_t) * nnz + 16));
+    TLP_CUDA_TRY(cudaMalloc(&keys_out.p, sizeof(int32_t) * nnz + 16));
+    TLP_CUDA_TRY(cudaMalloc(&iota.p, sizeof(int32_t) * nnz + 16));
+    TLP_CUDA_TRY(cudaMalloc(&perm.p, sizeof(int32_t) * nnz + 16));
+    TLP_CUDA_TRY(cudaMalloc(&t_col.p, sizeof(int32_t) * nnz + 16));
+    if (g->ew) TLP_CUDA_TRY(cudaMalloc(&t_ew.p, sizeof(float) * nnz + 16));
+    TLP_CUDA_TRY(cudaMalloc(&t_rp.p, sizeof(int64_t) * (n_src + 1)));
+    TLP_CUDA_TRY(cudaMalloc(&deg64.p, sizeof(int64_t) * (n_src + 1)));
+    if (n_dst) {
+        k_edge_rows<<<grid_for(n_dst, nsm), 256, 0, s>>>(g->rowptr, n_dst, dst.as<int32_t>());
+        TLP_CUDA_TRY(cudaGetLastError());
+    }
+    if (nnz) {
+        k_iota<<<grid_for(nnz, nsm), 256, 0, s>>>(iota.as<int32_t>(), nnz);
+        TLP_CUDA_TRY(cudaGetLastError());
+        size_t tb2 = 0;
+        TLP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb2, g->colidx, keys_out.as<int32_t>(),
+                                                     iota.as<int32_t>(), perm.as<int32_t>(), (int)nnz,
+                                                     0, 32, s));
+        TLP_CUDA_TRY(cudaMalloc(&temp.p, tb2));
+        TLP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(temp.p, tb2, g->colidx, keys_out.as<int32_t>(),
+                                                     iota.as<int32_t>(), perm.as<int32_t>(), (int)nnz,
+                                                     0, 32, s));
+        k_permute_edges<<<grid_for(nnz, nsm), 256, 0, s>>>(perm.as<int32_t>(), nnz, dst.as<int32_t>(),
+                                                           g->ew, t_col.as<int32_t>(), t_ew.as<float>());
+        TLP_CUDA_TRY(cudaGetLastError());
+    }
+    // transposed rowptr = exclusive scan of the out-degrees
+    k_deg_to_rowptr_input<<<grid_for(n_src + 1, nsm), 256, 0, s>>>(g->out_deg, n_src, deg64.as<int64_t>());
+    TLP_CUDA_TRY(cudaGetLastError());
+    {
+        DevBuf t3;
+        size_t b3 = 0;
+        TLP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, b3, deg64.as<int64_t>(), t_rp.as<int64_t>(),
+                                                   (int)(n_src + 1), s));
+        TLP_CUDA_TRY(cudaMalloc(&t3.p, b3));
+        TLP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(t3.p, b3, deg64.as<int64_t>(), t_rp.as<int64_t>(),
+                                                   (int)(n_src + 1), s));
+    }
+    tlp_create_opts o{g->H, g->C, 0};
+    tlp_graph t = nullptr;
+    tlp_status st = graph_create_impl(n_src, n_dst, nnz, t_rp.as<int64_t>(), t_col.as<int32_t>(),
+                                      g->ew ? t_ew.as<float>() : nullptr, nullptr, 0, 0, &o, s, &t);
+    if (st != TLP_OK) return st;
+    t->sched = g->sched;
+    t->warps_per_cta = g->warps_per_cta;
+    g->t = t;
+    g->device_bytes += t->device_bytes;
+    return TLP_OK;
+}
+
 tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s) {
     if (bytes <= g->scratch_bytes) return TLP_OK;
     if (g->scratch) {
@@ -568,6 +668,11 @@ tlp_status tlp_graph_plan(tlp_graph g, int32_t *tasks, int32_t *hub_rows, int32_
     return TLP_OK;
 }
 
+tlp_status tlp_graph_build_transpose(tlp_graph g, void *stream) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    return build_transpose(g, (cudaStream_t)stream);
+}
+
 tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta, int step) {
     if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
     if (sched < TLP_SCHED_DYNAMIC || sched > TLP_SCHED_PAPER)
@@ -577,6 +682,7 @@ tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta, int
     g->sched = sched;
     g->warps_per_cta = warps_per_cta ? warps_per_cta : 8;
     g->step = step;
+    if (g->t) tlp_graph_set_schedule(g->t, sched, warps_per_cta, step);
     return TLP_OK;
 }
 

@@ -16,6 +16,7 @@ namespace tlp {
 constexpr int64_t kDefaultHubThreshold = 1024;  // H
 constexpr int64_t kDefaultHubChunk = 512;       // C
 constexpr int64_t kDefaultUnitEdges = 64;       // K
+constexpr int kNormLeft = 3;  // internal: per-source 1/max(d_out(u),1), no row scale
 
 // Thread-local error detail; returns `s` for chaining.
 tlp_status set_error(tlp_status s, const std::string &msg);
@@ -44,6 +45,8 @@ struct tlp_graph_s {
     int32_t *out_deg = nullptr;  // [n_src] (global for a dist slice)
     float *c_out = nullptr;      // [n_src] 1/sqrt(max(out_deg,1))
     float *ew_both = nullptr;    // [nnz] c_out[colidx[e]] * w_e (GCN BOTH coefficient)
+    float *c_out_left = nullptr; // [n_src] 1/max(out_deg,1) (internal LEFT norm, backward of RIGHT)
+    tlp_graph_s *t = nullptr;    // transposed graph (tlp_graph_build_transpose), owned
 
     int2 *tasks = nullptr;       // [n_tasks]
     int32_t *hub_row = nullptr;  // [n_hubs]
@@ -86,6 +89,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
                              tlp_graph *out);
 
 tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s);
+tlp_status build_transpose(tlp_graph g, cudaStream_t s);
 
 // Enqueue one aggregation kernel; op: 0 GCN, 1 GIN, 2 GAT, 3 GraphSage mean,
 // 4 multi-head GAT.

@@ -630,3 +630,78 @@ def test_layer_epilogue_fused(tlp, op, act, param):
         x = torch.where(x > 0, x, param * torch.expm1(x))
     assert torch.allclose(Y, x, rtol=0, atol=1e-6)
     g.close()
+
+
+# ------------------------------------------------------------ NEXT-4 ---------
+
+@pytest.mark.parametrize("name", ["random64", "powerlaw_hubs", "selfloops_multi", "star_hub",
+                                  "rect_more_src", "rect_more_dst", "e0_n5", "isolated_last"])
+@pytest.mark.parametrize("norm", ["none", "right", "both"])
+@pytest.mark.parametrize("weighted", [False, True])
+def test_gcn_backward_parity(tlp, name, norm, weighted):
+    rp, ci, n_src = _edge_graphs()[name]
+    n_dst = len(rp) - 1
+    F, ld = 37, 40
+    dYh = synth.features(n_dst, F, ld, seed=3)
+    ew = synth.edge_weights(len(ci), 5) if (weighted and len(ci)) else None
+    g = tlp.Graph(_t(rp), _t(ci), n_src=n_src, edge_weight=None if ew is None else _t(ew),
+                  opts=dict(hub_threshold=64, hub_chunk=32))
+    g.build_transpose()
+    dX = torch.full((n_src, ld), float("nan"), device=DEV)
+    g.gcn_backward(_t(dYh), norm, dX=dX, F=F)
+    _check(f"gcn bwd {norm}", dX[:, :F], oracle.gcn_backward(rp, ci, dYh, norm, ew=ew, n_src=n_src, F=F))
+    assert torch.isnan(dX[:, F:]).all()
+    g.close()
+
+
+@pytest.mark.parametrize("name", ["random64", "powerlaw_hubs", "selfloops_multi", "star_hub"])
+def test_gin_backward_parity(tlp, name):
+    rp, ci, n = _edge_graphs()[name]
+    F = 70
+    dYh = synth.features(n, F, F, seed=4)
+    ew = synth.edge_weights(len(ci), 6)
+    g = tlp.Graph(_t(rp), _t(ci), edge_weight=_t(ew), opts=dict(hub_threshold=64, hub_chunk=32))
+    g.build_transpose()
+    _check("gin bwd", g.gin_backward(_t(dYh), 0.1), oracle.gin_backward(rp, ci, dYh, 0.1, ew=ew))
+    g.close()
+
+
+def test_backward_pubmed_all_rows_and_reddit_adjoint(tlp, reddit):
+    rp, ci = synth.dataset_graph("pubmed")
+    n = synth.CONFIGS["pubmed"]["n"]
+    dYh = synth.features(n, 500, 500, seed=6)
+    g = tlp.Graph(_t(rp), _t(ci))
+    g.build_transpose()
+    for norm in ("both", "right"):
+        _check("pubmed gcn bwd", g.gcn_backward(_t(dYh), norm), oracle.gcn_backward(rp, ci, dYh, norm))
+    g.close()
+    # full Reddit: <M X, G> == <X, M^T G> with both sides from the GPU (fp64 dot)
+    rp, ci = reddit
+    cfg = synth.CONFIGS["reddit"]
+    n, F = cfg["n"], 64
+    X = _t(synth.features(n, F, F, seed=1))
+    G = _t(synth.features(n, F, F, seed=2))
+    g = tlp.Graph(_t(rp), _t(ci))
+    g.build_transpose()
+    for norm in ("none", "right", "both"):
+        lhs = (g.gcn(X, norm).double() * G.double()).sum().item()
+        rhs = (X.double() * g.gcn_backward(G, norm).double()).sum().item()
+        assert abs(lhs - rhs) <= 1e-5 * (abs(lhs) + abs(rhs)) + 1e-3, (norm, lhs, rhs)
+    g.close()
+
+
+def test_backward_deterministic_and_transpose_once(tlp):
+    rp, ci = synth.chung_lu(3000, 60000, 0.5, 41, device="cpu")
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=100, hub_chunk=40))
+    g.build_transpose()
+    g.build_transpose()  # idempotent
+    G = _t(synth.features(3000, 130, 132, seed=3))
+    a = g.gcn_backward(G, "both", F=130).clone()
+    for sched in ("static", "hardware", "dynamic"):
+        g.set_schedule(sched)
+        assert torch.equal(g.gcn_backward(G, "both", F=130), a)
+    g.close()
+    g2 = tlp.Graph(_t(rp), _t(ci))
+    with pytest.raises(tlp.TlpError):
+        g2.gcn_backward(G, "both", F=130)  # transpose not built
+    g2.close()
