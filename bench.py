@@ -234,11 +234,23 @@ def run_tlp(args):
     X = torch.from_numpy(Xh).to(dev)
     el = torch.from_numpy(elh).to(dev)
     er = torch.from_numpy(erh).to(dev)
-    Y = {op: torch.empty((n, ld), dtype=torch.float32, device=dev) for op in ops}
-    Y1 = torch.empty((n, ld), dtype=torch.float32, device=dev) if "gcn2" in ops else None
+    sym_ptrs = []
+    fused = use_dist and args.fused
+
+    def out_buffer():
+        if fused:  # NEXT-2: NVLink-mapped symmetric Y_full written by the kernel itself
+            t_, p_ = tlp.tlp_comm_alloc_symmetric(comm, n, ld)
+            sym_ptrs.append(p_)
+            return t_
+        return torch.empty((n, ld), dtype=torch.float32, device=dev)
+
+    Y = {op: out_buffer() for op in ops}
+    Y1 = out_buffer() if "gcn2" in ops else None
 
     def gcn_to(Xin, out):
-        if use_dist:
+        if fused:
+            tlp.tlp_dist_aggregate_fused(g.handle, comm, "gcn", Xin, out, F=F, norm="both")
+        elif use_dist:
             tlp.tlp_dist_gcn_aggregate(g.handle, comm, Xin, out, "both", F=F)
         else:
             g.gcn(Xin, "both", Y=out, F=F)
@@ -251,6 +263,12 @@ def run_tlp(args):
             gcn_to(Xin, Yo[op])
         elif op == "gcn_bwd":
             g.gcn_backward(Xin, "both", dX=Yo[op], F=F)
+        elif fused:
+            kw = dict(eps=synth.EPS, slope=synth.SLOPE, include_self=True)
+            if op.startswith("gat"):
+                kw.update(el=elv, er=erv, heads=int(op[3:]) if op[3:].isdigit() else 1)
+            tlp.tlp_dist_aggregate_fused(g.handle, comm, "gat_mh" if op[3:].isdigit() else op,
+                                         Xin, Yo[op], F=F, **kw)
         elif use_dist:
             if op == "gin":
                 tlp.tlp_dist_gin_aggregate(g.handle, comm, Xin, Yo[op], synth.EPS, F=F)
@@ -321,7 +339,7 @@ def run_tlp(args):
         # each Y is read back on a second copy stream while the next op runs.
         Xd = [X, torch.empty_like(X)]
         eld, erd = [el, torch.empty_like(el)], [er, torch.empty_like(er)]
-        Yd = [Y, {op: torch.empty_like(Y[op]) for op in ops}]
+        Yd = [Y, {op: out_buffer() for op in ops}]
         s_h2d, s_d2h = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
         comp_done, d2h_done = [None, None], [{}, {}]
         if use_dist:
@@ -415,7 +433,9 @@ def run_tlp(args):
                              else "Chung-Lu G1 (SURVEY 8(d) d1), seed %d") % cfg["seed"],
                    "l2": "inputs larger than L2 (X = %.0f MB, colidx = %.0f MB vs 126 MB L2); no flush"
                          % (n * ld * 4 / 1e6, E * 4 / 1e6),
-                   "parallelism": ("rows%d (edge-balanced row ranges, X replicated, grouped-broadcast all-gather of Y)" % world) if use_dist else "single",
+                   "parallelism": ("rows%d (edge-balanced row ranges, X replicated, %s)" % (
+                       world, "fused peer-store all-gather (NEXT-2)" if fused else
+                       "grouped-broadcast all-gather of Y")) if use_dist else "single",
                    "frac_of_8TBs": round(value / NOMINAL_HBM_GBS, 4)},
         "ops": per_op, "create_ms": round(create_ms, 1),
         "plan": {k: info[k] for k in ("n_hubs", "n_hub_chunks", "n_units", "n_tasks",
@@ -428,6 +448,9 @@ def run_tlp(args):
     if rank == 0 and not args.no_cpu_baseline and world == 1:
         result["cpu_baseline"] = cpu_baseline(name, cfg, rp, ci, Xh, elh, erh, args.cpu_seconds)
     g.close()
+    torch.cuda.synchronize()
+    for p_ in sym_ptrs:
+        tlp.tlp_comm_free_symmetric(comm, p_)
     if comm is not None:
         tlp.tlp_comm_destroy(comm)
     if use_dist:
@@ -528,6 +551,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--fused", action="store_true",
+                    help="with --dist/torchrun: NEXT-2 fused compute + all-gather over NVLink peer memory")
     ap.add_argument("--dist", action="store_true",
                     help="use the NCCL dist API even at world size 1 (exercises the N>1 path)")
     args = ap.parse_args()

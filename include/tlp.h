@@ -324,6 +324,13 @@ tlp_status tlp_dist_graph_create(tlp_comm c, int64_t n, int64_t nnz,
                                  const tlp_create_opts *opts, void *stream,
                                  tlp_graph *out_local);
 
+/* NEXT-2: symmetric output buffers.  Collective over the communicator: every
+ * rank allocates `bytes` of device memory and maps every other rank's buffer
+ * through CUDA IPC (NVLink peer memory).  *local = this rank's buffer. */
+tlp_status tlp_comm_alloc_symmetric(tlp_comm c, size_t bytes, void **local);
+/* Collective: unmaps, barriers, frees. */
+tlp_status tlp_comm_free_symmetric(tlp_comm c, void *local);
+
 /* Copies the partition bounds (int64 [world+1], host). */
 tlp_status tlp_dist_bounds(tlp_graph local, int64_t *bounds_host);
 
@@ -349,6 +356,21 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph local, tlp_comm c,
                                   const float *X_full, int64_t F, int64_t ldx,
                                   const float *el, const float *er, float slope,
                                   float *Y_full, int64_t ldy, void *stream);
+/* NEXT-2 fused compute + all-gather: desc->Y must be a symmetric buffer
+ * (tlp_comm_alloc_symmetric) holding Y_full [n x ldy].  ONE kernel computes this
+ * rank's rows and stores each finished row vector into Y_full on every rank
+ * over NVLink, overlapping the exchange with the gather; a one-element NCCL
+ * all-reduce then orders `stream` after every rank's kernel.  Same result,
+ * bit for bit, as tlp_dist_aggregate. */
+tlp_status tlp_dist_aggregate_fused(tlp_graph local, tlp_comm c,
+                                    const tlp_agg_desc *desc, void *stream);
+
+/* Test hook of the multi-destination epilogue (single GPU): the aggregation
+ * stores every output row into each of the n device buffers listed in
+ * dests_host (host array), at the row's global index.  Synchronous. */
+tlp_status tlp_debug_multi_store(tlp_graph g, const tlp_agg_desc *desc,
+                                 float *const *dests_host, int n, void *stream);
+
 /* Descriptor form of the dist calls (desc->Y is Y_full). */
 tlp_status tlp_dist_aggregate(tlp_graph local, tlp_comm c,
                               const tlp_agg_desc *desc, void *stream);

@@ -98,6 +98,10 @@ _sig = {
     "tlp_dist_graph_create": ([_P, _I64, _I64, _P, _P, _P, ctypes.POINTER(tlp_create_opts), _P,
                                ctypes.POINTER(_P)], _I),
     "tlp_dist_bounds": ([_P, _P], _I),
+    "tlp_comm_alloc_symmetric": ([_P, ctypes.c_size_t, ctypes.POINTER(_P)], _I),
+    "tlp_comm_free_symmetric": ([_P, _P], _I),
+    "tlp_dist_aggregate_fused": ([_P, _P, ctypes.POINTER(tlp_agg_desc), _P], _I),
+    "tlp_debug_multi_store": ([_P, ctypes.POINTER(tlp_agg_desc), _P, _I, _P], _I),
     "tlp_dist_allgather_rows": ([_P, _P, _P, _I64, _P], _I),
     "tlp_dist_gcn_aggregate": ([_P, _P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_dist_gin_aggregate": ([_P, _P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
@@ -498,6 +502,57 @@ def tlp_dist_gat_aggregate(g, comm, X_full, Y_full, el, er, slope=0.2, F=None, s
                                        _ptr(Y), ldy, _stream(stream, X.device)),
            "tlp_dist_gat_aggregate")
     return Y_full
+
+
+class _CudaArray:
+    """Zero-copy torch view of library-owned device memory (CUDA array interface)."""
+
+    def __init__(self, ptr, shape):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": "<f4",
+                                         "data": (int(ptr), False), "version": 3, "strides": None}
+
+
+def tlp_comm_alloc_symmetric(comm, rows, ld):
+    """Collective: a [rows x ld] fp32 buffer on every rank, peer-mapped over NVLink.
+    Returns (tensor view, raw pointer); free with tlp_comm_free_symmetric."""
+    torch = _torch()
+    out = _P()
+    _check(_lib.tlp_comm_alloc_symmetric(comm, int(rows) * int(ld) * 4, ctypes.byref(out)),
+           "tlp_comm_alloc_symmetric")
+    t = torch.as_tensor(_CudaArray(out.value, (int(rows), int(ld))), device="cuda")
+    return t, out.value
+
+
+def tlp_comm_free_symmetric(comm, ptr):
+    _check(_lib.tlp_comm_free_symmetric(comm, ptr), "tlp_comm_free_symmetric")
+
+
+def tlp_dist_aggregate_fused(g, comm, op, X_full, Y_sym, F=None, stream=None, **kw):
+    """NEXT-2: one kernel computes this rank's rows and stores them into Y_full on
+    every rank (Y_sym from tlp_comm_alloc_symmetric)."""
+    X, F, ldx = _feat(X_full, F)
+    Y, _, ldy = _feat(Y_sym, F)
+    for k in ("el", "er", "bias"):
+        if kw.get(k) is not None:
+            kw[k] = _vec_cuda(kw[k], k)
+    d = _desc(op, X, Y, F, ldx, ldy, **kw)
+    _check(_lib.tlp_dist_aggregate_fused(g, comm, ctypes.byref(d), _stream(stream, X.device)),
+           "tlp_dist_aggregate_fused")
+    return Y_sym
+
+
+def tlp_debug_multi_store(g, op, X, dests, F=None, stream=None, **kw):
+    """Test hook: store the aggregation's output rows into every tensor of `dests`."""
+    X, F, ldx = _feat(X, F)
+    D0, _, ldy = _feat(dests[0], F)
+    for k in ("el", "er", "bias"):
+        if kw.get(k) is not None:
+            kw[k] = _vec_cuda(kw[k], k)
+    d = _desc(op, X, D0, F, ldx, ldy, **kw)
+    arr = (ctypes.c_void_p * len(dests))(*[t.data_ptr() for t in dests])
+    _check(_lib.tlp_debug_multi_store(g, ctypes.byref(d), arr, len(dests), _stream(stream, X.device)),
+           "tlp_debug_multi_store")
+    return dests
 
 
 def tlp_dist_aggregate(g, comm, op, X_full, Y_full, F=None, stream=None, **kw):

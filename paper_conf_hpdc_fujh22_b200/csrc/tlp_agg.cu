@@ -90,6 +90,11 @@ struct AggArgs {
     int act;
     float act_param;
     int heads, fh;  // OP_GATH: H heads of fh columns each (F = heads * fh)
+    // NEXT-2 fused all-gather: when n_dests > 0 every output row is stored to
+    // dests[i] + (row_offset + r) * ldy for each destination (the Y_full of every
+    // rank, mapped over NVLink) instead of to Y.
+    float *const *dests;
+    int n_dests;
 };
 
 template <int VEC>
@@ -822,6 +827,18 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_
     return y;
 }
 
+// Store a finished output vector of local row r: to Y, or (fused all-gather)
+// to the same global row of every destination buffer.
+template <int VEC>
+__device__ __forceinline__ void store_out(const AggArgs &a, int64_t r, int col, const Vec<VEC> &y) {
+    if (a.n_dests == 0) {
+        st_row<VEC>(a.Y + r * a.ldy, col, a.F, y);
+    } else {
+        const int64_t off = (a.row_offset + r) * a.ldy;
+        for (int i = 0; i < a.n_dests; ++i) st_row<VEC>(a.dests[i] + off, col, a.F, y);
+    }
+}
+
 // Column of this lane's 4-float vector in strip s (PAIR: 64-column strips,
 // lanes l and l+16 share a column), and whether this lane stores it.
 template <int VEC, bool PAIR>
@@ -851,7 +868,6 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
             const int64_t e1 = __shfl_sync(FULL, rp, k + 1);
             const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
             const int64_t r = rb + k;
-            float *yrow = a.Y + r * a.ldy;
             for (int s = s0; s < s1; ++s) {
                 const int col = strip_col<VEC, PAIR>(s, lane);
                 const bool active = col < a.F;
@@ -875,7 +891,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                     for (int c = 0; c < VEC; ++c)
                         y.v[c] = (e1 > e0) ? acc.v[c] / (c < split ? dA : dB) : 0.f;
                     apply_layer_epilogue<VEC>(a, col, y);
-                    if (active) st_row<VEC>(yrow, col, a.F, y);
+                    if (active) store_out<VEC>(a, r, col, y);
                     continue;
                 } else if constexpr (ASYNC) {
                     reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
@@ -883,7 +899,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                     reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den);
                 }
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
-                if (active && stores<PAIR>(lane)) st_row<VEC>(yrow, col, a.F, y);
+                if (active && stores<PAIR>(lane)) store_out<VEC>(a, r, col, y);
             }
         }
     }
@@ -948,7 +964,6 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     last = __shfl_sync(FULL, last, 0);
     if (!last) return;
     __threadfence();
-    float *yrow = a.Y + (int64_t)r * a.ldy;
     float M = -INFINITY, D = 0.f;
     if constexpr (OP == OP_GAT) {
         for (int q = 0; q < nch; ++q) M = fmaxf(M, __ldcg(md + 2 * (int64_t)(off + q)));
@@ -1010,7 +1025,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         } else {
             y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
         }
-        if (active && stores<PAIR>(lane)) st_row<VEC>(yrow, col, a.F, y);
+        if (active && stores<PAIR>(lane)) store_out<VEC>(a, r, col, y);
     }
     if (lane == 0) *ticket = 0;  // self-reset for the next launch
 }
@@ -1038,6 +1053,7 @@ __global__ void __launch_bounds__(TLP_MAXT, ASYNC ? TLP_MINB_ASYNC : TLP_MINB) k
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (a.sched == S_HARDWARE) {  // one warp per item
         if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC, PAIR>(a, wid, lane);
+        if (a.n_dests > 0) __threadfence_system();
         return;
     }
     const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -1051,6 +1067,7 @@ __global__ void __launch_bounds__(TLP_MAXT, ASYNC ? TLP_MINB_ASYNC : TLP_MINB) k
         if (a.sched == S_DYNAMIC) t = stride + (int64_t)__shfl_sync(FULL, v, 0);
         else t += stride;
     }
+    if (a.n_dests > 0) __threadfence_system();  // peer stores visible before the barrier
     if (a.sched == S_DYNAMIC && lane == 0) {
         // last warp out resets the counter: no memset launch between calls
         __threadfence();
@@ -1261,6 +1278,8 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.slope = r.slope;
     a.sage_self = r.sage_self;
     a.bias = r.bias;
+    a.dests = r.dests;
+    a.n_dests = r.n_dests;
     a.act = r.act;
     a.act_param = r.act_param;
     a.heads = (int)r.heads;

@@ -16,9 +16,21 @@
 
 #include "tlp_internal.h"
 
+// A symmetric output buffer (NEXT-2): allocated on every rank, each rank's
+// allocation mapped into every other rank's address space (CUDA IPC over
+// NVLink); dev_ptrs[r] = rank r's buffer as seen from this rank.
+struct SymBuf {
+    void *local = nullptr;
+    size_t bytes = 0;
+    std::vector<void *> peers;  // [world], peers[rank] = local
+    float **dev_ptrs = nullptr; // device copy of peers
+};
+
 struct tlp_comm_s {
     ncclComm_t comm = nullptr;
     int world = 1, rank = 0;
+    std::vector<SymBuf> sym;
+    int *barrier = nullptr;     // one device int for the stream barrier
 };
 
 namespace tlp {
@@ -95,6 +107,8 @@ tlp_status tlp_comm_create(const uint8_t id[128], int world, int rank, tlp_comm 
 
 tlp_status tlp_comm_destroy(tlp_comm c) {
     if (!c) return TLP_OK;
+    while (!c->sym.empty()) tlp_comm_free_symmetric(c, c->sym.back().local);
+    if (c->barrier) cudaFree(c->barrier);
     ncclResult_t r = ncclCommDestroy(c->comm);
     delete c;
     if (r != ncclSuccess) return nccl_error(r, "ncclCommDestroy");
@@ -148,6 +162,74 @@ tlp_status tlp_graph_create_rows(int64_t n, int64_t nnz, const int64_t *rowptr,
         cudaFree(staged);
     }
     return st;
+}
+
+static tlp_status comm_barrier(tlp_comm c, cudaStream_t s) {
+    if (c->world == 1) return TLP_OK;
+    if (!c->barrier) {
+        TLP_CUDA_TRY(cudaMalloc(&c->barrier, sizeof(int)));
+        TLP_CUDA_TRY(cudaMemset(c->barrier, 0, sizeof(int)));
+    }
+    TLP_NCCL_TRY(ncclAllReduce(c->barrier, c->barrier, 1, ncclInt, ncclSum, c->comm, s));
+    return TLP_OK;
+}
+
+tlp_status tlp_comm_alloc_symmetric(tlp_comm c, size_t bytes, void **local) {
+    if (!c || !local || bytes == 0) return set_error(TLP_ERR_INVALID_ARGUMENT, "alloc_symmetric: bad argument");
+    *local = nullptr;
+    SymBuf b;
+    b.bytes = bytes;
+    TLP_CUDA_TRY(cudaMalloc(&b.local, bytes));
+    b.peers.assign(c->world, nullptr);
+    b.peers[c->rank] = b.local;
+    if (c->world > 1) {
+        // exchange the IPC handles through NCCL (64 bytes per rank)
+        cudaIpcMemHandle_t h;
+        cudaError_t e = cudaIpcGetMemHandle(&h, b.local);
+        if (e != cudaSuccess) { cudaFree(b.local); return cuda_error(e, "cudaIpcGetMemHandle"); }
+        std::vector<cudaIpcMemHandle_t> all(c->world);
+        void *dh = nullptr;
+        TLP_CUDA_TRY(cudaMalloc(&dh, sizeof(cudaIpcMemHandle_t) * c->world));
+        TLP_CUDA_TRY(cudaMemcpy((char *)dh + sizeof(h) * c->rank, &h, sizeof(h), cudaMemcpyHostToDevice));
+        ncclResult_t r = ncclAllGather((char *)dh + sizeof(h) * c->rank, dh, sizeof(h), ncclUint8, c->comm, 0);
+        if (r != ncclSuccess) { cudaFree(dh); cudaFree(b.local); return nccl_error(r, "ncclAllGather(ipc handles)"); }
+        TLP_CUDA_TRY(cudaStreamSynchronize(0));
+        TLP_CUDA_TRY(cudaMemcpy(all.data(), dh, sizeof(h) * c->world, cudaMemcpyDeviceToHost));
+        cudaFree(dh);
+        for (int q = 0; q < c->world; ++q) {
+            if (q == c->rank) continue;
+            e = cudaIpcOpenMemHandle(&b.peers[q], all[q], cudaIpcMemLazyEnablePeerAccess);
+            if (e != cudaSuccess) {
+                for (int k = 0; k < q; ++k)
+                    if (k != c->rank && b.peers[k]) cudaIpcCloseMemHandle(b.peers[k]);
+                cudaFree(b.local);
+                return cuda_error(e, "cudaIpcOpenMemHandle");
+            }
+        }
+    }
+    TLP_CUDA_TRY(cudaMalloc(&b.dev_ptrs, sizeof(float *) * c->world));
+    TLP_CUDA_TRY(cudaMemcpy(b.dev_ptrs, b.peers.data(), sizeof(void *) * c->world, cudaMemcpyHostToDevice));
+    c->sym.push_back(b);
+    *local = b.local;
+    return TLP_OK;
+}
+
+tlp_status tlp_comm_free_symmetric(tlp_comm c, void *local) {
+    if (!c || !local) return set_error(TLP_ERR_INVALID_ARGUMENT, "free_symmetric: bad argument");
+    for (size_t i = 0; i < c->sym.size(); ++i) {
+        SymBuf &b = c->sym[i];
+        if (b.local != local) continue;
+        for (int q = 0; q < c->world; ++q)
+            if (q != c->rank && b.peers[q]) cudaIpcCloseMemHandle(b.peers[q]);
+        // every rank has unmapped before anyone frees
+        tlp_status st = comm_barrier(c, 0);
+        cudaStreamSynchronize(0);
+        cudaFree(b.dev_ptrs);
+        cudaFree(b.local);
+        c->sym.erase(c->sym.begin() + i);
+        return st;
+    }
+    return set_error(TLP_ERR_INVALID_ARGUMENT, "not a symmetric buffer of this communicator");
 }
 
 tlp_status tlp_dist_graph_create(tlp_comm c, int64_t n, int64_t nnz, const int64_t *rowptr,
@@ -246,6 +328,47 @@ tlp_status tlp_dist_aggregate(tlp_graph g, tlp_comm c, const tlp_agg_desc *d, vo
     if (!d) return set_error(TLP_ERR_INVALID_ARGUMENT, "null descriptor");
     AggRequest r = request_from_desc(*d);
     return dist_local(g, c, r, stream);
+}
+
+// NEXT-2: one kernel computes this rank's rows and stores every finished row
+// vector straight into Y_full on every rank over NVLink (peer-mapped symmetric
+// buffer), so the all-gather overlaps the gather tile by tile; a one-element
+// NCCL all-reduce then orders the stream after every rank's kernel.
+tlp_status tlp_dist_aggregate_fused(tlp_graph g, tlp_comm c, const tlp_agg_desc *d, void *stream) {
+    if (!g || !c || !d || !g->bounds_host) return set_error(TLP_ERR_INVALID_ARGUMENT, "not a dist graph");
+    if (c->world != g->world || c->rank != g->rank)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "communicator does not match the graph");
+    const SymBuf *b = nullptr;
+    for (const SymBuf &x : c->sym)
+        if (x.local == (void *)d->Y) b = &x;
+    if (!b) return set_error(TLP_ERR_INVALID_ARGUMENT, "Y_full must come from tlp_comm_alloc_symmetric");
+    if ((size_t)(g->n_global * d->ldy) * sizeof(float) > b->bytes)
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "symmetric buffer smaller than n x ldy floats");
+    AggRequest r = request_from_desc(*d);
+    r.Y = d->Y + g->row_offset * d->ldy;
+    r.dests = b->dev_ptrs;
+    r.n_dests = c->world;
+    tlp_status st = aggregate(g, r, (cudaStream_t)stream);
+    if (st != TLP_OK) return st;
+    return comm_barrier(c, (cudaStream_t)stream);
+}
+
+// Test hook for the multi-destination epilogue on one GPU: the aggregation of
+// `g` stores every output row to each of the n host-listed device buffers.
+tlp_status tlp_debug_multi_store(tlp_graph g, const tlp_agg_desc *d, float *const *dests_host, int n,
+                                 void *stream) {
+    if (!g || !d || !dests_host || n < 1) return set_error(TLP_ERR_INVALID_ARGUMENT, "bad argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    float **dd = nullptr;
+    TLP_CUDA_TRY(cudaMallocAsync((void **)&dd, sizeof(float *) * n, s));
+    TLP_CUDA_TRY(cudaMemcpyAsync(dd, dests_host, sizeof(float *) * n, cudaMemcpyHostToDevice, s));
+    AggRequest r = request_from_desc(*d);
+    r.dests = dd;
+    r.n_dests = n;
+    tlp_status st = aggregate(g, r, s);
+    cudaFreeAsync(dd, s);
+    TLP_CUDA_TRY(cudaStreamSynchronize(s));  // dests_host may be freed on return
+    return st;
 }
 
 tlp_status tlp_dist_sage_aggregate(tlp_graph g, tlp_comm c, const float *X_full, int64_t F,

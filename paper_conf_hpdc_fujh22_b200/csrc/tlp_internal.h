@@ -108,6 +108,8 @@ struct AggRequest {
     const float *bias = nullptr;  // layer epilogue: y = act(y + bias)
     int act = 0;
     float act_param = 0.f;
+    float *const *dests = nullptr;  // fused all-gather destinations (device array)
+    int n_dests = 0;
 };
 
 inline AggRequest request_from_desc(const tlp_agg_desc &d) {

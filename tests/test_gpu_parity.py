@@ -705,3 +705,45 @@ def test_backward_deterministic_and_transpose_once(tlp):
     with pytest.raises(tlp.TlpError):
         g2.gcn_backward(G, "both", F=130)  # transpose not built
     g2.close()
+
+
+# ------------------------------------------------------------ NEXT-2 ---------
+
+@pytest.mark.parametrize("op", ["gcn", "gin", "gat", "gat_mh"])
+def test_multi_destination_epilogue(tlp, op):
+    """The fused all-gather epilogue stores each finished row to every destination
+    (here: three local buffers), bitwise equal to the plain call, pads untouched."""
+    n = 2500
+    rp, ci = synth.chung_lu(n, 60000, 0.5, 51, device="cpu")
+    F, ld = 130, 132
+    X = _t(synth.features(n, F, ld, seed=5))
+    el, er = _t(synth.normal(n * 2, 1).reshape(n, 2)), _t(synth.normal(n * 2, 2).reshape(n, 2))
+    kw = dict(norm="both", eps=0.1, slope=0.2, heads=2 if op == "gat_mh" else 1,
+              el=el if op == "gat_mh" else el[:, 0].contiguous(),
+              er=er if op == "gat_mh" else er[:, 0].contiguous())
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    ref = g.aggregate(op, X, F=F, **kw)
+    dests = [torch.full((n, ld), float("nan"), device=DEV) for _ in range(3)]
+    tlp.tlp_debug_multi_store(g.handle, op, X, dests, F=F, **kw)
+    for d in dests:
+        assert torch.equal(d[:, :F], ref)
+        assert torch.isnan(d[:, F:]).all()
+    g.close()
+
+
+def test_fused_allgather_world1(tlp):
+    """NCCL world of one: symmetric buffer + fused dist aggregation == single GPU."""
+    n = 1500
+    rp, ci = synth.chung_lu(n, 30000, 0.5, 52, device="cpu")
+    F, ld = 70, 72
+    X = _t(synth.features(n, F, ld, seed=6))
+    comm = tlp.tlp_comm_create(tlp.tlp_comm_get_unique_id(), 1, 0)
+    h = tlp.tlp_dist_graph_create(comm, _t(rp), _t(ci))
+    Ysym, ptr = tlp.tlp_comm_alloc_symmetric(comm, n, ld)
+    tlp.tlp_dist_aggregate_fused(h, comm, "gcn", X, Ysym, F=F, norm="both")
+    g = tlp.Graph(_t(rp), _t(ci))
+    assert torch.equal(Ysym[:, :F], g.gcn(X, "both", F=F))
+    tlp.tlp_comm_free_symmetric(comm, ptr)
+    tlp.tlp_graph_destroy(h)
+    tlp.tlp_comm_destroy(comm)
+    g.close()
