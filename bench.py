@@ -296,6 +296,23 @@ def run_tlp(args):
     # ---- device-resident timed region ----
     ev = {op: [] for op in ops}
     start, stop = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    graphs = None
+    if args.cuda_graph:
+        # launch-bound small graphs: one CUDA graph per op, replayed (no host gaps)
+        graphs = {}
+        side = torch.cuda.Stream(dev)
+        side.wait_stream(stream)
+        with torch.cuda.stream(side):
+            for op in ops:
+                cg = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(cg, stream=side):
+                    launch(op)
+                graphs[op] = cg
+        stream.wait_stream(side)
+        torch.cuda.synchronize()
+        for op in ops:
+            graphs[op].replay()
+        torch.cuda.synchronize()
     if use_dist:
         dist.barrier()
     torch.cuda.synchronize()
@@ -305,15 +322,20 @@ def run_tlp(args):
             for op in ops:
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 a.record(stream)
-                launch(op)
+                if graphs is not None:
+                    for _r in range(args.graph_reps):
+                        graphs[op].replay()
+                else:
+                    launch(op)
                 b.record(stream)
                 ev[op].append((a, b))
         stop.record(stream)
         torch.cuda.synchronize()
     if use_dist:
         dist.barrier()
-    total_ms = start.elapsed_time(stop)
-    op_ms = {op: [a.elapsed_time(b) for a, b in ev[op]] for op in ops}
+    reps = args.graph_reps if graphs is not None else 1
+    total_ms = start.elapsed_time(stop) / reps
+    op_ms = {op: [a.elapsed_time(b) / reps for a, b in ev[op]] for op in ops}
     t = torch.tensor([total_ms], device=dev)
     if use_dist:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -440,7 +462,8 @@ def run_tlp(args):
         "ops": per_op, "create_ms": round(create_ms, 1),
         "plan": {k: info[k] for k in ("n_hubs", "n_hub_chunks", "n_units", "n_tasks",
                                       "hub_threshold", "hub_chunk", "max_in_degree")},
-        "roofline": roofline, "gpu_launches": args.steps * sum(LAUNCHES[o] for o in ops),
+        "roofline": roofline,
+        "gpu_launches": args.steps * sum(LAUNCHES[o] for o in ops) * (args.graph_reps if args.cuda_graph else 1),
         "clocks": clk.summary(), "e2e": e2e,
     }
     if use_dist:
@@ -551,6 +574,10 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--cuda-graph", action="store_true",
+                    help="replay each op as a captured CUDA graph (launch-bound small graphs)")
+    ap.add_argument("--graph-reps", type=int, default=20,
+                    help="graph replays per timed op with --cuda-graph (times are per replay)")
     ap.add_argument("--fused", action="store_true",
                     help="with --dist/torchrun: NEXT-2 fused compute + all-gather over NVLink peer memory")
     ap.add_argument("--dist", action="store_true",

@@ -1323,6 +1323,11 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         double width = panel ? (double)strip_w : (double)r.F;
         double bytes = edges_per_task * 4.0 * width;
         step = (int)std::min(32.0, std::max(1.0, std::ceil(32768.0 / std::max(bytes, 1.0))));
+        // ... but never so large that the resident warps (~SMs x 24) get fewer
+        // than ~4 fetches each: small graphs are latency-bound, spread them out
+        const double resident = (double)g->num_sms * 24.0;
+        const double cap = std::max(1.0, std::floor((double)a.n_items / (resident * 4.0)));
+        step = (int)std::min((double)step, cap);
     }
     a.step = step;
     a.sched = sched;

@@ -747,3 +747,54 @@ def test_fused_allgather_world1(tlp):
     tlp.tlp_graph_destroy(h)
     tlp.tlp_comm_destroy(comm)
     g.close()
+
+
+# ------------------------------------------------------------ robustness -----
+
+@pytest.mark.parametrize("scale", [30.0, 80.0])
+def test_gat_extreme_scores(tlp, scale):
+    """Large |el + er| (exp would overflow without the running max): still within tolerance."""
+    n = 1200
+    rp, ci = synth.chung_lu(n, 30000, 0.5, 61, device="cpu")
+    Xh = synth.features(n, 64, 64, seed=1)
+    el = synth.normal(n, 2) * scale
+    er = synth.normal(n, 3) * scale
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    for slope in (0.2, 1.0):
+        Y = g.gat(_t(Xh), _t(el), _t(er), slope)
+        assert torch.isfinite(Y).all()
+        _check(f"gat x{scale}", Y, oracle.gat(rp, ci, Xh, el, er, slope))
+    g.close()
+
+
+def test_very_wide_features(tlp):
+    n = 300
+    rp, ci = synth.power_law_rows(n, np.minimum((600 / (np.arange(n) + 1) ** 0.6).astype(int) + 1, 400), n, 5)
+    F, ld = 4100, 4104
+    Xh = synth.features(n, F, ld, seed=2)
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    _check("wide gcn", g.gcn(_t(Xh), "both", F=F), oracle.gcn(rp, ci, Xh, "both", F=F))
+    el, er = synth.normal(n, 1), synth.normal(n, 2)
+    _check("wide gat", g.gat(_t(Xh), _t(el), _t(er), 0.2, F=F), oracle.gat(rp, ci, Xh, el, er, 0.2, F=F))
+    g.close()
+
+
+def test_hub_of_one_repeated_source(tlp):
+    """A 5000-edge row whose edges all come from one source (multi-edges): every hub
+    chunk has the same partial; the ordered merge must still count each once."""
+    n = 50
+    src = np.concatenate([np.full(5000, 7), np.arange(1, 50)])
+    dst = np.concatenate([np.zeros(5000, np.int64), np.arange(1, 50)])
+    rp, ci = synth.csr_from_edges(n, src, dst)
+    Xh = synth.features(n, 33, 36, seed=3, low=0.0)
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    assert g.info["n_hubs"] == 1 and g.info["n_hub_chunks"] == 157
+    for nm in ("none", "right", "both"):
+        _check(f"repeat {nm}", g.gcn(_t(Xh), nm, F=33), oracle.gcn(rp, ci, Xh, nm, F=33))
+    Y = g.gcn(_t(Xh), "right", F=33)
+    # mean of 5000 copies of X[7] is X[7] (up to fp32 rounding of the sum)
+    assert torch.allclose(Y[0], _t(Xh)[7, :33], rtol=1e-5, atol=1e-6)
+    el = synth.normal(n, 4)
+    Yg = g.gat(_t(Xh), _t(el), _t(synth.normal(n, 5)), 0.2, F=33)
+    assert torch.allclose(Yg[0], _t(Xh)[7, :33], rtol=1e-5, atol=1e-6)
+    g.close()
