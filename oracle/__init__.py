@@ -77,6 +77,9 @@ def _load():
         lib.oracle_gcn_backward.restype = ctypes.c_int
         lib.oracle_gin_backward.argtypes = [I64, P, P, P, P, I64, I64, ctypes.c_double, P, P]
         lib.oracle_gin_backward.restype = ctypes.c_int
+        lib.oracle_gat_backward.argtypes = [I64, I64, P, P, P, I64, P, P, ctypes.c_double, P,
+                                            I64, I64, P, P, P, P, P, P]
+        lib.oracle_gat_backward.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -260,6 +263,29 @@ def gin_backward(rowptr, colidx, dY, eps, ew=None, F=None):
     if rc:
         raise ValueError("oracle_gin_backward: bad arguments")
     return dX, A
+
+
+def gat_backward(rowptr, colidx, X, el, er, slope, dY, F=None):
+    """Single-head GAT backward.  Returns ((dX, AdX), (del, Adel), (der, Ader)):
+    dX [n_src, F], del [n_src], der [n_dst] with their sum|terms| bounds."""
+    rowptr, colidx = _csr(rowptr, colidx)
+    X = _feat(X)
+    dY = _feat(dY)
+    n_dst = rowptr.shape[0] - 1
+    n_src = X.shape[0]
+    F = X.shape[1] if F is None else F
+    el = np.ascontiguousarray(el, dtype=np.float32)
+    er = np.ascontiguousarray(er, dtype=np.float32)
+    dX = np.empty((n_src, F)); AdX = np.empty((n_src, F))
+    dl = np.empty(n_src); Adl = np.empty(n_src)
+    dr = np.empty(n_dst); Adr = np.empty(n_dst)
+    rc = _load().oracle_gat_backward(n_dst, n_src, _ptr(rowptr), _ptr(colidx), _ptr(X),
+                                     X.strides[0] // 4, _ptr(el), _ptr(er), float(slope), _ptr(dY),
+                                     F, dY.strides[0] // 4, _ptr(dX), _ptr(AdX), _ptr(dl),
+                                     _ptr(Adl), _ptr(dr), _ptr(Adr))
+    if rc:
+        raise ValueError("oracle_gat_backward: bad arguments")
+    return (dX, AdX), (dl, Adl), (dr, Adr)
 
 
 ACTS = {"none": 0, "relu": 1, "leaky_relu": 2, "elu": 3}

@@ -469,3 +469,99 @@ int oracle_gin_backward(int64_t n, const int64_t *rowptr, const int32_t *colidx,
         }
     return 0;
 }
+
+/* GAT backward (single head; the training workload of the attention layer,
+ * P:1001-1007, Velickovic [43]).  Forward, per destination v with in-edges e
+ * (source u = colidx[e]):  t_e = el[u] + er[v],  s_e = LeakyReLU(t_e),
+ * alpha_e = softmax over the in-edges of v of s_e,  Y[v] = sum_e alpha_e X[u].
+ * Given dY, the chain rule written out step by step:
+ *   g_e   = sum_f dY[v,f] X[u,f]                 (dL/dalpha_e)
+ *   S_v   = sum_e alpha_e g_e
+ *   ds_e  = alpha_e (g_e - S_v)                  (softmax Jacobian)
+ *   dt_e  = ds_e * (t_e >= 0 ? 1 : slope)        (LeakyReLU, reading R6)
+ *   dX[u,f] += alpha_e dY[v,f];  del[u] += dt_e;  der[v] += dt_e.
+ * Bound terms (sum |terms|, for the parity criterion): G_e = sum_f |dY X|,
+ * B_e = |slope_e| alpha_e (G_e + sum_e' alpha_e' G_e') for dt_e, and
+ * |alpha_e dY[v,f]| for dX.  dX, AdX: [n_src x F]; del, Adel: [n_src];
+ * der, Ader: [n_dst].  Two-pass softmax as in oracle_gat. */
+int oracle_gat_backward(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
+                        const int32_t *colidx, const float *X, int64_t ldx,
+                        const float *el, const float *er, double slope,
+                        const float *dY, int64_t F, int64_t lddy,
+                        double *dX, double *AdX, double *del, double *Adel,
+                        double *der, double *Ader)
+{
+    if (F < 0 || ldx < F || lddy < F)
+        return -1;
+    for (int64_t i = 0; i < n_src * F; ++i) {
+        dX[i] = 0.0;
+        AdX[i] = 0.0;
+    }
+    for (int64_t u = 0; u < n_src; ++u) {
+        del[u] = 0.0;
+        Adel[u] = 0.0;
+    }
+    for (int64_t v = 0; v < n_dst; ++v) {
+        int64_t e0 = rowptr[v], e1 = rowptr[v + 1];
+        int64_t d = e1 - e0;
+        der[v] = 0.0;
+        Ader[v] = 0.0;
+        if (d == 0)
+            continue;
+        double *alpha = (double *)malloc(sizeof(double) * (size_t)d);
+        double *g = (double *)malloc(sizeof(double) * (size_t)d);
+        double *G = (double *)malloc(sizeof(double) * (size_t)d);
+        if (!alpha || !g || !G) {
+            free(alpha); free(g); free(G);
+            return -1;
+        }
+        double er_v = (double)er[v];
+        /* forward softmax, two passes (as oracle_gat) */
+        double m = -INFINITY;
+        for (int64_t e = e0; e < e1; ++e) {
+            double s = leaky_relu((double)el[colidx[e]] + er_v, slope);
+            alpha[e - e0] = s;
+            if (s > m)
+                m = s;
+        }
+        double z = 0.0;
+        for (int64_t k = 0; k < d; ++k)
+            z += exp(alpha[k] - m);
+        for (int64_t k = 0; k < d; ++k)
+            alpha[k] = exp(alpha[k] - m) / z;
+        /* g_e, S_v */
+        double S = 0.0, SA = 0.0;
+        for (int64_t e = e0; e < e1; ++e) {
+            int64_t u = colidx[e];
+            double gg = 0.0, GG = 0.0;
+            for (int64_t f = 0; f < F; ++f) {
+                double t = (double)dY[v * lddy + f] * (double)X[u * ldx + f];
+                gg += t;
+                GG += fabs(t);
+            }
+            g[e - e0] = gg;
+            G[e - e0] = GG;
+            S += alpha[e - e0] * gg;
+            SA += alpha[e - e0] * GG;
+        }
+        for (int64_t e = e0; e < e1; ++e) {
+            int64_t u = colidx[e];
+            double a = alpha[e - e0];
+            double t = (double)el[u] + er_v;
+            double lr = t >= 0.0 ? 1.0 : slope;
+            double dt = a * (g[e - e0] - S) * lr;
+            double bt = fabs(lr) * a * (G[e - e0] + SA);
+            der[v] += dt;
+            Ader[v] += bt;
+            del[u] += dt;
+            Adel[u] += bt;
+            for (int64_t f = 0; f < F; ++f) {
+                double term = a * (double)dY[v * lddy + f];
+                dX[u * F + f] += term;
+                AdX[u * F + f] += fabs(term);
+            }
+        }
+        free(alpha); free(g); free(G);
+    }
+    return 0;
+}

@@ -529,3 +529,117 @@ def test_p2_brute_gin_backward(case):
     A, _ = _dense_adj(rp, ci, n, n, ew)
     np.testing.assert_allclose(dX, 1.3 * dY.astype(np.float64) + A.T @ dY.astype(np.float64),
                                rtol=1e-12, atol=1e-13)
+
+
+# ---------------------------------------------------- NEXT-4: GAT backward -----
+
+def test_gat_backward_hand_worked():
+    """One destination with two sources, el = er = 0 (alpha = 1/2 each), F = 1,
+    X = [1, 3], dY = 1:  g = [1, 3], S = 2, ds = [-1/2, 1/2]; t = 0 >= 0 so
+    dt = ds;  del = [-1/2, 1/2], der = 0, dX = [1/2, 1/2]."""
+    rp = np.array([0, 2, 2, 2], dtype=np.int64)
+    ci = np.array([1, 2], dtype=np.int32)
+    X = np.array([[0.0], [1.0], [3.0]], dtype=np.float32)
+    z = np.zeros(3, dtype=np.float32)
+    dY = np.array([[1.0], [0.0], [0.0]], dtype=np.float32)
+    (dX, _), (dl, _), (dr, _) = oracle.gat_backward(rp, ci, X, z, z, 0.2, dY)
+    np.testing.assert_allclose(dX[:, 0], [0.0, 0.5, 0.5], atol=1e-15)
+    np.testing.assert_allclose(dl, [0.0, -0.5, 0.5], atol=1e-15)
+    np.testing.assert_allclose(dr, [0.0, 0.0, 0.0], atol=1e-15)
+
+
+def _torch_dense_gat_grads(rp, ci, X, el, er, slope, dY, n_src):
+    """Autograd (torch, fp64, CPU) of L = <Y, dY> for the dense masked-softmax
+    GAT (multi-edges weighted by their count): a library routine independent of
+    the oracle's hand-written chain rule."""
+    import torch
+    n_dst = len(rp) - 1
+    _, C = _dense_adj(rp, ci, n_dst, n_src)
+    Ct = torch.tensor(C, dtype=torch.float64)
+    Xt = torch.tensor(X.astype(np.float64), requires_grad=True)
+    elt = torch.tensor(el.astype(np.float64), requires_grad=True)
+    ert = torch.tensor(er.astype(np.float64)[:n_dst], requires_grad=True)
+    T = ert[:, None] + elt[None, :]
+    S = torch.where(T >= 0, T, slope * T)
+    mask = Ct > 0
+    Sm = torch.where(mask, S, torch.full_like(S, -1e300))
+    m = Sm.max(1, keepdim=True).values.detach()
+    P = torch.where(mask, Ct * torch.exp(torch.where(mask, S - m, torch.zeros_like(S))),
+                    torch.zeros_like(S))
+    Z = P.sum(1, keepdim=True)
+    P = P / torch.where(Z > 0, Z, torch.ones_like(Z))
+    Y = P @ Xt
+    (Y * torch.tensor(dY.astype(np.float64))).sum().backward()
+    return Xt.grad.numpy(), elt.grad.numpy(), ert.grad.numpy()
+
+
+@pytest.mark.parametrize("case", range(6))
+@pytest.mark.parametrize("slope", [0.2, 1.0, 0.0])
+def test_p2_autograd_gat_backward(case, slope):
+    rp, ci, n_src = _small_cases()[case]
+    n_dst = len(rp) - 1
+    F = 5
+    X = synth.features(n_src, F, seed=case + 60)
+    el = synth.normal(n_src, case + 61)
+    er = synth.normal(n_dst, case + 62)
+    dY = synth.features(n_dst, F, seed=case + 63)
+    (dX, AdX), (dl, Adl), (dr, Adr) = oracle.gat_backward(rp, ci, X, el, er, slope, dY)
+    tX, tl, tr = _torch_dense_gat_grads(rp, ci, X, el, er, slope, dY, n_src)
+    np.testing.assert_allclose(dX, tX, rtol=1e-11, atol=1e-13)
+    np.testing.assert_allclose(dl, tl, rtol=1e-10, atol=1e-12)
+    np.testing.assert_allclose(dr, tr, rtol=1e-10, atol=1e-12)
+    # bound terms dominate the values
+    assert np.all(np.abs(dX) <= AdX + 1e-15) and np.all(np.abs(dl) <= Adl + 1e-15)
+    assert np.all(np.abs(dr) <= Adr + 1e-15)
+
+
+def test_p4_gat_backward_invariants(pub):
+    """sum_v der = sum_u del (both are sum_e dt_e); slope = 1 gives der = 0
+    (softmax gradients sum to zero over a row, shift invariance); dX of
+    constant-score rows is the GCN-RIGHT transpose; <Y, G> = <X, dX> (Y is
+    linear in X for fixed scores)."""
+    rp, ci, n = pub
+    F = 3
+    X = synth.features(n, F, seed=5)
+    el = synth.normal(n, 6)
+    er = synth.normal(n, 7)
+    G = synth.features(n, F, seed=8)
+    (dX, _), (dl, Adl), (dr, Adr) = oracle.gat_backward(rp, ci, X, el, er, 0.2, G)
+    assert abs(dl.sum() - dr.sum()) <= 1e-9 * (Adl.sum() + 1)
+    Y, _ = oracle.gat(rp, ci, X, el, er, 0.2)
+    assert abs(float((Y * G.astype(np.float64)).sum()) -
+               float((X.astype(np.float64) * dX).sum())) <= 1e-9 * (np.abs(Y).sum() + 1)
+    (_, _), (_, _), (dr1, Adr1) = oracle.gat_backward(rp, ci, X, el, er, 1.0, G)
+    assert np.all(np.abs(dr1) <= 1e-12 * (Adr1 + 1))
+    z = np.zeros(n, dtype=np.float32)
+    (dXc, _), _, _ = oracle.gat_backward(rp, ci, X, z, z, 0.2, G)
+    dXr, _ = oracle.gcn_backward(rp, ci, G, "right")
+    np.testing.assert_allclose(dXc, dXr, rtol=1e-12, atol=1e-14)
+
+
+def test_gat_backward_finite_differences():
+    """Central differences of L = <GAT(X, el, er), dY> in fp64 (the dense
+    forward, h = 1e-6) against the oracle's del / der."""
+    rp, ci, n_src = _small_cases()[2]
+    n_dst = len(rp) - 1
+    X = synth.features(n_src, 4, seed=70)
+    el = synth.normal(n_src, 71).astype(np.float64)
+    er = synth.normal(n_dst, 72).astype(np.float64)
+    dY = synth.features(n_dst, 4, seed=73).astype(np.float64)
+    (_, _), (dl, _), (dr, _) = oracle.gat_backward(rp, ci, X, el.astype(np.float32),
+                                                   er.astype(np.float32), 0.2, dY.astype(np.float32))
+
+    def loss(el_, er_):
+        return float((_brute_gat(rp, ci, X, el_, er_, 0.2, n_src) * dY).sum())
+
+    h = 1e-6
+    for u in range(0, n_src, 5):
+        ep, em = el.copy(), el.copy()
+        ep[u] += h
+        em[u] -= h
+        assert abs((loss(ep, er) - loss(em, er)) / (2 * h) - dl[u]) <= 1e-6 * (abs(dl[u]) + 1)
+    for v in range(0, n_dst, 5):
+        ep, em = er.copy(), er.copy()
+        ep[v] += h
+        em[v] -= h
+        assert abs((loss(el, ep) - loss(el, em)) / (2 * h) - dr[v]) <= 1e-6 * (abs(dr[v]) + 1)
