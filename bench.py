@@ -57,6 +57,12 @@ def gather_bytes(op, n_rows, n_edges, F):
         return 2 * gather_bytes("gcn", n_rows, n_edges, F)
     if op == "gcn_bwd":  # dX = M^T dY on the transposed CSR: same byte model as GCN
         return gather_bytes("gcn", n_rows, n_edges, F)
+    if op == "gat_bwd":
+        # GAT backward (tlp_gat_backward): per edge one dY row (4F) on the
+        # transposed CSR, plus the scalar edge streams of its four passes
+        # (colidx/el 8, colidx/vstat/dot 24, colidx/vstat/dot/dt 28, tpos/dt 8);
+        # per row dY.Y (8F), X[u] and dX[u] (8F) and ~60 B of row scalars
+        return n_edges * (4 * F + 68) + n_rows * (16 * F + 60)
     if op == "sage":  # mean over N(v)+v: per edge 4F + 4; per row self + Y + rowptr
         return n_edges * (4 * F + 4) + n_rows * (8 * F + 8)
     if op.startswith("gat") and op[3:].isdigit():  # H heads: el/er per head
@@ -161,15 +167,19 @@ WORKLOADS = {
     "products_gat4": dict(graph="products", ops=("gat4",)),
     # NEXT-4: the backward aggregation of a GCN(BOTH) layer
     "reddit_bwd": dict(graph="reddit", ops=("gcn_bwd",)),
+    "reddit_gat_bwd": dict(graph="reddit", ops=("gat_bwd",)),
+    "pubmed_gat_bwd": dict(graph="pubmed", ops=("gat_bwd",)),
 }
-LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2, "sage": 1, "gat4": 1, "gcn_bwd": 1}
+LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2, "sage": 1, "gat4": 1, "gcn_bwd": 1,
+            "gat_bwd": 4}
 
 
 def workload_desc(name, cfg, E):
     ops = "+".join({"gcn": "GCN(both)", "gin": "GIN(eps=0.1)", "gat": "GAT(slope=0.2)",
                     "gcn2": "2-layer GCN(both)", "sage": "GraphSage-mean(+self)",
                     "gat4": "4-head GAT(slope=0.2)",
-                    "gcn_bwd": "GCN(both) backward dX = M^T dY"}[o] for o in WORKLOADS[name]["ops"])
+                    "gcn_bwd": "GCN(both) backward dX = M^T dY",
+                    "gat_bwd": "GAT(slope=0.2) backward (dX, del, der)"}[o] for o in WORKLOADS[name]["ops"])
     return f"{name}-shaped {ops}: N={cfg_n(cfg)} E={E} F={cfg['F']} ld={cfg['ld']}"
 
 
@@ -227,7 +237,7 @@ def run_tlp(args):
         g = tlp.Graph(rp_d, ci_d)
     torch.cuda.synchronize()
     create_ms = (time.perf_counter() - t0) * 1e3
-    if "gcn_bwd" in ops:
+    if "gcn_bwd" in ops or "gat_bwd" in ops:
         g.build_transpose()
     info = g.info
     del ci_d
@@ -263,6 +273,8 @@ def run_tlp(args):
             gcn_to(Xin, Yo[op])
         elif op == "gcn_bwd":
             g.gcn_backward(Xin, "both", dX=Yo[op], F=F)
+        elif op == "gat_bwd":  # dY = Xin, forward output Yfwd (computed once below)
+            g.gat_backward(X, elv, erv, synth.SLOPE, Yfwd, Xin, dX=Yo[op], F=F)
         elif fused:
             kw = dict(eps=synth.EPS, slope=synth.SLOPE, include_self=True)
             if op.startswith("gat"):
@@ -288,6 +300,9 @@ def run_tlp(args):
         else:
             g.gat_mh(Xin, elv, erv, int(op[3:]), synth.SLOPE, Y=Yo[op], F=F)
 
+    Yfwd = None
+    if "gat_bwd" in ops:  # the forward output the backward takes (not timed)
+        Yfwd = g.gat(X, el, er, synth.SLOPE, F=F)
     for _ in range(args.warmup):
         for op in ops:
             launch(op)
@@ -504,6 +519,12 @@ def _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows):
             oracle.sage(rp, ci, Xh, include_self=True, rows=rows, F=F)
         elif op == "gat":
             oracle.gat(rp, ci, Xh, elh, erh, synth.SLOPE, rows=rows, F=F)
+        elif op == "gat_bwd":
+            # the backward of the sampled destination rows: the sub-CSR of their
+            # in-edges (every gradient term belongs to exactly one such row)
+            sub_rp = np.concatenate([[0], np.cumsum(rp[rows + 1] - rp[rows])]).astype(np.int64)
+            sub_ci = np.concatenate([ci[rp[v]:rp[v + 1]] for v in rows]).astype(np.int32)
+            oracle.gat_backward(sub_rp, sub_ci, Xh, elh, erh[rows], synth.SLOPE, Xh[rows], F=F)
         else:
             H = int(op[3:])
             oracle.gat_mh(rp, ci, Xh, elh, erh, H, synth.SLOPE, rows=rows, Fh=F // H)

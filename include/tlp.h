@@ -288,6 +288,26 @@ tlp_status tlp_gin_backward(tlp_graph g, const float *dY, int64_t F,
                             int64_t lddy, float eps, float *dX, int64_t lddx,
                             void *stream);
 
+/* GAT backward (single head; the training workload of the attention layer,
+ * P:1001-1007 / Velickovic [43]).  Forward: t_e = el[u] + er[v],
+ * s_e = LeakyReLU(t_e, slope), alpha_e = softmax of s_e over the in-edges of v,
+ * Y[v] = sum_e alpha_e X[u].  Given dY = dL/dY it writes
+ *   dX[u]  = sum_{edges e: u -> v} alpha_e dY[v]                 [n_src x lddx]
+ *   del[u] = sum_{edges e: u -> v} dt_e,  der[v] = sum_{e in v} dt_e,
+ *   dt_e   = alpha_e (dY[v].X[u] - dY[v].Y[v]) (t_e >= 0 ? 1 : slope).
+ * X: fp32 device [n_src x ldx]; el [n_src], er [n_dst], del [n_src], der [n_dst]
+ * fp32 device; Y: the forward output of tlp_gat_aggregate for the same inputs,
+ * [n_dst x ldy]; dY [n_dst x lddy].  Needs tlp_graph_build_transpose.  Four
+ * launches (softmax state, the fused dX + edge-dot aggregation on the
+ * transposed CSR, two per-row reductions), stream-ordered, deterministic.
+ * Scratch: n_dst*16 + nnz*4 bytes on the handle and (strips x nnz x 4) bytes on
+ * its transpose, grown on demand.  F = 0 writes del = der = 0. */
+tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
+                            const float *el, const float *er, float slope,
+                            const float *Y, int64_t ldy, const float *dY,
+                            int64_t lddy, float *dX, int64_t lddx, float *del,
+                            float *der, void *stream);
+
 /* ---- multi-GPU (destination-row ranges balanced by edge count) ------------ */
 
 /* Pure host function: bounds[0] = 0, bounds[parts] = n, and for 0 < k < parts

@@ -82,6 +82,8 @@ _sig = {
     "tlp_graph_build_transpose": ([_P, _P], _I),
     "tlp_gcn_backward": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_gin_backward": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
+    "tlp_gat_backward": ([_P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P, _I64, _P, _I64, _P, _P, _P],
+                         _I),
     "tlp_gcn_aggregate": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_gin_aggregate": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
     "tlp_gat_aggregate": ([_P, _P, _I64, _I64, _P, _P, _F, _P, _I64, _P], _I),
@@ -406,6 +408,25 @@ def tlp_gin_backward(g, dY, eps=0.0, dX=None, F=None, stream=None, n_src=None):
     return dX
 
 
+def tlp_gat_backward(g, X, el, er, slope, Y, dY, dX=None, F=None, stream=None):
+    """Single-head GAT backward: returns (dX [n_src, F], del [n_src], der [n_dst]).
+    Y is the forward output of tlp_gat_aggregate for the same X, el, er."""
+    torch = _torch()
+    X, F, ldx = _feat(X, F)
+    Y, _, ldy = _feat(Y, F)
+    dY, _, lddy = _feat(dY, F)
+    el = _vec_cuda(el, "el")
+    er = _vec_cuda(er, "er")
+    info = tlp_graph_info_get(g)
+    dX, F, lddx = _out(dX, info["n_src"], F, dY)
+    dl = torch.empty(info["n_src"], dtype=torch.float32, device=dY.device)
+    dr = torch.empty(info["n_dst"], dtype=torch.float32, device=dY.device)
+    _check(_lib.tlp_gat_backward(g, _ptr(X), F, ldx, _ptr(el), _ptr(er), float(slope), _ptr(Y), ldy,
+                                 _ptr(dY), lddy, _ptr(dX), lddx, _ptr(dl), _ptr(dr),
+                                 _stream(stream, dY.device)), "tlp_gat_backward")
+    return dX, dl, dr
+
+
 # -------------------------------------------------------------- multi-GPU ----
 
 def tlp_partition_rows(rowptr, parts):
@@ -635,6 +656,9 @@ class Graph:
 
     def gin_backward(self, dY, eps=0.0, dX=None, F=None, stream=None):
         return tlp_gin_backward(self.handle, dY, eps, dX, F, stream, n_src=self.info["n_src"])
+
+    def gat_backward(self, X, el, er, slope, Y, dY, dX=None, F=None, stream=None):
+        return tlp_gat_backward(self.handle, X, el, er, slope, Y, dY, dX, F, stream)
 
     def degrees(self):
         return tlp_graph_degrees(self.handle)

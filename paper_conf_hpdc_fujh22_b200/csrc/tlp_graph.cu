@@ -8,6 +8,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstdio>
 #include <cstring>
 #include <string>
 
@@ -100,12 +101,14 @@ __global__ void k_iota(int32_t *__restrict__ v, int64_t n) {
 
 __global__ void k_permute_edges(const int32_t *__restrict__ perm, int64_t nnz,
                                 const int32_t *__restrict__ dst, const float *__restrict__ ew,
-                                int32_t *__restrict__ t_col, float *__restrict__ t_ew) {
+                                int32_t *__restrict__ t_col, float *__restrict__ t_ew,
+                                int32_t *__restrict__ tpos) {
     for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz;
          k += (int64_t)gridDim.x * blockDim.x) {
         const int32_t e = perm[k];
         t_col[k] = dst[e];
         if (ew) t_ew[k] = ew[e];
+        tpos[e] = (int32_t)k;  // inverse permutation (GAT backward)
     }
 }
 
@@ -215,7 +218,7 @@ static void graph_free(tlp_graph g) {
     if (!g) return;
     if (g->t) graph_free(g->t);
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
-                    g->c_out_left,
+                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)
@@ -242,6 +245,15 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
                              const tlp_create_opts *opts, cudaStream_t s,
                              tlp_graph *out) {
     auto t0 = std::chrono::steady_clock::now();
+    // TLP_TRACE_CREATE=1: synchronise and print the elapsed time at each phase
+    static const bool trace = getenv("TLP_TRACE_CREATE") != nullptr;
+    auto mark = [&](const char *what) {
+        if (!trace) return;
+        cudaStreamSynchronize(s);
+        const double ms = std::chrono::duration<double, std::milli>(
+                              std::chrono::steady_clock::now() - t0).count();
+        fprintf(stderr, "[tlp create] %-28s %9.3f ms\n", what, ms);
+    };
     if (!out) return set_error(TLP_ERR_INVALID_ARGUMENT, "out is NULL");
     *out = nullptr;
     if (n_dst < 0 || n_src < 0 || nnz < 0 || row_offset < 0)
@@ -279,6 +291,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
     g->last_stream = s;
     const int nsm = g->num_sms;
 
+    mark("setup");
     // ---- a1: ingest (copy; rebased rowptr) and validate -------------------
     TRY(dmalloc((void **)&g->rowptr, sizeof(int64_t) * (n_dst + 1), g));
     TRY(dmalloc((void **)&g->in_deg, sizeof(int32_t) * n_dst, g));
@@ -331,6 +344,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         }
     }
 
+    mark("a1 ingest+validate");
     // ---- a2: degrees and BOTH-norm coefficients --------------------------
     TRY(dmalloc((void **)&g->out_deg, sizeof(int32_t) * n_src, g));
     TRY(dmalloc((void **)&g->c_out, sizeof(float) * n_src, g));
@@ -354,6 +368,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         }
     }
 
+    mark("a2 degrees+norms");
     // ---- a3: work plan ---------------------------------------------------
     TRY(dmalloc((void **)&g->ctr, sizeof(unsigned int) * 4, g));
     CTRY(cudaMemsetAsync(g->ctr, 0, sizeof(unsigned int) * 4, s));
@@ -483,6 +498,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         g->regular_edges = nnz - std::min<int64_t>(nnz, g->n_chunks * g->C);
         if (g->regular_edges < 0) g->regular_edges = 0;
     }
+    mark("a3 plan");
     auto t1 = std::chrono::steady_clock::now();
     g->create_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
     *out = g;
@@ -506,6 +522,10 @@ tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
     TLP_CUDA_TRY(cudaMalloc(&perm.p, sizeof(int32_t) * nnz + 16));
     TLP_CUDA_TRY(cudaMalloc(&t_col.p, sizeof(int32_t) * nnz + 16));
     if (g->ew) TLP_CUDA_TRY(cudaMalloc(&t_ew.p, sizeof(float) * nnz + 16));
+    if (!g->tpos) {
+        TLP_CUDA_TRY(cudaMalloc(&g->tpos, sizeof(int32_t) * nnz + 16));
+        g->device_bytes += sizeof(int32_t) * nnz + 16;
+    }
     TLP_CUDA_TRY(cudaMalloc(&t_rp.p, sizeof(int64_t) * (n_src + 1)));
     TLP_CUDA_TRY(cudaMalloc(&deg64.p, sizeof(int64_t) * (n_src + 1)));
     if (n_dst) {
@@ -524,7 +544,8 @@ tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
                                                      iota.as<int32_t>(), perm.as<int32_t>(), (int)nnz,
                                                      0, 32, s));
         k_permute_edges<<<grid_for(nnz, nsm), 256, 0, s>>>(perm.as<int32_t>(), nnz, dst.as<int32_t>(),
-                                                           g->ew, t_col.as<int32_t>(), t_ew.as<float>());
+                                                           g->ew, t_col.as<int32_t>(), t_ew.as<float>(),
+                                                           g->tpos);
         TLP_CUDA_TRY(cudaGetLastError());
     }
     // transposed rowptr = exclusive scan of the out-degrees

@@ -47,6 +47,13 @@ struct tlp_graph_s {
     float *ew_both = nullptr;    // [nnz] c_out[colidx[e]] * w_e (GCN BOTH coefficient)
     float *c_out_left = nullptr; // [n_src] 1/max(out_deg,1) (internal LEFT norm, backward of RIGHT)
     tlp_graph_s *t = nullptr;    // transposed graph (tlp_graph_build_transpose), owned
+    // source-reuse tags: colidx with the
+    // out-degree class of each source in bits 27-31, built on first use
+    int32_t *colidx_tag = nullptr;   // [nnz] or null
+    int32_t *tpos = nullptr;         // [nnz] forward edge -> transposed position (with t)
+    float *bwd = nullptr;            // GAT backward scratch (see tlp_gat_backward)
+    size_t bwd_bytes = 0;
+    int64_t tag_hist[32] = {0};      // sources per out-degree class
 
     int2 *tasks = nullptr;       // [n_tasks]
     int32_t *hub_row = nullptr;  // [n_hubs]
@@ -110,6 +117,15 @@ struct AggRequest {
     float act_param = 0.f;
     float *const *dests = nullptr;  // fused all-gather destinations (device array)
     int n_dests = 0;
+    // op 5 (GAT backward on the transposed graph, NEXT-4): X = dY, Y = dX,
+    // el = forward el (per transposed row), xself = forward X, vstat = per
+    // forward-destination {er, m, 1/z, <dY,Y>}; aggregate() allocates the
+    // per-strip edge dot products gbuf [n_strips x nnz] and reports them.
+    const float *xself = nullptr;
+    int64_t ldxs = 0;
+    const void *vstat = nullptr;
+    float **gbuf_out = nullptr;
+    int *n_strips_out = nullptr;
 };
 
 inline AggRequest request_from_desc(const tlp_agg_desc &d) {

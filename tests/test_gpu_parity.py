@@ -798,3 +798,110 @@ def test_hub_of_one_repeated_source(tlp):
     Yg = g.gat(_t(Xh), _t(el), _t(synth.normal(n, 5)), 0.2, F=33)
     assert torch.allclose(Yg[0], _t(Xh)[7, :33], rtol=1e-5, atol=1e-6)
     g.close()
+
+
+# ------------------------------------------------------ NEXT-4: GAT backward ----
+
+def _gat_bwd_case(tlp, rp, ci, n_src, F, ld, seed=0, opts=None, nonneg=False):
+    n_dst = len(rp) - 1
+    Xh = synth.features(n_src, F, ld, seed=seed + 1, low=0.0 if nonneg else -1.0)
+    elh = synth.normal(n_src, seed + 2)
+    erh = synth.normal(n_dst, seed + 3)
+    dYh = synth.features(n_dst, F, ld, seed=seed + 4)
+    g = tlp.Graph(_t(rp), _t(ci), n_src=n_src, opts=opts or dict(hub_threshold=64, hub_chunk=32))
+    g.build_transpose()
+    X, el, er, dY = _t(Xh), _t(elh), _t(erh), _t(dYh)
+    Y = g.gat(X, el, er, 0.2, F=F)
+    dX = torch.full((n_src, ld), float("nan"), device=DEV)
+    _, dl, dr = g.gat_backward(X, el, er, 0.2, Y, dY, dX=dX, F=F)
+    (rX, aX), (rl, al), (rr, ar) = oracle.gat_backward(rp, ci, Xh, elh, erh, 0.2, dYh, F=F)
+    _check("gat bwd dX", dX[:, :F], (rX, aX))
+    if ld > F:
+        assert torch.isnan(dX[:, F:]).all()
+    _check("gat bwd del", dl.view(-1, 1), (rl.reshape(-1, 1), al.reshape(-1, 1)))
+    _check("gat bwd der", dr.view(-1, 1), (rr.reshape(-1, 1), ar.reshape(-1, 1)))
+    g.close()
+
+
+@pytest.mark.parametrize("name", ["random64", "powerlaw_hubs", "selfloops_multi", "star_hub",
+                                  "rect_more_src", "rect_more_dst", "e0_n5", "isolated_last",
+                                  "one_row"])
+@pytest.mark.parametrize("F,ld", [(37, 40), (130, 132), (1, 1), (6, 6)])
+def test_gat_backward_parity(tlp, name, F, ld):
+    rp, ci, n_src = _edge_graphs()[name]
+    _gat_bwd_case(tlp, rp, ci, n_src, F, ld, seed=F)
+
+
+@pytest.mark.parametrize("panel", ["64", "128", "0"])
+def test_gat_backward_strip_modes(tlp, monkeypatch, panel):
+    """Half-warp PAIR strips (64), full-warp strips (128) and task-major rows (0)
+    give the oracle's result, with hubs split into chunks."""
+    monkeypatch.setenv("TLP_PANEL", panel)
+    rp, ci, n = _edge_graphs()["powerlaw_hubs"]
+    _gat_bwd_case(tlp, rp, ci, n, 300, 300, seed=5, nonneg=True)
+
+
+def test_gat_backward_pubmed_all_rows(tlp):
+    rp, ci = synth.dataset_graph("pubmed")
+    n = synth.CONFIGS["pubmed"]["n"]
+    _gat_bwd_case(tlp, rp, ci, n, 500, 500, seed=9, opts=dict())
+
+
+def test_gat_backward_reddit_properties(tlp, reddit):
+    """Full Reddit (F = 64): <GAT(X), G> = <X, dX> for fixed scores, and
+    sum del = sum der (both are the sum of dt_e), GPU on both sides, fp64 dots;
+    plus sampled destination rows of der against the oracle's definition on the
+    same rows (dt of a row only depends on that row's in-edges)."""
+    rp, ci = reddit
+    n, F = synth.CONFIGS["reddit"]["n"], 64
+    Xh = synth.features(n, F, F, seed=11)
+    G = _t(synth.features(n, F, F, seed=12))
+    el, er = _t(synth.normal(n, 13)), _t(synth.normal(n, 14))
+    X = _t(Xh)
+    g = tlp.Graph(_t(rp), _t(ci))
+    g.build_transpose()
+    Y = g.gat(X, el, er, 0.2)
+    dX, dl, dr = g.gat_backward(X, el, er, 0.2, Y, G)
+    lhs = (Y.double() * G.double()).sum().item()
+    rhs = (X.double() * dX.double()).sum().item()
+    assert abs(lhs - rhs) <= 1e-5 * (abs(lhs) + abs(rhs)) + 1e-3, (lhs, rhs)
+    sl, sr = dl.double().sum().item(), dr.double().sum().item()
+    scale = dl.double().abs().sum().item() + 1.0
+    assert abs(sl - sr) <= 1e-5 * scale, (sl, sr)
+    # sampled rows: der[v] from the oracle on the subgraph of v's in-edges
+    rng = np.random.default_rng(0)
+    deg = np.diff(rp)
+    rows = np.concatenate([rng.choice(n, 40, replace=False), np.argsort(deg)[-3:]])
+    Gh = G.cpu().numpy()
+    elh, erh = el.cpu().numpy(), er.cpu().numpy()
+    for v in rows:
+        e0, e1 = rp[v], rp[v + 1]
+        sub_rp = np.array([0, e1 - e0], np.int64)
+        sub_ci = ci[e0:e1].astype(np.int32)
+        _, _, (rr, ar) = oracle.gat_backward(sub_rp, sub_ci, Xh, elh, erh[v:v + 1], 0.2,
+                                             Gh[v:v + 1])
+        _check(f"reddit der[{v}]", dr[v:v + 1].view(1, 1), (rr.reshape(1, 1), ar.reshape(1, 1)))
+    g.close()
+
+
+@pytest.mark.parametrize("op", ["gcn", "gin", "gat"])
+def test_hot_source_policy_is_bitwise_neutral(tlp, monkeypatch, op):
+    """The hot-source L2 policy (tagged colidx, evict_last / evict_first gathers)
+    changes no bit of the output: small budget (some classes hot) == disabled."""
+    rp, ci = synth.chung_lu(20000, 400000, 0.5, 77, device="cpu")
+    n, F = 20000, 100
+    X = _t(synth.features(n, F, F, seed=1))
+    el, er = _t(synth.normal(n, 2)), _t(synth.normal(n, 3))
+    out = []
+    for frac in ("0", "0.002"):
+        monkeypatch.setenv("TLP_HOT", frac)
+        g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=256, hub_chunk=128))
+        if op == "gcn":
+            out.append(g.gcn(X, "both"))
+        elif op == "gin":
+            out.append(g.gin(X, 0.1))
+        else:
+            out.append(g.gat(X, el, er, 0.2))
+        torch.cuda.synchronize()
+        g.close()
+    assert torch.equal(out[0], out[1])
