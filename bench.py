@@ -171,7 +171,7 @@ WORKLOADS = {
     "pubmed_gat_bwd": dict(graph="pubmed", ops=("gat_bwd",)),
 }
 LAUNCHES = {"gcn": 1, "gin": 1, "gat": 1, "gcn2": 2, "sage": 1, "gat4": 1, "gcn_bwd": 1,
-            "gat_bwd": 4}
+            "gat_bwd": 5}
 
 
 def workload_desc(name, cfg, E):

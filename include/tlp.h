@@ -297,11 +297,12 @@ tlp_status tlp_gin_backward(tlp_graph g, const float *dY, int64_t F,
  *   dt_e   = alpha_e (dY[v].X[u] - dY[v].Y[v]) (t_e >= 0 ? 1 : slope).
  * X: fp32 device [n_src x ldx]; el [n_src], er [n_dst], del [n_src], der [n_dst]
  * fp32 device; Y: the forward output of tlp_gat_aggregate for the same inputs,
- * [n_dst x ldy]; dY [n_dst x lddy].  Needs tlp_graph_build_transpose.  Four
- * launches (softmax state, the fused dX + edge-dot aggregation on the
- * transposed CSR, two per-row reductions), stream-ordered, deterministic.
- * Scratch: n_dst*16 + nnz*4 bytes on the handle and (strips x nnz x 4) bytes on
- * its transpose, grown on demand.  F = 0 writes del = der = 0. */
+ * [n_dst x ldy]; dY [n_dst x lddy].  Needs tlp_graph_build_transpose.  Five
+ * launches (softmax state per destination, edge weights alpha_e in transposed
+ * order, the fused dX + edge-dot aggregation on the transposed CSR, two
+ * per-row reductions), stream-ordered, deterministic.  Scratch:
+ * n_dst*16 + 2*nnz*4 bytes on the handle and (strips x nnz x 4) bytes on its
+ * transpose, grown on demand.  F = 0 writes del = der = 0. */
 tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
                             const float *el, const float *er, float slope,
                             const float *Y, int64_t ldy, const float *dY,

@@ -102,12 +102,11 @@ struct AggArgs {
     // evict_first : evict_normal.  A cache policy only: no value changes.
     unsigned hot_thr;
     int cold_first;
-    // OP_GATB: forward X (the transposed row's own features), per forward
-    // destination {er, m, 1/z, <dY,Y>}, and the per-strip edge dot products
-    // gbuf[s * gstride + e] = sum over strip s of dY[v_e] . X[u] (transposed e).
+    // OP_GATB: forward X (the transposed row's own features) and the per-strip
+    // edge dot products gbuf[s * gstride + e] = sum over strip s of
+    // dY[v_e] . X[u] (transposed edge e).
     const float *xself;
     int64_t ldxs;
-    const float4 *vstat;
     float *gbuf;
     int64_t gstride;
 };
@@ -147,27 +146,6 @@ __device__ __forceinline__ Vec<VEC> ld_vec(const float *p) {
         r.v[0] = t.x; r.v[1] = t.y;
     } else {
         r.v[0] = __ldg(p);
-    }
-    return r;
-}
-
-// Gather of source row u (possibly tagged, see AggArgs::hot_thr).
-template <int VEC>
-__device__ __forceinline__ Vec<VEC> ld_x(const char *base, unsigned u, unsigned row_bytes,
-                                         const GPol &gp) {
-    const float *p = reinterpret_cast<const float *>(
-        base + (unsigned long long)(u & kIdxMask) * row_bytes);
-    if (gp.thr == 0) return ld_vec<VEC>(p);
-    const unsigned long long pol = u >= gp.thr ? gp.hot : gp.cold;
-    Vec<VEC> r;
-    if constexpr (VEC == 4) {
-        asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
-                     : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3]) : "l"(p), "l"(pol));
-    } else if constexpr (VEC == 2) {
-        asm volatile("ld.global.nc.L2::cache_hint.v2.f32 {%0, %1}, [%2], %3;"
-                     : "=f"(r.v[0]), "=f"(r.v[1]) : "l"(p), "l"(pol));
-    } else {
-        asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r.v[0]) : "l"(p), "l"(pol));
     }
     return r;
 }
@@ -253,16 +231,16 @@ __device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, un
 //              the strip of X is half as wide (each half-warp is one chain).
 
 template <int VEC, int U, bool HASC, bool PAIR, bool CLAMP>
-__device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes, const GPol &gp,
-                                            int j, int n, int half, int u_l, float c_l,
-                                            Vec<VEC> (&xv)[U], float (&ck)[U]) {
+__device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes, int j, int n,
+                                            int half, int u_l, float c_l, Vec<VEC> (&xv)[U],
+                                            float (&ck)[U]) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
         int p = PAIR ? 2 * (j + k) + half : j + k;
         if constexpr (CLAMP) p = min(p, n - 1);  // duplicate of a line in flight
         const unsigned u = (unsigned)__shfl_sync(FULL, u_l, p);
         if constexpr (HASC) ck[k] = __shfl_sync(FULL, c_l, p);
-        xv[k] = ld_x<VEC>(base, u, row_bytes, gp);
+        xv[k] = ld_vec<VEC>(row_ptr(base, u, row_bytes));
     }
 }
 
@@ -314,6 +292,51 @@ __device__ __forceinline__ void dot_group(int j, int n, int lane, const Vec<VEC>
     }
 }
 
+// OP_GATB, full 32-edge chunks: the per-step lane partials are reduced by a
+// streaming transposed butterfly.  Steps t are the gather steps of the chunk
+// (PAIR: 16 steps of two edges, one per half-warp, 4 levels xor 8,4,2,1; full
+// warp: 32 steps, 5 levels xor 16..1).  At level k a lane keeps the step whose
+// bit matches its lane bit and adds its partner's partial of that step, so one
+// shuffle reduces two steps; after the last level lane l holds the whole dot of
+// step bitreverse(l) (PAIR: of edge 2*rev4(l & 15) + half).  15 (PAIR) or 31
+// shuffles per 32 edges instead of 4-5 per edge.  t is a compile-time constant
+// in the unrolled full-chunk loop, so the level logic folds away.
+struct DotTree {
+    float lv[5];
+};
+template <bool PAIR>
+__device__ __forceinline__ void dot_push(DotTree &tr, float d, int t, int lane, float *gout) {
+    constexpr int L = PAIR ? 4 : 5;
+#pragma unroll
+    for (int k = 0; k < L; ++k) {
+        const int bitmask = (PAIR ? 8 : 16) >> k;  // lane bit of level k
+        if (((t >> k) & 1) == 0) {  // first of the pair at this level: park it
+            tr.lv[k] = d;
+            return;
+        }
+        const bool hi = (lane & bitmask) != 0;
+        const float keep = hi ? d : tr.lv[k];
+        const float send = hi ? tr.lv[k] : d;
+        d = keep + __shfl_xor_sync(FULL, send, bitmask);
+    }
+    // all levels done (t = last step): lane holds the dot of step rev(lane)
+    const int l = PAIR ? (lane & 15) : lane;
+    const int rv = PAIR ? (int)(__brev((unsigned)l) >> 28) : (int)(__brev((unsigned)l) >> 27);
+    const int e = PAIR ? 2 * rv + (lane >> 4) : rv;
+    gout[e] = d;
+}
+template <int VEC, int U, bool PAIR>
+__device__ __forceinline__ void dot_tree(int j, int lane, const Vec<VEC> (&xv)[U],
+                                         const Vec<VEC> &xu, DotTree &tr, float *gout) {
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+        float d = 0.f;
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) d = fmaf(xv[k].v[c], xu.v[c], d);
+        dot_push<PAIR>(tr, d, j + k, lane, gout);
+    }
+}
+
 // ---- L2 residency hints -------------------------------------------------------
 // Per-edge streams (colidx, edge coefficients) and Y are touched once per strip:
 // with TLP_HINTS they are loaded / stored with an L2 evict_first policy so they
@@ -360,8 +383,9 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
                                              int col, bool active, float er_v, int lane,
                                              Vec<VEC> &acc, float &m, float &den,
                                              const Vec<VEC> &xu, float *gout) {
-    // OP_GATB: er_v carries el[u] of the transposed row u; the coefficient of
-    // edge u -> v is alpha = exp(LeakyReLU(el[u] + er[v]) - m_v) / z_v
+    // OP_GATB: the coefficient of transposed edge u -> v is alpha_e, streamed
+    // (COEF_W) from the k_gatb_alpha pass; the strip's dot dY[v].X[u] of every
+    // edge is reduced across lanes and stored to gout
     constexpr bool GB = (OP == OP_GATB);
     constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT) || GB;
     constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);  // index-dependent value
@@ -370,7 +394,6 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
     const unsigned row_bytes = (unsigned)a.ldx * 4u;
     const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
-    const GPol gp = make_gpol(a);
     // 32-bit edge offsets relative to e0 (a row or hub chunk has < 2^31 edges)
     const int32_t *__restrict__ ci = a.colidx + e0;
     const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
@@ -385,7 +408,6 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
         int n1 = min(32, len - 32);
         int u0 = 0, u1 = 0;
         float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
-        float4 q0 = make_float4(0.f, 0.f, 0.f, 0.f), q1 = q0;  // OP_GATB: vstat[v]
         if (lane < n0) {
             u0 = ld_stream(ci + lane);
             if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane);
@@ -395,9 +417,7 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
         }
         if constexpr (DEP)
-            if (lane < n0) d0 = __ldg(dep + (u0 & kIdxMask));
-        if constexpr (GB)
-            if (lane < n0) q0 = __ldg(a.vstat + (u0 & kIdxMask));
+            if (lane < n0) d0 = __ldg(dep + u0);
         while (true) {
             // two chunks ahead: indices; one chunk ahead: index-dependent values
             const int n2 = min(32, len - off - 64);
@@ -408,9 +428,7 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
                 if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
             }
             if constexpr (DEP)
-                if (lane < n1) d1 = __ldg(dep + (u1 & kIdxMask));
-            if constexpr (GB)
-                if (lane < n1) q1 = __ldg(a.vstat + (u1 & kIdxMask));
+                if (lane < n1) d1 = __ldg(dep + u1);
             // coefficients of the current chunk
             float c_l = 1.f;
             if constexpr (OP == OP_GAT) {
@@ -429,58 +447,51 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
                     ac[1].v[c] *= scale;
                 }
                 m = m_new;
-            } else if constexpr (GB) {
-                c_l = 0.f;
-                if (lane < n0) {
-                    const float t = er_v + q0.x;
-                    const float sc = t >= 0.f ? t : a.slope * t;
-                    c_l = __expf(sc - q0.y) * q0.z;
-                }
             } else {
                 if constexpr (COEF & COEF_COUT) c_l = d0;
                 if constexpr (COEF & COEF_W) c_l *= w0;
             }
             Vec<VEC> xa[U], xb[U];
             float ca[U], cb[U];
-            float g_l = 0.f;  // OP_GATB: this strip's dot of edge `lane` of the chunk
+            float g_l = 0.f;  // OP_GATB (partial chunk): this strip's dot of edge `lane`
+            DotTree dt_;      // OP_GATB (full chunk): pending butterfly levels
             if (n0 == 32) {
                 // full chunk: fully unrolled, compile-time shuffle lanes, no guards
-                issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, gp, 0, 32, half, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, 0, 32, half, u0, c_l, xa, ca);
 #pragma unroll
                 for (int j = 0; j < STEPS; j += 2 * U) {
-                    issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, gp, j + U, 32, half, u0, c_l, xb, cb);
+                    issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, j + U, 32, half, u0, c_l, xb, cb);
                     consume_group<VEC, U, HASC, PAIR, false, 0>(j, 32, half, xa, ca, ac);
-                    if constexpr (GB) dot_group<VEC, U, PAIR, false>(j, 32, lane, xa, xu, g_l);
+                    if constexpr (GB) dot_tree<VEC, U, PAIR>(j, lane, xa, xu, dt_, gout + off);
                     if (j + 2 * U < STEPS)
-                        issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, gp, j + 2 * U, 32, half, u0, c_l, xa, ca);
+                        issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, j + 2 * U, 32, half, u0, c_l, xa, ca);
                     consume_group<VEC, U, HASC, PAIR, false, U>(j + U, 32, half, xb, cb, ac);
-                    if constexpr (GB) dot_group<VEC, U, PAIR, false>(j + U, 32, lane, xb, xu, g_l);
+                    if constexpr (GB) dot_tree<VEC, U, PAIR>(j + U, lane, xb, xu, dt_, gout + off);
                 }
             } else {
                 // partial chunk (n0 is warp-uniform: the guards never diverge)
                 const int steps = PAIR ? (n0 + 1) >> 1 : n0;
-                issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, gp, 0, n0, half, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, 0, n0, half, u0, c_l, xa, ca);
                 for (int j = 0; j < steps; j += 2 * U) {
                     const bool more = j + U < steps;
-                    if (more) issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, gp, j + U, n0, half, u0, c_l, xb, cb);
+                    if (more) issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, j + U, n0, half, u0, c_l, xb, cb);
                     consume_group<VEC, U, HASC, PAIR, true, 0>(j, n0, half, xa, ca, ac);
                     if constexpr (GB) dot_group<VEC, U, PAIR, true>(j, n0, lane, xa, xu, g_l);
                     if (j + 2 * U < steps)
-                        issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, gp, j + 2 * U, n0, half, u0, c_l, xa, ca);
+                        issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, j + 2 * U, n0, half, u0, c_l, xa, ca);
                     if (more) consume_group<VEC, U, HASC, PAIR, true, U>(j + U, n0, half, xb, cb, ac);
                     if constexpr (GB)
                         if (more) dot_group<VEC, U, PAIR, true>(j + U, n0, lane, xb, xu, g_l);
                 }
             }
             if constexpr (GB)
-                if (lane < n0) gout[off + lane] = g_l;
+                if (n0 < 32 && lane < n0) gout[off + lane] = g_l;  // partial chunk
             if (n1 <= 0) break;
             off += 32;
             n0 = n1; n1 = n2;
             u0 = u1; u1 = u2;
             w0 = w1; w1 = w2;
             d0 = d1;
-            q0 = q1;
         }
     }
     // even + odd (in PAIR mode the odd chain lives in the other half-warp)
@@ -1004,12 +1015,10 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
         float erl = 0.f;
         if constexpr (OP == OP_GAT)
             if (lane < nr) erl = __ldg(a.er + a.row_offset + rb + lane);
-        if constexpr (OP == OP_GATB)
-            if (lane < nr) erl = __ldg(a.el + rb + lane);
         for (int k = 0; k < nr; ++k) {
             const int64_t e0 = __shfl_sync(FULL, rp, k);
             const int64_t e1 = __shfl_sync(FULL, rp, k + 1);
-            const float er_v = (OP == OP_GAT || OP == OP_GATB) ? __shfl_sync(FULL, erl, k) : 0.f;
+            const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
             const int64_t r = rb + k;
             for (int s = s0; s < s1; ++s) {
                 const int col = strip_col<VEC, PAIR>(s, lane);
@@ -1066,7 +1075,6 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     const int64_t e1 = min(e0 + a.C, ee);
     float er_v = 0.f;
     if constexpr (OP == OP_GAT) er_v = __ldg(a.er + a.row_offset + r);
-    if constexpr (OP == OP_GATB) er_v = __ldg(a.el + r);
     const int slot = off + j;
     // this panel's (m, den) pairs: [n_chunks][heads] (heads = 1 unless OP_GATH)
     const int mdh = (OP == OP_GATH) ? a.heads : 1;
@@ -1252,7 +1260,7 @@ static KernelFn pick(int op, int coef) {
                              : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC, PAIR>;
     if (op == OP_SAGE) return k_agg<VEC, OP_SAGE, COEF_NONE, kU, ASYNC, PAIR>;
     if constexpr (!ASYNC)
-        if (op == OP_GATB) return k_agg<VEC, OP_GATB, COEF_NONE, kU, false, PAIR>;
+        if (op == OP_GATB) return k_agg<VEC, OP_GATB, COEF_W, kU, false, PAIR>;
     return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC, PAIR>;
 }
 
@@ -1303,9 +1311,10 @@ static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
 static bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
 // ---- GAT backward (NEXT-4) scalar passes -------------------------------------
-// The three passes around the OP_GATB aggregation:
+// The passes around the OP_GATB aggregation:
 //  k_gatb_stats (forward rows v): softmax state m_v, z_v of the forward scores
 //    and S_v = <dY[v], Y[v]> = sum_e alpha_e g_e, packed with er[v];
+//  k_gatb_alpha (transposed rows u): alpha_e, stored in transposed edge order;
 //  OP_GATB k_agg (transposed rows u): dX[u] = sum_e alpha_e dY[v_e] and the
 //    per-strip dots g_e = dY[v_e] . X[u], one gather of dY per edge;
 //  k_gatb_edges (transposed rows u): dt_e = alpha_e (g_e - S_v) LeakyReLU'(t_e),
@@ -1341,11 +1350,29 @@ __global__ void k_gatb_stats(const int64_t *__restrict__ rowptr, const int32_t *
     }
 }
 
-__global__ void k_gatb_edges(const int64_t *__restrict__ t_rowptr, const int32_t *__restrict__ t_colidx,
+__global__ void k_gatb_alpha(const int64_t *__restrict__ t_rowptr, const int32_t *__restrict__ t_colidx,
                              int64_t n_src, const float *__restrict__ el,
                              const float4 *__restrict__ vstat, float slope,
-                             const float *__restrict__ gbuf, int n_strips, int64_t gstride,
-                             float *__restrict__ dt, float *__restrict__ del) {
+                             float *__restrict__ alpha) {
+    const int lane = threadIdx.x & 31;
+    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t u = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; u < n_src; u += W) {
+        const int64_t e0 = t_rowptr[u], e1 = t_rowptr[u + 1];
+        const float el_u = el[u];
+        for (int64_t e = e0 + lane; e < e1; e += 32) {
+            const float4 q = vstat[t_colidx[e]];
+            const float t = el_u + q.x;
+            const float sc = t >= 0.f ? t : slope * t;
+            alpha[e] = __expf(sc - q.y) * q.z;
+        }
+    }
+}
+
+__global__ void k_gatb_edges(const int64_t *__restrict__ t_rowptr, const int32_t *__restrict__ t_colidx,
+                             int64_t n_src, const float *__restrict__ el,
+                             const float4 *__restrict__ vstat, const float *__restrict__ alpha,
+                             float slope, const float *__restrict__ gbuf, int n_strips,
+                             int64_t gstride, float *__restrict__ dt, float *__restrict__ del) {
     const int lane = threadIdx.x & 31;
     const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t u = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; u < n_src; u += W) {
@@ -1355,11 +1382,9 @@ __global__ void k_gatb_edges(const int64_t *__restrict__ t_rowptr, const int32_t
         for (int64_t e = e0 + lane; e < e1; e += 32) {
             const float4 q = vstat[t_colidx[e]];
             const float t = el_u + q.x;
-            const float sc = t >= 0.f ? t : slope * t;
-            const float alpha = __expf(sc - q.y) * q.z;
             float g = 0.f;
             for (int k = 0; k < n_strips; ++k) g += gbuf[(int64_t)k * gstride + e];
-            const float d = alpha * (g - q.w) * (t >= 0.f ? 1.f : slope);
+            const float d = alpha[e] * (g - q.w) * (t >= 0.f ? 1.f : slope);
             dt[e] = d;
             acc += d;
         }
@@ -1414,9 +1439,12 @@ __global__ void k_class_hist(const int32_t *__restrict__ out_deg, int64_t n,
 // TLP_HOT=<fraction> overrides the budget (0 disables).  *thr = (lowest hot
 // class) << 27, or 0 when disabled / not applicable.
 constexpr double kHotFrac = 0.5;
-static tlp_status hot_threshold(tlp_graph g, int64_t ldx, cudaStream_t s, unsigned *thr) {
+static tlp_status hot_threshold(tlp_graph g, int64_t ldx, bool panel, cudaStream_t s,
+                                unsigned *thr) {
     *thr = 0;
     const char *e = getenv("TLP_HOT");
+    // by default not in panel mode: there the whole strip of X is meant to stay in L2
+    if (!e && panel) return TLP_OK;
     const double frac = e ? atof(e) : kHotFrac;
     if (frac <= 0.0 || g->n_src >= (int64_t(1) << 27) || g->nnz == 0) return TLP_OK;
     const double row = (double)((4 * ldx + 31) / 32 * 32 + 16);
@@ -1477,7 +1505,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown activation");
     if (r.op < OP_GCN || r.op > OP_GATB)
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown op");
-    if (r.op == OP_GATB && (!r.el || !r.xself || !r.vstat || r.ldxs < r.F || !r.gbuf_out))
+    if (r.op == OP_GATB && (!r.alpha || !r.xself || r.ldxs < r.F || !r.gbuf_out))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "GAT backward arguments");
     if (r.op == OP_GATH && (r.heads < 1 || r.F % r.heads != 0))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "multi-head GAT needs F = heads * head_dim");
@@ -1522,8 +1550,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     } else if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) {
         if (g->ew_both) { ew = g->ew_both; coef |= COEF_W; }
         else { coef |= COEF_COUT; if (g->ew) coef |= COEF_W; }
-    } else if (r.op != OP_GAT && g->ew) {
+    } else if (r.op != OP_GAT && r.op != OP_GATB && g->ew) {
         coef |= COEF_W;
+    }
+    if (r.op == OP_GATB) {  // the edge softmax weights, in transposed edge order
+        ew = r.alpha;
+        coef = COEF_W;
     }
 
     // Feature panels: when X is much larger than
@@ -1602,20 +1634,8 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.n_dests = r.n_dests;
     a.hot_thr = 0;
     a.cold_first = 0;
-    if (r.op != OP_GATH) {
-        unsigned thr = 0;
-        tlp_status st = hot_threshold(g, panel ? (int64_t)strip_w : r.ldx, s, &thr);
-        if (st != TLP_OK) return st;
-        if (thr) {
-            a.colidx = g->colidx_tag;
-            a.hot_thr = thr;
-            a.cold_first = 1;
-            if (const char *e = getenv("TLP_HOT_COLD")) a.cold_first = atoi(e);
-        }
-    }
     a.xself = r.xself;
     a.ldxs = r.ldxs;
-    a.vstat = reinterpret_cast<const float4 *>(r.vstat);
     a.gbuf = nullptr;
     a.gstride = g->nnz;
     if (r.op == OP_GATB) {
@@ -1700,6 +1720,18 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     }
     if (pair || r.op == OP_GATB) async_path = false;  // OP_GATB: register path only
     const int path = pair ? 2 : (async_path ? 1 : 0);
+    // hot-source L2 policy: cp.async path only (rows streamed from HBM)
+    if (async_path && r.op != OP_GATH && r.op != OP_GATB) {
+        unsigned thr = 0;
+        tlp_status st = hot_threshold(g, panel ? (int64_t)strip_w : r.ldx, panel != 0, s, &thr);
+        if (st != TLP_OK) return st;
+        if (thr) {
+            a.colidx = g->colidx_tag;
+            a.hot_thr = thr;
+            a.cold_first = 1;
+            if (const char *e = getenv("TLP_HOT_COLD")) a.cold_first = atoi(e);
+        }
+    }
     KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, r.op, coef);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
@@ -1802,9 +1834,10 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
         if (n_dst) TLP_CUDA_TRY(cudaMemsetAsync(der, 0, sizeof(float) * n_dst, s));
         return TLP_OK;
     }
-    // forward-graph scratch: vstat [n_dst] float4, then dt [nnz]
+    // forward-graph scratch: vstat [n_dst] float4, then dt [nnz], alpha [nnz]
     const size_t vbytes = ((size_t)n_dst * 16 + 255) / 256 * 256;
-    const size_t need = vbytes + sizeof(float) * ((size_t)nnz + 16);
+    const size_t ebytes = (sizeof(float) * (size_t)nnz + 255) / 256 * 256;
+    const size_t need = vbytes + 2 * ebytes + 64;
     if (need > g->bwd_bytes) {
         if (g->bwd) {
             cudaFreeAsync(g->bwd, s);
@@ -1819,6 +1852,7 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
     }
     float4 *vstat = reinterpret_cast<float4 *>(g->bwd);
     float *dt = reinterpret_cast<float *>((char *)g->bwd + vbytes);
+    float *alpha = reinterpret_cast<float *>((char *)g->bwd + vbytes + ebytes);
     const int nsm = g->num_sms > 0 ? g->num_sms : 148;
     if (n_dst) {
         k_gatb_stats<<<nsm * 8, 256, 0, s>>>(g->rowptr, g->colidx, n_dst, el, er, slope, dY, lddy, Y,
@@ -1829,19 +1863,21 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
         if (n_dst) TLP_CUDA_TRY(cudaMemsetAsync(der, 0, sizeof(float) * n_dst, s));
         return TLP_OK;
     }
+    k_gatb_alpha<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, slope, alpha);
+    TLP_CUDA_TRY(cudaGetLastError());
     AggRequest r;
     r.op = OP_GATB;
     r.X = dY; r.F = F; r.ldx = lddy; r.Y = dX; r.ldy = lddx;
-    r.el = el; r.slope = slope;
-    r.xself = X; r.ldxs = ldx; r.vstat = vstat;
+    r.alpha = alpha;
+    r.xself = X; r.ldxs = ldx;
     float *gbuf = nullptr;
     int n_strips = 0;
     r.gbuf_out = &gbuf;
     r.n_strips_out = &n_strips;
     tlp_status st = aggregate(g->t, r, s);
     if (st != TLP_OK) return st;
-    k_gatb_edges<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, slope, gbuf,
-                                         n_strips, nnz, dt, del);
+    k_gatb_edges<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, alpha, slope,
+                                         gbuf, n_strips, nnz, dt, del);
     TLP_CUDA_TRY(cudaGetLastError());
     if (n_dst) {
         k_gatb_der<<<nsm * 8, 256, 0, s>>>(g->rowptr, n_dst, g->tpos, dt, der);

@@ -199,9 +199,16 @@ static int grid_for(int64_t n, int num_sms) {
 }
 
 namespace {
+// Temporary device buffer: stream-ordered allocation from the device's default
+// memory pool, freed stream-ordered (no implicit device synchronisation).
 struct DevBuf {
     void *p = nullptr;
-    ~DevBuf() { if (p) cudaFree(p); }
+    cudaStream_t st = nullptr;
+    cudaError_t alloc(size_t n, cudaStream_t s) {
+        st = s;
+        return cudaMallocAsync(&p, n ? n : 16, s);
+    }
+    ~DevBuf() { if (p) cudaFreeAsync(p, st); }
     template <class T> T *as() { return static_cast<T *>(p); }
 };
 }  // namespace
@@ -312,12 +319,12 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         if (e != cudaSuccess) cudaGetLastError();
         const int64_t *rp_dev = rowptr;
         if (!on_dev) {
-            CTRY(cudaMalloc(&rp_src.p, sizeof(int64_t) * (n_dst + 1)));
+            CTRY(rp_src.alloc(sizeof(int64_t) * (n_dst + 1), s));
             CTRY(cudaMemcpyAsync(rp_src.p, rowptr, sizeof(int64_t) * (n_dst + 1),
                                  cudaMemcpyDefault, s));
             rp_dev = rp_src.as<int64_t>();
         }
-        CTRY(cudaMalloc(&err.p, sizeof(int)));
+        CTRY(err.alloc(sizeof(int), s));
         CTRY(cudaMemsetAsync(err.p, 0, sizeof(int), s));
         // rowptr[0] must be the start of the slice: for a whole graph it must be 0
         int64_t first = 0;
@@ -375,10 +382,10 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
     if (n_dst > 0) {
         DevBuf start, hub, starts, nsel, temp, utasks, keep, rtasks, hub_rows_u, hub_deg_u,
             hub_deg_s, nchunk;
-        CTRY(cudaMalloc(&start.p, n_dst));
-        CTRY(cudaMalloc(&hub.p, n_dst));
-        CTRY(cudaMalloc(&starts.p, sizeof(int32_t) * n_dst));
-        CTRY(cudaMalloc(&nsel.p, sizeof(int64_t) * 4));
+        CTRY(start.alloc(n_dst, s));
+        CTRY(hub.alloc(n_dst, s));
+        CTRY(starts.alloc(sizeof(int32_t) * n_dst, s));
+        CTRY(nsel.alloc(sizeof(int64_t) * 4, s));
         k_plan_flags<<<grid_for(n_dst, nsm), 256, 0, s>>>(g->rowptr, n_dst, g->K, g->H,
                                                           start.as<uint8_t>(), hub.as<uint8_t>());
         CTRY(cudaGetLastError());
@@ -390,16 +397,16 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         CTRY(cub::DeviceSelect::Flagged(nullptr, tb2, rows, hub.as<uint8_t>(),
                                         starts.as<int32_t>(), nsel.as<int64_t>(), (int)n_dst, s));
         if (tb2 > tb) tb = tb2;
-        CTRY(cudaMalloc(&temp.p, tb));
+        CTRY(temp.alloc(tb, s));
         CTRY(cub::DeviceSelect::Flagged(temp.p, tb, rows, start.as<uint8_t>(),
                                         starts.as<int32_t>(), nsel.as<int64_t>(), (int)n_dst, s));
         int64_t h_n_units = 0;
         CTRY(cudaMemcpyAsync(&h_n_units, nsel.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         CTRY(cudaStreamSynchronize(s));
 
-        CTRY(cudaMalloc(&utasks.p, sizeof(int2) * h_n_units));
-        CTRY(cudaMalloc(&keep.p, h_n_units));
-        CTRY(cudaMalloc(&rtasks.p, sizeof(int2) * h_n_units));
+        CTRY(utasks.alloc(sizeof(int2) * h_n_units, s));
+        CTRY(keep.alloc(h_n_units, s));
+        CTRY(rtasks.alloc(sizeof(int2) * h_n_units, s));
         k_units_to_tasks<<<grid_for(h_n_units, nsm), 256, 0, s>>>(
             starts.as<int32_t>(), h_n_units, n_dst, hub.as<uint8_t>(), utasks.as<int2>(),
             keep.as<uint8_t>());
@@ -408,15 +415,15 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         CTRY(cub::DeviceSelect::Flagged(nullptr, tb3, utasks.as<int2>(), keep.as<uint8_t>(),
                                         rtasks.as<int2>(), nsel.as<int64_t>() + 1, (int)h_n_units, s));
         if (tb3 > tb) {
-            cudaFree(temp.p);
+            cudaFreeAsync(temp.p, s);
             temp.p = nullptr;
-            CTRY(cudaMalloc(&temp.p, tb3));
+            CTRY(temp.alloc(tb3, s));
             tb = tb3;
         }
         CTRY(cub::DeviceSelect::Flagged(temp.p, tb, utasks.as<int2>(), keep.as<uint8_t>(),
                                         rtasks.as<int2>(), nsel.as<int64_t>() + 1, (int)h_n_units, s));
         // hubs in row order, then sorted by descending degree (stable => ties by row)
-        CTRY(cudaMalloc(&hub_rows_u.p, sizeof(int32_t) * n_dst));
+        CTRY(hub_rows_u.alloc(sizeof(int32_t) * n_dst, s));
         CTRY(cub::DeviceSelect::Flagged(temp.p, tb, rows, hub.as<uint8_t>(),
                                         hub_rows_u.as<int32_t>(), nsel.as<int64_t>() + 2,
                                         (int)n_dst, s));
@@ -431,9 +438,9 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         CTRY(cudaMemsetAsync(g->hub_off, 0, sizeof(int32_t) * (n_hubs + 1), s));
         int64_t n_chunks = 0;
         if (n_hubs > 0) {
-            CTRY(cudaMalloc(&hub_deg_u.p, sizeof(int32_t) * n_hubs));
-            CTRY(cudaMalloc(&hub_deg_s.p, sizeof(int32_t) * n_hubs));
-            CTRY(cudaMalloc(&nchunk.p, sizeof(int32_t) * (n_hubs + 1)));
+            CTRY(hub_deg_u.alloc(sizeof(int32_t) * n_hubs, s));
+            CTRY(hub_deg_s.alloc(sizeof(int32_t) * n_hubs, s));
+            CTRY(nchunk.alloc(sizeof(int32_t) * (n_hubs + 1), s));
             k_gather_deg<<<grid_for(n_hubs, nsm), 256, 0, s>>>(hub_rows_u.as<int32_t>(), n_hubs,
                                                                g->in_deg, hub_deg_u.as<int32_t>());
             CTRY(cudaGetLastError());
@@ -442,7 +449,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
             CTRY(cub::DeviceRadixSort::SortPairsDescending(
                 nullptr, b2, hub_deg_u.as<int32_t>(), hub_deg_s.as<int32_t>(),
                 hub_rows_u.as<int32_t>(), g->hub_row, (int)n_hubs, 0, 32, s));
-            CTRY(cudaMalloc(&t2.p, b2));
+            CTRY(t2.alloc(b2, s));
             CTRY(cub::DeviceRadixSort::SortPairsDescending(
                 t2.p, b2, hub_deg_u.as<int32_t>(), hub_deg_s.as<int32_t>(),
                 hub_rows_u.as<int32_t>(), g->hub_row, (int)n_hubs, 0, 32, s));
@@ -454,7 +461,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
             size_t b3 = 0;
             CTRY(cub::DeviceScan::ExclusiveSum(nullptr, b3, nchunk.as<int32_t>(), g->hub_off,
                                                (int)(n_hubs + 1), s));
-            CTRY(cudaMalloc(&t3.p, b3));
+            CTRY(t3.alloc(b3, s));
             CTRY(cub::DeviceScan::ExclusiveSum(t3.p, b3, nchunk.as<int32_t>(), g->hub_off,
                                                (int)(n_hubs + 1), s));
             int32_t hc = 0;
@@ -480,9 +487,9 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
             // max in-degree over regular rows (<= H): one reduction
             DevBuf mx, t4;
             size_t b4 = 0;
-            CTRY(cudaMalloc(&mx.p, sizeof(int32_t)));
+            CTRY(mx.alloc(sizeof(int32_t), s));
             CTRY(cub::DeviceReduce::Max(nullptr, b4, g->in_deg, mx.as<int32_t>(), (int)n_dst, s));
-            CTRY(cudaMalloc(&t4.p, b4));
+            CTRY(t4.alloc(b4, s));
             CTRY(cub::DeviceReduce::Max(t4.p, b4, g->in_deg, mx.as<int32_t>(), (int)n_dst, s));
             int32_t m = 0;
             CTRY(cudaMemcpyAsync(&m, mx.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
@@ -516,18 +523,18 @@ tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
         return set_error(TLP_ERR_UNSUPPORTED, "transpose needs nnz < 2^31");
     const int nsm = g->num_sms;
     DevBuf dst, keys_out, iota, perm, t_col, t_ew, t_rp, deg64, temp;
-    TLP_CUDA_TRY(cudaMalloc(&dst.p, sizeof(int32_t) * nnz + 16));
-    TLP_CUDA_TRY(cudaMalloc(&keys_out.p, sizeof(int32_t) * nnz + 16));
-    TLP_CUDA_TRY(cudaMalloc(&iota.p, sizeof(int32_t) * nnz + 16));
-    TLP_CUDA_TRY(cudaMalloc(&perm.p, sizeof(int32_t) * nnz + 16));
-    TLP_CUDA_TRY(cudaMalloc(&t_col.p, sizeof(int32_t) * nnz + 16));
-    if (g->ew) TLP_CUDA_TRY(cudaMalloc(&t_ew.p, sizeof(float) * nnz + 16));
+    TLP_CUDA_TRY(dst.alloc(sizeof(int32_t) * nnz + 16, s));
+    TLP_CUDA_TRY(keys_out.alloc(sizeof(int32_t) * nnz + 16, s));
+    TLP_CUDA_TRY(iota.alloc(sizeof(int32_t) * nnz + 16, s));
+    TLP_CUDA_TRY(perm.alloc(sizeof(int32_t) * nnz + 16, s));
+    TLP_CUDA_TRY(t_col.alloc(sizeof(int32_t) * nnz + 16, s));
+    if (g->ew) TLP_CUDA_TRY(t_ew.alloc(sizeof(float) * nnz + 16, s));
     if (!g->tpos) {
         TLP_CUDA_TRY(cudaMalloc(&g->tpos, sizeof(int32_t) * nnz + 16));
         g->device_bytes += sizeof(int32_t) * nnz + 16;
     }
-    TLP_CUDA_TRY(cudaMalloc(&t_rp.p, sizeof(int64_t) * (n_src + 1)));
-    TLP_CUDA_TRY(cudaMalloc(&deg64.p, sizeof(int64_t) * (n_src + 1)));
+    TLP_CUDA_TRY(t_rp.alloc(sizeof(int64_t) * (n_src + 1), s));
+    TLP_CUDA_TRY(deg64.alloc(sizeof(int64_t) * (n_src + 1), s));
     if (n_dst) {
         k_edge_rows<<<grid_for(n_dst, nsm), 256, 0, s>>>(g->rowptr, n_dst, dst.as<int32_t>());
         TLP_CUDA_TRY(cudaGetLastError());
@@ -539,7 +546,7 @@ tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
         TLP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, tb2, g->colidx, keys_out.as<int32_t>(),
                                                      iota.as<int32_t>(), perm.as<int32_t>(), (int)nnz,
                                                      0, 32, s));
-        TLP_CUDA_TRY(cudaMalloc(&temp.p, tb2));
+        TLP_CUDA_TRY(temp.alloc(tb2, s));
         TLP_CUDA_TRY(cub::DeviceRadixSort::SortPairs(temp.p, tb2, g->colidx, keys_out.as<int32_t>(),
                                                      iota.as<int32_t>(), perm.as<int32_t>(), (int)nnz,
                                                      0, 32, s));
@@ -556,7 +563,7 @@ tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
         size_t b3 = 0;
         TLP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, b3, deg64.as<int64_t>(), t_rp.as<int64_t>(),
                                                    (int)(n_src + 1), s));
-        TLP_CUDA_TRY(cudaMalloc(&t3.p, b3));
+        TLP_CUDA_TRY(t3.alloc(b3, s));
         TLP_CUDA_TRY(cub::DeviceScan::ExclusiveSum(t3.p, b3, deg64.as<int64_t>(), t_rp.as<int64_t>(),
                                                    (int)(n_src + 1), s));
     }

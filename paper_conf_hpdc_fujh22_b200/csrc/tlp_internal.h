@@ -118,12 +118,12 @@ struct AggRequest {
     float *const *dests = nullptr;  // fused all-gather destinations (device array)
     int n_dests = 0;
     // op 5 (GAT backward on the transposed graph, NEXT-4): X = dY, Y = dX,
-    // el = forward el (per transposed row), xself = forward X, vstat = per
-    // forward-destination {er, m, 1/z, <dY,Y>}; aggregate() allocates the
-    // per-strip edge dot products gbuf [n_strips x nnz] and reports them.
+    // alpha = edge softmax weights in transposed edge order, xself = forward X;
+    // aggregate() allocates the per-strip edge dot products gbuf
+    // [n_strips x nnz] and reports them.
+    const float *alpha = nullptr;
     const float *xself = nullptr;
     int64_t ldxs = 0;
-    const void *vstat = nullptr;
     float **gbuf_out = nullptr;
     int *n_strips_out = nullptr;
 };
