@@ -119,6 +119,14 @@ typedef struct tlp_agg_desc {
     const float *bias;        /* epilogue: fp32 device [F] or NULL             */
     int act;                  /* epilogue: tlp_act                             */
     float act_param;          /* LeakyReLU slope / ELU alpha                   */
+    /* epilogue projections (NEXT-3, single head, single GPU): after bias and
+     * activation, el_out[v] = sum_f Y[v,f] att_l[f] and er_out[v] =
+     * sum_f Y[v,f] att_r[f] -- the next GAT layer's attention terms, formed
+     * while the row is still in registers (per-strip partials reduced in strip
+     * order by one extra launch: deterministic).  att_*: fp32 device [F] or
+     * NULL; *_out: fp32 device [n_dst] or NULL (set both of a pair). */
+    const float *att_l, *att_r;
+    float *el_out, *er_out;
 } tlp_agg_desc;
 
 typedef struct tlp_graph_s *tlp_graph;

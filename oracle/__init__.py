@@ -80,6 +80,8 @@ def _load():
         lib.oracle_gat_backward.argtypes = [I64, I64, P, P, P, I64, P, P, ctypes.c_double, P,
                                             I64, I64, P, P, P, P, P, P]
         lib.oracle_gat_backward.restype = ctypes.c_int
+        lib.oracle_project.argtypes = [I64, I64, P, I64, P, P, P]
+        lib.oracle_project.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -286,6 +288,18 @@ def gat_backward(rowptr, colidx, X, el, er, slope, dY, F=None):
     if rc:
         raise ValueError("oracle_gat_backward: bad arguments")
     return (dX, AdX), (dl, Adl), (dr, Adr)
+
+
+def project(Y, a, F=None):
+    """el[v] = sum_f Y[v,f] a[f] for an fp32 layer output Y.  Returns (el, A)."""
+    Y = _feat(Y)
+    F = Y.shape[1] if F is None else F
+    a = np.ascontiguousarray(a, dtype=np.float32)
+    out = np.empty(Y.shape[0]); A = np.empty(Y.shape[0])
+    rc = _load().oracle_project(Y.shape[0], F, _ptr(Y), Y.strides[0] // 4, _ptr(a), _ptr(out), _ptr(A))
+    if rc:
+        raise ValueError("oracle_project: bad arguments")
+    return out, A
 
 
 ACTS = {"none": 0, "relu": 1, "leaky_relu": 2, "elu": 3}

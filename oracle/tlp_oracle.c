@@ -565,3 +565,27 @@ int oracle_gat_backward(int64_t n_dst, int64_t n_src, const int64_t *rowptr,
     }
     return 0;
 }
+
+/* NEXT-3: the next GAT layer's attention terms of a layer output (after the
+ * epilogue), el[v] = sum_f Y[v,f] a[f]  (Velickovic [43]: a^T [W h_i || W h_j]
+ * splits into a per-source and a per-destination dot product).
+ * Y is fp32 [n_rows x ldy] (the previous stage's output, reading R22);
+ * out, A: [n_rows] (A = sum |terms|). */
+int oracle_project(int64_t n_rows, int64_t F, const float *Y, int64_t ldy,
+                   const float *a, double *out, double *A)
+{
+    if (F < 0 || ldy < F)
+        return -1;
+    for (int64_t v = 0; v < n_rows; ++v) {
+        double s = 0.0, b = 0.0;
+        for (int64_t f = 0; f < F; ++f) {
+            double t = (double)Y[v * ldy + f] * (double)a[f];
+            s += t;
+            b += fabs(t);
+        }
+        out[v] = s;
+        if (A)
+            A[v] = b;
+    }
+    return 0;
+}

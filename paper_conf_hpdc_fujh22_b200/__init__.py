@@ -57,7 +57,8 @@ class tlp_agg_desc(ctypes.Structure):
                 ("norm", ctypes.c_int), ("eps", ctypes.c_float), ("el", ctypes.c_void_p),
                 ("er", ctypes.c_void_p), ("slope", ctypes.c_float), ("heads", ctypes.c_int64),
                 ("include_self", ctypes.c_int), ("bias", ctypes.c_void_p), ("act", ctypes.c_int),
-                ("act_param", ctypes.c_float)]
+                ("act_param", ctypes.c_float), ("att_l", ctypes.c_void_p), ("att_r", ctypes.c_void_p),
+                ("el_out", ctypes.c_void_p), ("er_out", ctypes.c_void_p)]
 
 
 OPS = {"gcn": 0, "gin": 1, "gat": 2, "sage": 3, "gat_mh": 4}
@@ -333,7 +334,8 @@ def tlp_gat_aggregate(g, X, el, er, slope=0.2, Y=None, F=None, stream=None, n_ds
 
 
 def _desc(op, X, Y, F, ldx, ldy, norm="both", eps=0.0, el=None, er=None, slope=0.2, heads=1,
-          include_self=False, bias=None, act="none", act_param=0.0):
+          include_self=False, bias=None, act="none", act_param=0.0, att_l=None, att_r=None,
+          el_out=None, er_out=None):
     d = tlp_agg_desc()
     d.op = OPS[op] if isinstance(op, str) else int(op)
     d.X, d.F, d.ldx, d.Y, d.ldy = _ptr(X), int(F), int(ldx), _ptr(Y), int(ldy)
@@ -345,18 +347,28 @@ def _desc(op, X, Y, F, ldx, ldy, norm="both", eps=0.0, el=None, er=None, slope=0
     d.bias = _ptr(None if bias is None else _vec_cuda(bias, "bias"))
     d.act = ACTS[act] if isinstance(act, str) else int(act)
     d.act_param = float(act_param)
+    d.att_l = _ptr(None if att_l is None else _vec_cuda(att_l, "att_l"))
+    d.att_r = _ptr(None if att_r is None else _vec_cuda(att_r, "att_r"))
+    d.el_out = _ptr(None if el_out is None else _vec_cuda(el_out, "el_out"))
+    d.er_out = _ptr(None if er_out is None else _vec_cuda(er_out, "er_out"))
     return d
 
 
 def tlp_aggregate(g, op, X, Y=None, F=None, stream=None, n_dst=None, **kw):
     """Descriptor API: op in {gcn, gin, gat, sage, gat_mh}; keyword arguments of
     tlp_agg_desc (norm, eps, el, er, slope, heads, include_self) plus the fused
-    layer epilogue bias=[F] tensor, act in {none, relu, leaky_relu, elu}, act_param."""
+    layer epilogue bias=[F] tensor, act in {none, relu, leaky_relu, elu}, act_param,
+    and the next layer's attention projections att_l / att_r ([F]) written to
+    el_out / er_out ([n_dst] float32 CUDA tensors, contiguous)."""
     X, F, ldx = _feat(X, F)
     n = _n_dst(g) if n_dst is None else n_dst
     Y, F, ldy = _out(Y, n, F, X)
-    keep = [kw.get(k) for k in ("el", "er", "bias")]  # keep contiguous copies alive
-    for k in ("el", "er", "bias"):
+    for k in ("el_out", "er_out"):
+        o = kw.get(k)
+        if o is not None and (not o.is_contiguous() or o.numel() != n):
+            raise ValueError(f"{k} must be a contiguous float32 CUDA tensor of n_dst elements")
+    keep = [kw.get(k) for k in ("el", "er", "bias", "att_l", "att_r")]  # keep copies alive
+    for k in ("el", "er", "bias", "att_l", "att_r"):
         if kw.get(k) is not None:
             kw[k] = _vec_cuda(kw[k], k)
     d = _desc(op, X, Y, F, ldx, ldy, **kw)

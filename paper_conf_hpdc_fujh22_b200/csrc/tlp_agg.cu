@@ -107,6 +107,12 @@ struct AggArgs {
     // dY[v_e] . X[u] (transposed edge e).
     const float *xself;
     int64_t ldxs;
+    // NEXT-3 epilogue projections: per strip s and local row r, the strip's
+    // partial dots proj[(s * n_dst + r) * 2 + {0,1}] of the finished output
+    // row with att_l / att_r (NULL proj: off)
+    const float *att_l, *att_r;
+    float *proj;
+    int64_t n_dst;
     float *gbuf;
     int64_t gstride;
 };
@@ -989,6 +995,32 @@ __device__ __forceinline__ bool stores(int lane) {
     return !PAIR || lane < 16;
 }
 
+// NEXT-3: the strip's partial dots of a finished row vector with att_l, att_r
+// (per-lane fma over the vector, butterfly over the warp; lane 0 stores).
+template <int VEC, bool PAIR>
+__device__ __forceinline__ void project_row(const AggArgs &a, int64_t r, int s, int col, bool active,
+                                            const Vec<VEC> &y, int lane) {
+    if (a.proj == nullptr) return;
+    float pl = 0.f, pr = 0.f;
+    if (active && stores<PAIR>(lane)) {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) {
+            if (col + c < a.F) {
+                if (a.att_l) pl = fmaf(y.v[c], __ldg(a.att_l + col + c), pl);
+                if (a.att_r) pr = fmaf(y.v[c], __ldg(a.att_r + col + c), pr);
+            }
+        }
+    }
+    pl = warp_sum(pl);
+    pr = warp_sum(pr);
+    if (lane == 0) {
+        float *p = a.proj + ((int64_t)s * a.n_dst + r) * 2;
+        p[0] = pl;
+        p[1] = pr;
+    }
+}
+
+
 // OP_GATB: the transposed row's own forward features X[u] for this lane's
 // columns of strip s, and where the strip's edge dot products go.
 template <int VEC, int OP>
@@ -1056,6 +1088,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                 }
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
                 if (active && stores<PAIR>(lane)) store_out<VEC>(a, r, col, y);
+                project_row<VEC, PAIR>(a, r, s, col, active, y, lane);
             }
         }
     }
@@ -1186,6 +1219,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
             y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
         }
         if (active && stores<PAIR>(lane)) store_out<VEC>(a, r, col, y);
+        if constexpr (OP != OP_GATH) project_row<VEC, PAIR>(a, r, s, col, active, y, lane);
     }
     if (lane == 0) *ticket = 0;  // self-reset for the next launch
 }
@@ -1309,6 +1343,23 @@ static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
 }
 
 static bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+// NEXT-3: el_out[v] / er_out[v] = sum over strips (in strip order) of the
+// epilogue's partial dots.
+__global__ void k_proj_sum(const float *__restrict__ proj, int n_strips, int64_t n_dst,
+                           float *__restrict__ el_out, float *__restrict__ er_out) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n_dst;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        float l = 0.f, rr = 0.f;
+        for (int k = 0; k < n_strips; ++k) {
+            const float2 p = *reinterpret_cast<const float2 *>(proj + ((int64_t)k * n_dst + v) * 2);
+            l += p.x;
+            rr += p.y;
+        }
+        if (el_out) el_out[v] = l;
+        if (er_out) er_out[v] = rr;
+    }
+}
 
 // ---- GAT backward (NEXT-4) scalar passes -------------------------------------
 // The passes around the OP_GATB aggregation:
@@ -1505,6 +1556,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown activation");
     if (r.op < OP_GCN || r.op > OP_GATB)
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown op");
+    const bool want_proj = r.el_out || r.er_out;
+    if ((r.el_out && !r.att_l) || (r.er_out && !r.att_r) || ((r.att_l || r.att_r) && !want_proj))
+        return set_error(TLP_ERR_INVALID_ARGUMENT, "epilogue projection needs att_* with *_out");
+    if (want_proj && (r.op == OP_GATH || r.op == OP_GATB || r.n_dests > 0))
+        return set_error(TLP_ERR_UNSUPPORTED,
+                         "epilogue projections: single-head ops, single-GPU output only");
     if (r.op == OP_GATB && (!r.alpha || !r.xself || r.ldxs < r.F || !r.gbuf_out))
         return set_error(TLP_ERR_INVALID_ARGUMENT, "GAT backward arguments");
     if (r.op == OP_GATH && (r.heads < 1 || r.F % r.heads != 0))
@@ -1636,6 +1693,26 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.cold_first = 0;
     a.xself = r.xself;
     a.ldxs = r.ldxs;
+    a.att_l = r.att_l;
+    a.att_r = r.att_r;
+    a.proj = nullptr;
+    a.n_dst = g->n_dst;
+    if (want_proj) {
+        const size_t need = sizeof(float) * 2 * (size_t)n_strips * (size_t)g->n_dst + 64;
+        if (need > g->proj_bytes) {
+            if (g->proj) {
+                cudaFreeAsync(g->proj, s);
+                g->device_bytes -= g->proj_bytes;
+                g->proj = nullptr;
+                g->proj_bytes = 0;
+            }
+            cudaError_t e = cudaMallocAsync((void **)&g->proj, need, s);
+            if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(projections)");
+            g->proj_bytes = need;
+            g->device_bytes += need;
+        }
+        a.proj = g->proj;
+    }
     a.gbuf = nullptr;
     a.gstride = g->nnz;
     if (r.op == OP_GATB) {
@@ -1752,6 +1829,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     fn<<<(unsigned)blocks, threads, smem, s>>>(a);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_agg launch");
+    if (want_proj) {
+        const int pb = (int)std::min<int64_t>((g->n_dst + 255) / 256, (int64_t)g->num_sms * 8);
+        k_proj_sum<<<pb, 256, 0, s>>>(g->proj, n_strips, g->n_dst, r.el_out, r.er_out);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "k_proj_sum launch");
+    }
     g->last_stream = s;
     return TLP_OK;
 }

@@ -326,6 +326,8 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph g, tlp_comm c, const float *X_full, 
 
 tlp_status tlp_dist_aggregate(tlp_graph g, tlp_comm c, const tlp_agg_desc *d, void *stream) {
     if (!d) return set_error(TLP_ERR_INVALID_ARGUMENT, "null descriptor");
+    if (d->el_out || d->er_out || d->att_l || d->att_r)
+        return set_error(TLP_ERR_UNSUPPORTED, "epilogue projections are single-GPU only");
     AggRequest r = request_from_desc(*d);
     return dist_local(g, c, r, stream);
 }
@@ -336,6 +338,8 @@ tlp_status tlp_dist_aggregate(tlp_graph g, tlp_comm c, const tlp_agg_desc *d, vo
 // NCCL all-reduce then orders the stream after every rank's kernel.
 tlp_status tlp_dist_aggregate_fused(tlp_graph g, tlp_comm c, const tlp_agg_desc *d, void *stream) {
     if (!g || !c || !d || !g->bounds_host) return set_error(TLP_ERR_INVALID_ARGUMENT, "not a dist graph");
+    if (d->el_out || d->er_out || d->att_l || d->att_r)
+        return set_error(TLP_ERR_UNSUPPORTED, "epilogue projections are single-GPU only");
     if (c->world != g->world || c->rank != g->rank)
         return set_error(TLP_ERR_INVALID_ARGUMENT, "communicator does not match the graph");
     const SymBuf *b = nullptr;

@@ -225,7 +225,7 @@ static void graph_free(tlp_graph g) {
     if (!g) return;
     if (g->t) graph_free(g->t);
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
-                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd,
+                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd, g->proj,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)

@@ -53,6 +53,8 @@ struct tlp_graph_s {
     int32_t *tpos = nullptr;         // [nnz] forward edge -> transposed position (with t)
     float *bwd = nullptr;            // GAT backward scratch (see tlp_gat_backward)
     size_t bwd_bytes = 0;
+    float *proj = nullptr;           // epilogue projection partials [strips x n_dst x 2]
+    size_t proj_bytes = 0;
     int64_t tag_hist[32] = {0};      // sources per out-degree class
 
     int2 *tasks = nullptr;       // [n_tasks]
@@ -117,6 +119,9 @@ struct AggRequest {
     float act_param = 0.f;
     float *const *dests = nullptr;  // fused all-gather destinations (device array)
     int n_dests = 0;
+    // epilogue projections (NEXT-3): el_out = Y.att_l, er_out = Y.att_r
+    const float *att_l = nullptr, *att_r = nullptr;
+    float *el_out = nullptr, *er_out = nullptr;
     // op 5 (GAT backward on the transposed graph, NEXT-4): X = dY, Y = dX,
     // alpha = edge softmax weights in transposed edge order, xself = forward X;
     // aggregate() allocates the per-strip edge dot products gbuf
@@ -136,6 +141,7 @@ inline AggRequest request_from_desc(const tlp_agg_desc &d) {
     r.el = d.el; r.er = d.er; r.slope = d.slope; r.heads = d.heads > 0 ? d.heads : 1;
     r.sage_self = d.include_self;
     r.bias = d.bias; r.act = d.act; r.act_param = d.act_param;
+    r.att_l = d.att_l; r.att_r = d.att_r; r.el_out = d.el_out; r.er_out = d.er_out;
     return r;
 }
 tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s);

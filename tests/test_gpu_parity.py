@@ -905,3 +905,50 @@ def test_hot_source_policy_is_bitwise_neutral(tlp, monkeypatch, op):
         torch.cuda.synchronize()
         g.close()
     assert torch.equal(out[0], out[1])
+
+
+# ----------------------------------------------- NEXT-3: epilogue projections ----
+
+@pytest.mark.parametrize("op", ["gcn", "gin", "gat", "sage"])
+@pytest.mark.parametrize("panel", ["auto", "64", "0"])
+def test_epilogue_projections(tlp, monkeypatch, op, panel):
+    """el_out = act(Y + b).att_l, er_out = ... .att_r, fused into the store:
+    each against the oracle's projection of the GPU's own fp32 output (R22), in
+    every strip mode (partials summed in strip order: deterministic)."""
+    if panel != "auto":
+        monkeypatch.setenv("TLP_PANEL", panel)
+    rp, ci, n = _edge_graphs()["powerlaw_hubs"]
+    F = 200
+    X = _t(synth.features(n, F, F, seed=21))
+    el, er = _t(synth.normal(n, 22)), _t(synth.normal(n, 23))
+    bias = _t(synth.normal(F, 24))
+    al, ar = _t(synth.normal(F, 25)), _t(synth.normal(F, 26))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    elo = torch.full((n,), float("nan"), device=DEV)
+    ero = torch.full((n,), float("nan"), device=DEV)
+    kw = dict(bias=bias, act="leaky_relu", act_param=0.2, att_l=al, att_r=ar, el_out=elo, er_out=ero)
+    if op == "gat":
+        kw.update(el=el, er=er)
+    if op == "sage":
+        kw.update(include_self=True)
+    Y = g.aggregate(op, X, **kw)
+    torch.cuda.synchronize()
+    Yh = Y.cpu().numpy()
+    _check(f"{op} el_out", elo.view(-1, 1), tuple(v.reshape(-1, 1) for v in oracle.project(Yh, al.cpu().numpy())))
+    _check(f"{op} er_out", ero.view(-1, 1), tuple(v.reshape(-1, 1) for v in oracle.project(Yh, ar.cpu().numpy())))
+    # the plain call (no projections) writes the same Y bit for bit
+    kw2 = {k: v for k, v in kw.items() if k not in ("att_l", "att_r", "el_out", "er_out")}
+    assert torch.equal(g.aggregate(op, X, **kw2), Y)
+    g.close()
+
+
+def test_epilogue_projection_argument_errors(tlp):
+    rp, ci, n = _edge_graphs()["random64"]
+    g = tlp.Graph(_t(rp), _t(ci))
+    X = _t(synth.features(n, 8, 8, seed=1))
+    out = torch.empty(n, device=DEV)
+    with pytest.raises(Exception):
+        g.aggregate("gcn", X, el_out=out)  # no att_l
+    with pytest.raises(Exception):
+        g.aggregate("gcn", X, att_l=_t(synth.normal(8, 2)))  # no el_out
+    g.close()

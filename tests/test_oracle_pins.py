@@ -643,3 +643,23 @@ def test_gat_backward_finite_differences():
         ep[v] += h
         em[v] -= h
         assert abs((loss(el, ep) - loss(el, em)) / (2 * h) - dr[v]) <= 1e-6 * (abs(dr[v]) + 1)
+
+
+# ------------------------------------------------- NEXT-3: epilogue projections --
+
+def test_project_closed_forms():
+    """Unit vector e_k picks column k exactly; ones give the row sum; the star's
+    GCN-NONE output [10, 3, 4, 5] (F = 1) times a = 0.5 is [5, 1.5, 2, 2.5]."""
+    Y = synth.features(50, 7, 9, seed=3)
+    for k in range(7):
+        e = np.zeros(7, np.float32)
+        e[k] = 1.0
+        out, A = oracle.project(Y, e, F=7)
+        np.testing.assert_array_equal(out, Y[:, k].astype(np.float64))
+        np.testing.assert_array_equal(A, np.abs(Y[:, k].astype(np.float64)))
+    out, _ = oracle.project(Y, np.ones(7, np.float32), F=7)
+    np.testing.assert_allclose(out, Y[:, :7].astype(np.float64).sum(1), rtol=1e-13)
+    rp, ci = synth.figure1_star(self_loops=True)
+    Ys, _ = oracle.gcn(rp, ci, np.array([[1.0], [2.0], [3.0], [4.0]], np.float32), "none")
+    out, _ = oracle.project(Ys.astype(np.float32), np.array([0.5], np.float32))
+    np.testing.assert_allclose(out, [5.0, 1.5, 2.0, 2.5], rtol=0, atol=0)
