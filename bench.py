@@ -71,6 +71,27 @@ def gather_bytes(op, n_rows, n_edges, F):
     raise ValueError(op)
 
 
+def l2_gather_peak():
+    """Measured L2-resident random-row gather bandwidth (256-byte rows, the
+    largest table that still fits L2 like a 64-column panel), or None."""
+    p = os.path.join(ROOT, "profiles", "l2_gather_probe.jsonl")
+    try:
+        rows, mhz = [], None
+        for line in open(p):
+            line = line.strip()
+            if line.startswith("{"):
+                rows.append(json.loads(line))
+            elif line.endswith("MHz"):
+                mhz = line.split()[0]
+        cands = [r for r in rows if r["row_bytes"] == 256 and r["table_MB"] < 80]
+        best = max(cands, key=lambda r: r["table_MB"] * 1e6 + r["GBs"])
+        best = max([r for r in cands if r["table_MB"] == best["table_MB"]], key=lambda r: r["GBs"])
+        best["sm_mhz"] = mhz
+        return best
+    except (OSError, ValueError, KeyError):
+        return None
+
+
 def peak_hbm():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -459,6 +480,15 @@ def run_tlp(args):
         roofline["traffic_frac_of_peak"] = round(roofline["traffic_GBs"] / peak, 4)
         roofline["note"] = ("frac > 1: feature panels keep the gathered slice of X in L2, so most of "
                             "the gather-model bytes are L2 hits; traffic_GBs is the HBM rate")
+    l2 = l2_gather_peak()
+    if l2:
+        # the ceiling that binds when the gathered rows are L2-resident (panel mode):
+        # random-row L2 gather bandwidth measured by scripts/l2_probe.cu on a B200
+        roofline["l2_gather"] = {"peak": l2["GBs"], "unit": "GB/s",
+                                 "frac": round(achieved / l2["GBs"], 4),
+                                 "source": "profiles/l2_gather_probe.jsonl (%d-byte rows, %.0f MB "
+                                           "table, sm clock at measurement %s)"
+                                           % (l2["row_bytes"], l2["table_MB"], l2.get("sm_mhz"))}
 
     result = {
         "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
