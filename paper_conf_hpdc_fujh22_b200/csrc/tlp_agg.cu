@@ -88,6 +88,7 @@ struct AggArgs {
     unsigned int *done;
     int64_t ldx, ldy, ldp, row_offset, n_tasks, n_items, n_hubs, n_chunks, C;
     int F, n_strips, norm, step, sched, panel;
+    int lps;  // lanes per strip (full-warp strips: lps * VEC columns, lps <= 32)
     float eps1, slope;
     int sage_self;  // OP_SAGE: include X[v] in the mean
     const float *bias;  // layer epilogue (NEXT-3): y = act(y + bias)
@@ -991,8 +992,14 @@ __device__ __forceinline__ void store_out(const AggArgs &a, int64_t r, int col, 
 // Column of this lane's 4-float vector in strip s (PAIR: 64-column strips,
 // lanes l and l+16 share a column), and whether this lane stores it.
 template <int VEC, bool PAIR>
-__device__ __forceinline__ int strip_col(int s, int lane) {
-    return PAIR ? s * 64 + (lane & 15) * 4 : s * 32 * VEC + lane * VEC;
+__device__ __forceinline__ int strip_col(const AggArgs &a, int s, int lane) {
+    return PAIR ? s * 64 + (lane & 15) * 4 : s * a.lps * VEC + lane * VEC;
+}
+// Whether this lane's column of the strip exists (narrow strips leave lanes
+// >= lps idle; they gather column 0 of the same row, a sector already fetched).
+template <bool PAIR>
+__device__ __forceinline__ bool in_strip(const AggArgs &a, int lane, int col) {
+    return (PAIR || lane < a.lps) && col < a.F;
 }
 template <bool PAIR>
 __device__ __forceinline__ bool stores(int lane) {
@@ -1057,8 +1064,8 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
             const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
             const int64_t r = rb + k;
             for (int s = s0; s < s1; ++s) {
-                const int col = strip_col<VEC, PAIR>(s, lane);
-                const bool active = col < a.F;
+                const int col = strip_col<VEC, PAIR>(a, s, lane);
+                const bool active = in_strip<PAIR>(a, lane, col);
                 Vec<VEC> acc;
 #pragma unroll
                 for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
@@ -1118,8 +1125,8 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     float *md = a.md + 2 * (int64_t)s0 * a.n_chunks * mdh;
     int32_t *ticket = a.hub_ticket + (int64_t)s0 * a.n_hubs + h;
     for (int s = s0; s < s1; ++s) {
-        const int col = strip_col<VEC, PAIR>(s, lane);
-        const bool active = col < a.F;
+        const int col = strip_col<VEC, PAIR>(a, s, lane);
+        const bool active = in_strip<PAIR>(a, lane, col);
         Vec<VEC> acc;
 #pragma unroll
         for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
@@ -1171,14 +1178,14 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         }
     }
     for (int s = s0; s < s1; ++s) {
-        const int col = strip_col<VEC, PAIR>(s, lane);
-        const bool active = col < a.F;
+        const int col = strip_col<VEC, PAIR>(a, s, lane);
+        const bool active = in_strip<PAIR>(a, lane, col);
         // OP_GATH: the lane's (up to two) heads and their merged softmax states
         int64_t mA = 0, mB = 0;
         int split = VEC;
         float MA = -INFINITY, DA = 0.f, MB = -INFINITY, DB = 0.f;
         if constexpr (OP == OP_GATH) {
-            const int cc = active ? col : s * 32 * VEC;
+            const int cc = active ? col : s * a.lps * VEC;
             mA = cc / a.fh;
             split = (int)((mA + 1) * a.fh - cc);
             mB = min(mA + (split < VEC ? 1 : 0), (int64_t)a.heads - 1);
@@ -1637,6 +1644,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // reduction order is the canonical two-chain order in every case, so panel
     // mode and strip width never change a single output bit.
     int panel = 0, pair = 0;
+    int lps = 32;  // lanes per full-warp strip
     bool panel_off = false;
     {
         const double budget = 0.6 * (double)g->l2_bytes;
@@ -1655,6 +1663,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         } else if (mode == 32) {
             panel = 1;
             vec = 1;
+        } else if (mode > 0 && mode < 128 && mode % 4 == 0 && vec == 4 && r.op != OP_GATH) {
+            panel = 1;  // narrow full-warp strips of `mode` columns
+            lps = mode / 4;
         } else if (xbytes > budget && vec == 4) {
             // GAT recomputes its scores and online-softmax state per strip, so it
             // keeps the wider 128-column strips (measured)
@@ -1662,7 +1673,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             else if (512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
         }
     }
-    const int strip_w = pair ? 64 : 32 * vec;
+    const int strip_w = pair ? 64 : lps * vec;
     const int n_strips = (int)((r.F + strip_w - 1) / strip_w);
     // Few tasks for the resident warps (small graphs): split every task into its
     // strips as separate work items too, so all SMs get work.
@@ -1693,6 +1704,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.C = g->C;
     a.F = (int)r.F;
     a.n_strips = n_strips;
+    a.lps = lps;
     a.panel = panel;
     a.n_items = panel ? g->n_tasks * n_strips : g->n_tasks;
     a.norm = norm;

@@ -8,8 +8,9 @@ prof() {  # <regex> <name> <workload>
       -k "regex:$1" -s 3 -c 1 -o gpurun_out/$R/$2 -f \
       python bench.py --workload $3 --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/$R/$2.log 2>&1
 }
+export TLP_SYNTH_CACHE=/tmp/tlp_synth
 if [ "$P" = "a" ]; then
-  python bench.py > gpurun_out/$R/bench.json 2> gpurun_out/$R/bench.err
+  TLP_TRACE_CREATE=1 python bench.py > gpurun_out/$R/bench.json 2> gpurun_out/$R/bench.err
   ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/$R/launches.csv \
       python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
   prof "_ZN3tlp5k_aggILi4ELi0E" reddit_gcn reddit
@@ -17,5 +18,16 @@ if [ "$P" = "a" ]; then
 else
   prof "_ZN3tlp5k_aggILi4ELi1E" reddit_gin reddit
   prof "_ZN3tlp5k_agg" products_gat products
+  prof "_ZN3tlp5k_aggILi4ELi5E" reddit_gatb reddit_gat_bwd
 fi
 ls -la gpurun_out/$R
+if [ "$P" = "b" ] || [ "$P" = "ab" ]; then
+  # summarise on the box (gpurun copies back at most 64 MiB): raw pages as CSV,
+  # the summary tables, then drop the large .ncu-rep files
+  mkdir -p gpurun_out/prof_$R
+  for f in gpurun_out/$R/*.ncu-rep; do
+    ncu -i "$f" --page raw --csv > gpurun_out/prof_$R/$(basename "$f" .ncu-rep)_raw.csv 2>/dev/null
+  done
+  PROFILES_OUT=gpurun_out/prof_$R python scripts/make_profiles.py $R > /dev/null 2>&1
+  rm -f gpurun_out/$R/*.ncu-rep
+fi

@@ -8,7 +8,7 @@ from ncu_summary import summarise  # noqa: E402
 
 R = sys.argv[1] if len(sys.argv) > 1 else "r01"
 src = os.path.join(ROOT, "gpurun_out", R)
-dst = os.path.join(ROOT, "profiles")
+dst = os.environ.get("PROFILES_OUT") or os.path.join(ROOT, "profiles")
 os.makedirs(dst, exist_ok=True)
 out = [f"# Round {R} profile summary\n"]
 
@@ -49,7 +49,8 @@ if os.path.exists(lc):
 # ncu --set full reports
 traffic = {}
 names = {"reddit_gcn": ("reddit", "gcn"), "reddit_gin": ("reddit", "gin"),
-         "reddit_gat": ("reddit", "gat"), "products_gat": ("products", "gat")}
+         "reddit_gat": ("reddit", "gat"), "products_gat": ("products", "gat"),
+         "reddit_gatb": ("reddit_gat_bwd", "gat_bwd")}
 out.append("## ncu --set full (one launch each, --clock-control none, cold L2)\n\n")
 for nm, (wl, op) in names.items():
     p = os.path.join(src, nm + ".ncu-rep")

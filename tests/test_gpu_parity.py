@@ -952,3 +952,27 @@ def test_epilogue_projection_argument_errors(tlp):
     with pytest.raises(Exception):
         g.aggregate("gcn", X, att_l=_t(synth.normal(8, 2)))  # no el_out
     g.close()
+
+
+@pytest.mark.parametrize("cols", ["96", "80", "44", "4"])
+def test_narrow_strips_bitwise(tlp, monkeypatch, cols):
+    """Narrow full-warp feature strips (lanes >= cols/4 idle) give bitwise the
+    result of the default layout (the per-element reduction order does not
+    depend on the strip), for every single-head op, with hub chunks."""
+    rp, ci, n = _edge_graphs()["powerlaw_hubs"]
+    F = 203
+    X = _t(synth.features(n, F, 204, seed=31))
+    el, er = _t(synth.normal(n, 32)), _t(synth.normal(n, 33))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+
+    def run():
+        return [g.gcn(X, "both", F=F), g.gin(X, 0.1, F=F), g.gat(X, el, er, 0.2, F=F),
+                g.sage(X, True, F=F)]
+    monkeypatch.setenv("TLP_PANEL", "128")
+    ref = run()
+    monkeypatch.setenv("TLP_PANEL", cols)
+    got = run()
+    for a_, b_ in zip(ref, got):
+        assert torch.equal(a_, b_)
+    _check("gcn narrow", got[0], oracle.gcn(rp, ci, X.cpu().numpy(), "both", F=F))
+    g.close()
