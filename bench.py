@@ -384,6 +384,31 @@ def run_tlp(args):
     step_bytes = sum(gather_bytes(op, n, E, F) for op in ops)
     value = step_bytes / (ms_per_step * 1e-3) / 1e9
 
+    # ---- SURVEY 8(d) d3 extras: host wall time of one API call (launch
+    # overhead, not synchronised) and, with --cold, each op with L2 flushed
+    host_us = {}
+    for op in ops:
+        torch.cuda.synchronize()
+        t_h = time.perf_counter()
+        launch(op)
+        host_us[op] = (time.perf_counter() - t_h) * 1e6
+        torch.cuda.synchronize()
+    cold_ms = {}
+    if args.cold:
+        flush = torch.empty(int(2.5 * 126e6) // 4, dtype=torch.float32, device=dev)  # > 2x L2
+        for op in ops:
+            vals = []
+            for _ in range(max(3, min(args.steps, 10))):
+                flush.zero_()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                launch(op)
+                b.record(stream)
+                torch.cuda.synchronize()
+                vals.append(a.elapsed_time(b))
+            cold_ms[op] = statistics.median(vals)
+        del flush
+
     # ---- end to end through the public API with host buffers ----
     e2e = None
     if not args.no_e2e:
@@ -461,10 +486,16 @@ def run_tlp(args):
     for op in ops:
         ms = statistics.mean(op_ms[op])
         by = gather_bytes(op, n, E, F)
+        srt = sorted(op_ms[op])
         per_op[op] = {"ms_mean": round(ms, 4), "ms_median": round(statistics.median(op_ms[op]), 4),
+                      "ms_min": round(srt[0], 4),
+                      "ms_p90": round(srt[min(len(srt) - 1, int(0.9 * len(srt)))], 4),
+                      "host_call_us": round(host_us[op], 1),
                       "gather_bytes": int(by), "gather_GBs": round(by / (ms * 1e-3) / 1e9, 1),
                       "frac_of_8TBs": round(by / (ms * 1e-3) / 1e9 / NOMINAL_HBM_GBS, 4),
                       "edges_x_features_per_s": float(E * F / (ms * 1e-3))}
+        if op in cold_ms:
+            per_op[op]["ms_cold_l2_flushed"] = round(cold_ms[op], 4)
     dom = max(ops, key=lambda o: per_op[o]["ms_mean"])
     traffic = load_traffic(name).get(dom)
     achieved = per_op[dom]["gather_GBs"]
@@ -623,6 +654,8 @@ def main():
     ap.add_argument("--impl", default="tlp", choices=["tlp", "reference"])
     ap.add_argument("--workload", default="reddit", choices=sorted(WORKLOADS))
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cold", action="store_true",
+                    help="also time each op with L2 flushed before it (SURVEY 8(d) d3 cold regime)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--cuda-graph", action="store_true",

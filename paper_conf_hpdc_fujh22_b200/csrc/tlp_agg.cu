@@ -1253,12 +1253,14 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
 }
 
 // Resident CTAs per SM the kernel is compiled for (register budget).  The
-// coefficient-free sums (GIN, SAGE) fit 64 registers, so they run 32 warps per
-// SM (measured: Reddit GIN 24.0 -> 21.8 ms); GCN/GAT keep 85 registers (24
+// coefficient-free sums (GIN, SAGE, GCN NONE / RIGHT / pre-scaled BOTH) fit 64
+// registers, so they run 32 warps per SM (measured: Reddit GIN 24.0 -> 21.8
+// ms); ops with an edge coefficient (weighted, GAT) keep 85 registers (24
 // warps), where fewer registers spill into the edge loop (measured slower).
 constexpr int min_blocks(int op, int coef, bool async) {
     return async ? TLP_MINB_ASYNC
-                 : ((op == OP_GIN || op == OP_SAGE) && coef == COEF_NONE) ? TLP_MINB_LIGHT : TLP_MINB;
+                 : ((op == OP_GIN || op == OP_SAGE || op == OP_GCN) && coef == COEF_NONE)
+                       ? TLP_MINB_LIGHT : TLP_MINB;
 }
 
 template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
@@ -1363,6 +1365,36 @@ static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
 }
 
 static bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
+
+// X'[u, f] = c_out[u] * X[u, f] for f < F (unweighted GCN BOTH); pad columns
+// of X' are never read.
+template <int VEC>
+__global__ void k_prescale(const float *__restrict__ X, const float *__restrict__ c_out, int64_t n,
+                           int64_t F, int64_t ldx, int64_t nvec, float *__restrict__ Xs) {
+    const int64_t tot = n * nvec;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < tot;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t u = i / nvec;
+        const int64_t c = (i - u * nvec) * VEC;
+        const float cu = __ldg(c_out + u);
+        const float *src = X + u * ldx + c;
+        float *dst = Xs + u * ldx + c;
+        if constexpr (VEC == 4) {
+            if (c + 4 <= F) {
+                const float4 x = __ldg(reinterpret_cast<const float4 *>(src));
+                *reinterpret_cast<float4 *>(dst) = make_float4(cu * x.x, cu * x.y, cu * x.z, cu * x.w);
+                continue;
+            }
+        } else if constexpr (VEC == 2) {
+            if (c + 2 <= F) {
+                const float2 x = __ldg(reinterpret_cast<const float2 *>(src));
+                *reinterpret_cast<float2 *>(dst) = make_float2(cu * x.x, cu * x.y);
+                continue;
+            }
+        }
+        for (int k = 0; k < VEC && c + k < F; ++k) dst[k] = cu * __ldg(src + k);
+    }
+}
 
 // NEXT-3: el_out[v] / er_out[v] = sum over strips (in strip order) of the
 // epilogue's partial dots.
@@ -1615,6 +1647,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // c_out[colidx[e]] * w_e precomputed at create (the same fp32 value the
     // kernel would form, so bitwise identical), instead of a dependent gather.
     int coef = COEF_NONE;
+    bool prescale = false;
     const float *ew = g->ew;
     const float *cvec = g->c_out;
     int norm = r.norm;
@@ -1625,14 +1658,51 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         if (g->ew) coef |= COEF_W;
         norm = TLP_NORM_NONE;
     } else if (r.op == OP_GCN && r.norm == TLP_NORM_BOTH) {
-        if (g->ew_both) { ew = g->ew_both; coef |= COEF_W; }
-        else { coef |= COEF_COUT; if (g->ew) coef |= COEF_W; }
+        if (g->ew) {
+            ew = g->ew_both;  // weighted: w_e c_out[u] streamed per edge
+            coef |= COEF_W;
+        } else {
+            prescale = true;  // unweighted: gather X' = c_out (.) X, no edge coefficient
+        }
     } else if (r.op != OP_GAT && r.op != OP_GATB && g->ew) {
         coef |= COEF_W;
     }
     if (r.op == OP_GATB) {  // the edge softmax weights, in transposed edge order
         ew = r.alpha;
         coef = COEF_W;
+    }
+    // Unweighted GCN BOTH: one pass writes
+    // X'[u] = c_out[u] X[u] (each term rounded once, as the oracle's product),
+    // then every gather path sums X' rows with no per-edge coefficient, i.e.
+    // the register budget and instruction count of GIN.  Same bits on every
+    // path, schedule and partition (every path gathers the same X').
+    const float *Xg = r.X;
+    if (prescale) {
+        const size_t need = sizeof(float) * ((size_t)g->n_src * (size_t)r.ldx) + 64;
+        if (need > g->xs_bytes) {
+            if (g->xs) {
+                cudaFreeAsync(g->xs, s);
+                g->device_bytes -= g->xs_bytes;
+                g->xs = nullptr;
+                g->xs_bytes = 0;
+            }
+            cudaError_t e = cudaMallocAsync((void **)&g->xs, need, s);
+            if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(prescaled X)");
+            g->xs_bytes = need;
+            g->device_bytes += need;
+        }
+        const int64_t nvec = (r.F + vec - 1) / vec;
+        const int64_t tot = g->n_src * nvec;
+        const int pb = (int)std::max<int64_t>(1, std::min<int64_t>((tot + 255) / 256, (int64_t)g->num_sms * 16));
+        if (vec == 4)
+            k_prescale<4><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
+        else if (vec == 2)
+            k_prescale<2><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
+        else
+            k_prescale<1><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "k_prescale launch");
+        Xg = g->xs;
     }
 
     // Feature panels: when X is much larger than
@@ -1685,7 +1755,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.colidx = g->colidx;
     a.ew = ew;
     a.c_out = cvec;
-    a.X = r.X;
+    a.X = Xg;
     a.Y = r.Y;
     a.el = r.el;
     a.er = r.er;

@@ -225,7 +225,7 @@ static void graph_free(tlp_graph g) {
     if (!g) return;
     if (g->t) graph_free(g->t);
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
-                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd, g->proj,
+                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd, g->proj, g->xs,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)
@@ -368,7 +368,7 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
             k_norm<<<grid_for(n_src, nsm), 256, 0, s>>>(g->out_deg, n_src, g->c_out, g->c_out_left);
             CTRY(cudaGetLastError());
         }
-        if (nnz) {
+        if (nnz && ew) {  // weighted BOTH streams w_e c_out[u]; unweighted pre-scales X
             TRY(dmalloc((void **)&g->ew_both, sizeof(float) * nnz + 16, g));
             k_edge_both<<<grid_for(nnz, nsm), 256, 0, s>>>(g->colidx, g->ew, g->c_out, nnz, g->ew_both);
             CTRY(cudaGetLastError());

@@ -44,7 +44,9 @@ struct tlp_graph_s {
     int32_t *in_deg = nullptr;   // [n_dst]
     int32_t *out_deg = nullptr;  // [n_src] (global for a dist slice)
     float *c_out = nullptr;      // [n_src] 1/sqrt(max(out_deg,1))
-    float *ew_both = nullptr;    // [nnz] c_out[colidx[e]] * w_e (GCN BOTH coefficient)
+    float *ew_both = nullptr;    // [nnz] c_out[colidx[e]] * w_e (weighted GCN BOTH coefficient)
+    float *xs = nullptr;         // unweighted GCN BOTH: X' = c_out (.) X  [n_src x ldx]
+    size_t xs_bytes = 0;
     float *c_out_left = nullptr; // [n_src] 1/max(out_deg,1) (internal LEFT norm, backward of RIGHT)
     tlp_graph_s *t = nullptr;    // transposed graph (tlp_graph_build_transpose), owned
     // source-reuse tags: colidx with the

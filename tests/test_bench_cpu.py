@@ -50,3 +50,13 @@ def test_reference_arm_runs_on_host():
     d = json.loads(r.stdout.strip().splitlines()[-1])
     assert d["impl"] == "reference" and d["value"] > 0 and d["gpu_launches"] == 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_l2_gather_peak_parses_committed_probe():
+    """bench.py's L2 roofline reads the committed probe: the 256-byte-row,
+    L2-resident (< 80 MB table) entry with the highest bandwidth."""
+    import bench
+    p = bench.l2_gather_peak()
+    assert p is not None
+    assert p["row_bytes"] == 256 and p["table_MB"] < 80
+    assert 5000 < p["GBs"] < 40000
