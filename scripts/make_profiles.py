@@ -36,12 +36,12 @@ if os.path.exists(lc):
         if len(r) > vi:
             tot[r[ki]] += float(r[vi].replace(",", ""))
             cnt[r[ki]] += 1
-    agg = {k: v for k, v in tot.items() if "k_agg" in k}
+    agg = {k: v for k, v in tot.items() if "k_agg" in k or "k_prescale" in k}
     T = sum(agg.values())
     out.append("## ncu launch list (gpu__time_duration.sum, --clock-control none; cold, serialised)\n")
     out.append("Share of the aggregation kernels within the timed bench step (2 steps):\n\n")
     for k, v in sorted(agg.items(), key=lambda x: -x[1]):
-        out.append(f"* {k}: {v / 1e6 / cnt[k]:.2f} ms per launch, {cnt[k]} launches, {100 * v / T:.1f}% of k_agg time\n")
+        out.append(f"* {k}: {v / 1e6 / cnt[k]:.2f} ms per launch, {cnt[k]} launches, {100 * v / T:.1f}% of the step's kernel time\n")
     out.append("\n(other launches in the file are the one-time synthetic-graph generation and graph create)\n\n")
     with open(os.path.join(dst, f"{R}_launches.csv"), "w") as f:
         f.write(open(lc).read())
