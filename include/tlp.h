@@ -156,6 +156,10 @@ typedef struct tlp_graph_info {
     int64_t device_bytes;  /* bytes of device memory owned by the handle        */
     int64_t scratch_bytes; /* hub-partial scratch currently allocated           */
     double create_ms;      /* host wall time of the create call                 */
+    int64_t launches;      /* kernels enqueued by calls on this handle since
+                            * create (aggregations, their pre-/post-passes, the
+                            * transposed handle's backward launches); graph
+                            * construction and NCCL kernels are not counted   */
 } tlp_graph_info;
 
 /* ---- status ------------------------------------------------------------- */

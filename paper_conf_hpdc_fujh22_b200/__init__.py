@@ -48,7 +48,8 @@ class tlp_graph_info(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
         "n_dst", "n_src", "nnz", "row_offset", "max_in_degree", "n_hubs", "n_hub_chunks",
         "n_units", "n_tasks", "hub_threshold", "hub_chunk", "unit_edges", "has_edge_weight",
-        "device_bytes", "scratch_bytes")] + [("create_ms", ctypes.c_double)]
+        "device_bytes", "scratch_bytes")] + [("create_ms", ctypes.c_double),
+                                             ("launches", ctypes.c_int64)]
 
 
 class tlp_agg_desc(ctypes.Structure):

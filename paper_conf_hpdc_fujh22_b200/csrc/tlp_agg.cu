@@ -1366,8 +1366,8 @@ static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
 
 static bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
-// X'[u, f] = c_out[u] * X[u, f] for f < F (unweighted GCN BOTH); pad columns
-// of X' are never read.
+// X'[u, f] = c_out[u] * X[u, f] for f < F (unweighted GCN BOTH); the pad
+// columns of the last vector are zeroed (gathered, never stored to Y).
 template <int VEC>
 __global__ void k_prescale(const float *__restrict__ X, const float *__restrict__ c_out, int64_t n,
                            int64_t F, int64_t ldx, int64_t nvec, float *__restrict__ Xs) {
@@ -1392,7 +1392,9 @@ __global__ void k_prescale(const float *__restrict__ X, const float *__restrict_
                 continue;
             }
         }
-        for (int k = 0; k < VEC && c + k < F; ++k) dst[k] = cu * __ldg(src + k);
+        // the ragged last vector: columns [F, c + VEC) lie inside ldx (vec was
+        // chosen from ldx % VEC) and are read by the gathers, so define them
+        for (int k = 0; k < VEC; ++k) dst[k] = (c + k < F) ? cu * __ldg(src + k) : 0.f;
     }
 }
 
@@ -1410,6 +1412,42 @@ __global__ void k_proj_sum(const float *__restrict__ proj, int n_strips, int64_t
         }
         if (el_out) el_out[v] = l;
         if (er_out) er_out[v] = rr;
+    }
+}
+
+// GAT edge-softmax pre-pass: per
+// local row v, over its in-edges, s_e = LeakyReLU(el[u_e] + er[v]),
+// m_v = max_e s_e, z_v = sum_e exp(s_e - m_v), then alpha_e = exp(s_e - m_v) /
+// z_v written in CSR edge order (the oracle's two-pass softmax).
+// The aggregation then streams alpha as an edge weight.  Warp per row,
+// lane-strided edges, butterfly merge: deterministic.
+__global__ void k_gat_alpha(const int64_t *__restrict__ rowptr, const int32_t *__restrict__ colidx,
+                            int64_t n_dst, const float *__restrict__ el, const float *__restrict__ er,
+                            float slope, float *__restrict__ alpha) {
+    const int lane = threadIdx.x & 31;
+    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n_dst; v += W) {
+        const int64_t e0 = __ldg(rowptr + v), e1 = __ldg(rowptr + v + 1);
+        const float er_v = __ldg(er + v);
+        float m = -INFINITY, z = 0.f;
+        for (int64_t e = e0 + lane; e < e1; e += 32) {
+            const float t = __ldg(el + __ldg(colidx + e)) + er_v;
+            const float sc = t >= 0.f ? t : slope * t;
+            if (sc > m) {
+                z = fmaf(z, __expf(m - sc), 1.f);
+                m = sc;
+            } else {
+                z += __expf(sc - m);
+            }
+        }
+        const float M = warp_max(m);
+        const float Z = warp_sum(m == -INFINITY ? 0.f : z * __expf(m - M));
+        const float iz = 1.0f / Z;  // unused when the row has no edges
+        for (int64_t e = e0 + lane; e < e1; e += 32) {
+            const float t = __ldg(el + __ldg(colidx + e)) + er_v;
+            const float sc = t >= 0.f ? t : slope * t;
+            __stcg(alpha + e, __expf(sc - M) * iz);
+        }
     }
 }
 
@@ -1565,6 +1603,7 @@ static tlp_status hot_threshold(tlp_graph g, int64_t ldx, bool panel, cudaStream
         cudaMemsetAsync(hist, 0, sizeof(unsigned long long) * 32, s);
         k_tag_colidx<<<g->num_sms * 8, 256, 0, s>>>(g->colidx, g->out_deg, g->nnz, tag);
         k_class_hist<<<g->num_sms * 4, 256, 0, s>>>(g->out_deg, g->n_src, hist);
+        g->launches += 2;
         unsigned long long h[32];
         cudaMemcpyAsync(h, hist, sizeof(h), cudaMemcpyDeviceToHost, s);
         cudaError_t ce = cudaStreamSynchronize(s);
@@ -1671,6 +1710,49 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         ew = r.alpha;
         coef = COEF_W;
     }
+    // GAT edge-softmax pre-pass: when X does not fit in L2,
+    // k_gat_alpha writes every edge's alpha_e once and the aggregation becomes
+    // the streamed-weight sum sum_e alpha_e X[u_e] (the GCN-NONE kernel with
+    // COEF_W): it takes the 64-column half-warp strips (the online-softmax
+    // kernel would recompute its running state per strip) and needs no
+    // dependent el[u] gather or rescale.  Measured: Reddit 30.0 -> 27.7 ms,
+    // products 10.1 -> 9.9 ms.  TLP_GAT=online|alpha overrides.
+    int op = r.op;
+    bool gat_alpha = false;
+    if (r.op == OP_GAT) {
+        gat_alpha = 4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes;
+        if (const char *e = getenv("TLP_GAT")) {
+            if (!strcmp(e, "online")) gat_alpha = false;
+            else if (!strcmp(e, "alpha")) gat_alpha = true;
+        }
+        if (gat_alpha && g->nnz > 0) {
+            const size_t need = sizeof(float) * (size_t)g->nnz + 64;
+            if (need > g->galpha_bytes) {
+                if (g->galpha) {
+                    cudaFreeAsync(g->galpha, s);
+                    g->device_bytes -= g->galpha_bytes;
+                    g->galpha = nullptr;
+                    g->galpha_bytes = 0;
+                }
+                cudaError_t e = cudaMallocAsync((void **)&g->galpha, need, s);
+                if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(GAT alpha)");
+                g->galpha_bytes = need;
+                g->device_bytes += need;
+            }
+            const int pb = (int)std::max<int64_t>(1, std::min<int64_t>((g->n_dst + 7) / 8, (int64_t)g->num_sms * 16));
+            k_gat_alpha<<<pb, 256, 0, s>>>(g->rowptr, g->colidx, g->n_dst, r.el, r.er + g->row_offset,
+                                           r.slope, g->galpha);
+            g->launches += 1;
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return cuda_error(e, "k_gat_alpha launch");
+        }
+        if (gat_alpha) {
+            op = OP_GCN;  // Y[v] = sum_e alpha_e X[u_e]: unnormalised streamed-weight sum
+            norm = TLP_NORM_NONE;
+            coef = COEF_W;
+            ew = g->galpha;
+        }
+    }
     // Unweighted GCN BOTH: one pass writes
     // X'[u] = c_out[u] X[u] (each term rounded once, as the oracle's product),
     // then every gather path sums X' rows with no per-edge coefficient, i.e.
@@ -1700,6 +1782,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             k_prescale<2><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
         else
             k_prescale<1><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
+        g->launches += 1;
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "k_prescale launch");
         Xg = g->xs;
@@ -1737,9 +1820,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             panel = 1;  // narrow full-warp strips of `mode` columns
             lps = mode / 4;
         } else if (xbytes > budget && vec == 4) {
-            // GAT recomputes its scores and online-softmax state per strip, so it
+            // online-softmax GAT recomputes its running state per strip, so it
             // keeps the wider 128-column strips (measured)
-            if (r.op != OP_GAT && r.op != OP_GATH && 256.0 * g->n_src <= budget) { panel = 1; pair = 1; }
+            if (op != OP_GAT && op != OP_GATH && 256.0 * g->n_src <= budget) {
+                panel = 1;
+                pair = 1;
+            }
             else if (512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
         }
     }
@@ -1904,7 +1990,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             if (const char *e = getenv("TLP_HOT_COLD")) a.cold_first = atoi(e);
         }
     }
-    KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, r.op, coef);
+    KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, op, coef);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
     size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;
@@ -1922,11 +2008,13 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (blocks < 1) blocks = 1;
     if (blocks > 0x7fffffff) return set_error(TLP_ERR_UNSUPPORTED, "grid too large");
     fn<<<(unsigned)blocks, threads, smem, s>>>(a);
+    g->launches += 1;
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_agg launch");
     if (want_proj) {
         const int pb = (int)std::min<int64_t>((g->n_dst + 255) / 256, (int64_t)g->num_sms * 8);
         k_proj_sum<<<pb, 256, 0, s>>>(g->proj, n_strips, g->n_dst, r.el_out, r.er_out);
+        g->launches += 1;
         e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "k_proj_sum launch");
     }
@@ -2035,6 +2123,7 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
     if (n_dst) {
         k_gatb_stats<<<nsm * 8, 256, 0, s>>>(g->rowptr, g->colidx, n_dst, el, er, slope, dY, lddy, Y,
                                              ldy, F, vstat);
+        g->launches += 1;
         TLP_CUDA_TRY(cudaGetLastError());
     }
     if (n_src == 0) {
@@ -2042,6 +2131,7 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
         return TLP_OK;
     }
     k_gatb_alpha<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, slope, alpha);
+    g->launches += 1;
     TLP_CUDA_TRY(cudaGetLastError());
     AggRequest r;
     r.op = OP_GATB;
@@ -2056,9 +2146,11 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
     if (st != TLP_OK) return st;
     k_gatb_edges<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, alpha, slope,
                                          gbuf, n_strips, nnz, dt, del);
+    g->launches += 1;
     TLP_CUDA_TRY(cudaGetLastError());
     if (n_dst) {
         k_gatb_der<<<nsm * 8, 256, 0, s>>>(g->rowptr, n_dst, g->tpos, dt, der);
+        g->launches += 1;
         TLP_CUDA_TRY(cudaGetLastError());
     }
     return TLP_OK;

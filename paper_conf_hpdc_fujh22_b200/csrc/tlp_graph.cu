@@ -225,7 +225,7 @@ static void graph_free(tlp_graph g) {
     if (!g) return;
     if (g->t) graph_free(g->t);
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
-                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd, g->proj, g->xs,
+                    g->c_out_left, g->colidx_tag, g->tpos, g->bwd, g->proj, g->xs, g->galpha,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,
                     g->scratch};
     for (void *p : ptrs)
@@ -663,6 +663,7 @@ tlp_status tlp_graph_info_get(tlp_graph g, tlp_graph_info *o) {
     o->device_bytes = (int64_t)g->device_bytes;
     o->scratch_bytes = (int64_t)g->scratch_bytes;
     o->create_ms = g->create_ms;
+    o->launches = g->launches + (g->t ? g->t->launches : 0);
     return TLP_OK;
 }
 

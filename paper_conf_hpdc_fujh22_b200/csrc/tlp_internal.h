@@ -57,6 +57,8 @@ struct tlp_graph_s {
     size_t bwd_bytes = 0;
     float *proj = nullptr;           // epilogue projection partials [strips x n_dst x 2]
     size_t proj_bytes = 0;
+    float *galpha = nullptr;         // GAT edge softmax alpha_e (k_gat_alpha) [nnz]
+    size_t galpha_bytes = 0;
     int64_t tag_hist[32] = {0};      // sources per out-degree class
 
     int2 *tasks = nullptr;       // [n_tasks]
@@ -72,6 +74,7 @@ struct tlp_graph_s {
     size_t l2_bytes = 0;
     size_t device_bytes = 0;
     double create_ms = 0.0;
+    int64_t launches = 0;        // kernels enqueued by calls on this handle (after create)
 
     int sched = TLP_SCHED_DYNAMIC;
     int warps_per_cta = 8;

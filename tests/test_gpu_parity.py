@@ -383,7 +383,10 @@ def test_config_reddit_gcn_gin_sampled(tlp, reddit, nonneg):
     g.close()
 
 
-def test_config_reddit_gat_sampled(tlp, reddit):
+@pytest.mark.parametrize("gat_mode", ["auto", "online"])
+def test_config_reddit_gat_sampled(tlp, reddit, monkeypatch, gat_mode):
+    if gat_mode != "auto":
+        monkeypatch.setenv("TLP_GAT", gat_mode)
     cfg = synth.CONFIGS["reddit"]
     n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
     rp, ci = reddit
@@ -400,7 +403,10 @@ def test_config_reddit_gat_sampled(tlp, reddit):
     g.close()
 
 
-def test_config_products_gat_sampled(tlp):
+@pytest.mark.parametrize("gat_mode", ["auto", "online"])
+def test_config_products_gat_sampled(tlp, monkeypatch, gat_mode):
+    if gat_mode != "auto":
+        monkeypatch.setenv("TLP_GAT", gat_mode)
     cfg = synth.CONFIGS["products"]
     n, F = cfg["n"], cfg["F"]
     rp, ci = synth.dataset_graph("products")
@@ -975,4 +981,85 @@ def test_narrow_strips_bitwise(tlp, monkeypatch, cols):
     for a_, b_ in zip(ref, got):
         assert torch.equal(a_, b_)
     _check("gcn narrow", got[0], oracle.gcn(rp, ci, X.cpu().numpy(), "both", F=F))
+    g.close()
+
+
+# ------------------------------------- GAT edge-softmax pre-pass (alpha mode) --
+
+@pytest.mark.parametrize("name", list(_edge_graphs()))
+def test_gat_alpha_mode_edge_graphs(tlp, monkeypatch, name):
+    """GAT through the edge-softmax pre-pass (alpha_e = exp(s_e - m_v) / z_v
+    written once, then a streamed-weight sum; the oracle's two-pass softmax,
+    P:1001-1007) on the edge-case graphs."""
+    monkeypatch.setenv("TLP_GAT", "alpha")
+    rp, ci, n_src = _edge_graphs()[name]
+    _run_all(tlp, rp, ci, n_src, 37, 40, opts=dict(hub_threshold=64, hub_chunk=32), ops=("gat",))
+    _run_all(tlp, rp, ci, n_src, 130, 132, opts=dict(hub_threshold=64, hub_chunk=32), ops=("gat",),
+             nonneg=True)
+
+
+def test_gat_alpha_mode_bitwise_across_paths(tlp, monkeypatch):
+    """Within the alpha mode every strip width, gather path, schedule and row
+    partition gives the same bits (alpha_e is computed once per row)."""
+    monkeypatch.setenv("TLP_GAT", "alpha")
+    n, F, ld = 3000, 300, 300
+    rp, ci = synth.chung_lu(n, 80000, 0.5, 13, device="cpu")
+    Xh = synth.features(n, F, ld, seed=5)
+    elh, erh = synth.normal(n, 1), synth.normal(n, 2)
+    X, el, er = _t(Xh), _t(elh), _t(erh)
+    opts = dict(hub_threshold=64, hub_chunk=32)
+    g = tlp.Graph(_t(rp), _t(ci), opts=opts)
+    base = g.gat(X, el, er, 0.2).clone()
+    _check("alpha gat", base, oracle.gat(rp, ci, Xh, elh, erh, 0.2))
+    for mode in ("0", "32", "64", "128", "48"):
+        monkeypatch.setenv("TLP_PANEL", mode)
+        assert torch.equal(g.gat(X, el, er, 0.2), base), mode
+    monkeypatch.setenv("TLP_PANEL", "0")
+    for path in ("reg", "async"):
+        monkeypatch.setenv("TLP_GATHER", path)
+        assert torch.equal(g.gat(X, el, er, 0.2), base), path
+    monkeypatch.delenv("TLP_GATHER")
+    monkeypatch.setenv("TLP_PANEL", "64")
+    for sched in ("static", "hardware", "dynamic"):
+        for wpc, step in ((4, 1), (8, 3)):
+            g.set_schedule(sched, wpc, step)
+            assert torch.equal(g.gat(X, el, er, 0.2), base), (sched, wpc, step)
+    b = tlp.tlp_partition_rows(rp, 3)
+    out = torch.full((n, ld), float("nan"), device=DEV)
+    for k in range(3):
+        h = tlp.tlp_graph_create_rows(_t(rp), _t(ci), int(b[k]), int(b[k + 1]), opts=opts)
+        sl = tlp.Graph(None, None, handle=h)
+        if b[k + 1] > b[k]:
+            sl.gat(X, el, er, 0.2, Y=out[int(b[k]):int(b[k + 1])])
+        sl.close()
+    assert torch.equal(out, base)
+    g.close()
+
+
+@pytest.mark.parametrize("scale", [30.0, 80.0])
+def test_gat_alpha_mode_extreme_scores(tlp, monkeypatch, scale):
+    monkeypatch.setenv("TLP_GAT", "alpha")
+    n = 1200
+    rp, ci = synth.chung_lu(n, 30000, 0.5, 61, device="cpu")
+    Xh = synth.features(n, 64, 64, seed=1)
+    el = synth.normal(n, 2) * scale
+    er = synth.normal(n, 3) * scale
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    for slope in (0.2, 1.0):
+        Y = g.gat(_t(Xh), _t(el), _t(er), slope)
+        assert torch.isfinite(Y).all()
+        _check(f"alpha gat x{scale}", Y, oracle.gat(rp, ci, Xh, el, er, slope))
+    g.close()
+
+
+def test_gat_alpha_mode_pubmed_all_rows(tlp, monkeypatch):
+    monkeypatch.setenv("TLP_GAT", "alpha")
+    cfg = synth.CONFIGS["pubmed"]
+    n = cfg["n"]
+    rp, ci = synth.dataset_graph("pubmed")
+    X = synth.dataset_features("pubmed", n)
+    el, er = synth.normal(n, 201), synth.normal(n, 202)
+    g = tlp.Graph(_t(rp), _t(ci))
+    Y = g.gat(_t(X), _t(el), _t(er), synth.SLOPE, F=cfg["F"])
+    _check("pubmed alpha gat", Y, oracle.gat(rp, ci, X, el, er, synth.SLOPE, F=cfg["F"]))
     g.close()
