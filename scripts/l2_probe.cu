@@ -6,6 +6,7 @@
 // build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o build/l2_probe scripts/l2_probe.cu
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 template <int ROWB, int U>
@@ -61,5 +62,14 @@ int main() {
         run<256, 8>(tab, tb, sms, out);
         run<512, 4>(tab, tb, sms, out);
     }
+    // narrow rows (narrow feature panels for X >> L2, e.g. products F = 100):
+    // 16..128-byte random rows from an L2-resident table
+    if (getenv("PROBE_NARROW"))
+        for (int64_t tb : {int64_t(60) << 20, int64_t(78) << 20}) {
+            run<16, 8>(tab, tb, sms, out);
+            run<32, 8>(tab, tb, sms, out);
+            run<64, 8>(tab, tb, sms, out);
+            run<128, 8>(tab, tb, sms, out);
+        }
     return 0;
 }

@@ -36,7 +36,7 @@ if os.path.exists(lc):
         if len(r) > vi:
             tot[r[ki]] += float(r[vi].replace(",", ""))
             cnt[r[ki]] += 1
-    agg = {k: v for k, v in tot.items() if "k_agg" in k or "k_prescale" in k}
+    agg = {k: v for k, v in tot.items() if "k_agg" in k or "k_prescale" in k or "k_gat_alpha" in k}
     T = sum(agg.values())
     out.append("## ncu launch list (gpu__time_duration.sum, --clock-control none; cold, serialised)\n")
     out.append("Share of the aggregation kernels within the timed bench step (2 steps):\n\n")
@@ -49,7 +49,8 @@ if os.path.exists(lc):
 # ncu --set full reports
 traffic = {}
 names = {"reddit_gcn": ("reddit", "gcn"), "reddit_gin": ("reddit", "gin"),
-         "reddit_gat": ("reddit", "gat"), "products_gat": ("products", "gat"),
+         "reddit_gat": ("reddit", "gat"), "reddit_gat_alpha": ("reddit", "gat_alpha"),
+         "products_gat": ("products", "gat"),
          "reddit_gatb": ("reddit_gat_bwd", "gat_bwd")}
 out.append("## ncu --set full (one launch each, --clock-control none, cold L2)\n\n")
 for nm, (wl, op) in names.items():
