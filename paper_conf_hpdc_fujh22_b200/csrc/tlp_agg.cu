@@ -1419,35 +1419,89 @@ __global__ void k_proj_sum(const float *__restrict__ proj, int n_strips, int64_t
 // local row v, over its in-edges, s_e = LeakyReLU(el[u_e] + er[v]),
 // m_v = max_e s_e, z_v = sum_e exp(s_e - m_v), then alpha_e = exp(s_e - m_v) /
 // z_v written in CSR edge order (the oracle's two-pass softmax).
-// The aggregation then streams alpha as an edge weight.  Warp per row,
-// lane-strided edges, butterfly merge: deterministic.
-__global__ void k_gat_alpha(const int64_t *__restrict__ rowptr, const int32_t *__restrict__ colidx,
-                            int64_t n_dst, const float *__restrict__ el, const float *__restrict__ er,
-                            float slope, float *__restrict__ alpha) {
-    const int lane = threadIdx.x & 31;
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n_dst; v += W) {
-        const int64_t e0 = __ldg(rowptr + v), e1 = __ldg(rowptr + v + 1);
-        const float er_v = __ldg(er + v);
-        float m = -INFINITY, z = 0.f;
-        for (int64_t e = e0 + lane; e < e1; e += 32) {
-            const float t = __ldg(el + __ldg(colidx + e)) + er_v;
-            const float sc = t >= 0.f ? t : slope * t;
-            if (sc > m) {
-                z = fmaf(z, __expf(m - sc), 1.f);
-                m = sc;
-            } else {
-                z += __expf(sc - m);
+// The aggregation then streams alpha as an edge weight.
+//   blocks [0, n_hubs): one hub row (in-degree > H) per CTA, thread-strided
+//     edges, fixed-order block reduction (a 20K-edge hub does not serialise
+//     one warp);
+//   blocks [n_hubs, grid): warp per regular row.
+// Pass 1 gathers 8 scores per thread per step (8 independent colidx -> el
+// chains in flight) and parks s_e in alpha[e]; pass 2 re-reads them (the same
+// thread's own stores, L2-resident: no dependent gather) and writes alpha_e.
+// Deterministic; hub-ness depends only on the degree and H, so a row slice
+// (dist) produces the same bits.
+constexpr int kAlphaUnroll = 8;
+
+template <int NT>
+__device__ __forceinline__ void alpha_row(const int32_t *__restrict__ colidx, const float *__restrict__ el,
+                                          int64_t e0, int64_t e1, float er_v, float slope, int tid,
+                                          float *alpha, float *red) {
+    constexpr int UN = kAlphaUnroll;
+    const int lane = tid & 31;
+    float m = -INFINITY, z = 0.f;
+    for (int64_t b = e0 + tid; b < e1; b += (int64_t)NT * UN) {
+        int c[UN];
+#pragma unroll
+        for (int k = 0; k < UN; ++k) c[k] = (b + k * NT < e1) ? __ldg(colidx + b + k * NT) : -1;
+        float sc[UN];
+        float mk = -INFINITY;
+#pragma unroll
+        for (int k = 0; k < UN; ++k) {
+            sc[k] = -INFINITY;
+            if (c[k] >= 0) {
+                const float t = __ldg(el + c[k]) + er_v;
+                sc[k] = t >= 0.f ? t : slope * t;  // LeakyReLU (R6)
+                alpha[b + k * NT] = sc[k];
             }
+            mk = fmaxf(mk, sc[k]);
         }
-        const float M = warp_max(m);
-        const float Z = warp_sum(m == -INFINITY ? 0.f : z * __expf(m - M));
-        const float iz = 1.0f / Z;  // unused when the row has no edges
-        for (int64_t e = e0 + lane; e < e1; e += 32) {
-            const float t = __ldg(el + __ldg(colidx + e)) + er_v;
-            const float sc = t >= 0.f ? t : slope * t;
-            __stcg(alpha + e, __expf(sc - M) * iz);
+        if (mk > m) {  // one rescale per step
+            z *= __expf(m - mk);
+            m = mk;
         }
+#pragma unroll
+        for (int k = 0; k < UN; ++k) z += __expf(sc[k] - m);  // exp(-inf) = 0
+    }
+    float M = warp_max(m);
+    float Z = warp_sum(m == -INFINITY ? 0.f : z * __expf(m - M));
+    if constexpr (NT > 32) {
+        const int w = tid >> 5;
+        if (lane == 0) { red[w] = M; red[8 + w] = Z; }
+        __syncthreads();
+        const float mw = lane < NT / 32 ? red[lane] : -INFINITY;
+        const float zw = lane < NT / 32 ? red[8 + lane] : 0.f;
+        M = warp_max(mw);
+        Z = warp_sum(mw == -INFINITY ? 0.f : zw * __expf(mw - M));
+    }
+    const float iz = 1.0f / Z;  // unused when the row has no edges
+    for (int64_t b = e0 + tid; b < e1; b += (int64_t)NT * UN) {
+        float sc[UN];
+#pragma unroll
+        for (int k = 0; k < UN; ++k)
+            if (b + k * NT < e1) sc[k] = alpha[b + k * NT];
+#pragma unroll
+        for (int k = 0; k < UN; ++k)
+            if (b + k * NT < e1) __stcg(alpha + b + k * NT, __expf(sc[k] - M) * iz);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_gat_alpha(const int64_t *__restrict__ rowptr,
+                                                   const int32_t *__restrict__ colidx, int64_t n_dst,
+                                                   const float *__restrict__ el, const float *__restrict__ er,
+                                                   float slope, const int32_t *__restrict__ hub_row,
+                                                   int64_t n_hubs, int64_t H, float *alpha) {
+    __shared__ float red[16];
+    if ((int64_t)blockIdx.x < n_hubs) {
+        const int r = __ldg(hub_row + blockIdx.x);
+        alpha_row<256>(colidx, el, __ldg(rowptr + r), __ldg(rowptr + r + 1), __ldg(er + r), slope,
+                       threadIdx.x, alpha, red);
+        return;
+    }
+    const int lane = threadIdx.x & 31;
+    const int64_t W = ((int64_t)(gridDim.x - n_hubs) * blockDim.x) >> 5;
+    for (int64_t v = (((int64_t)blockIdx.x - n_hubs) * blockDim.x + threadIdx.x) >> 5; v < n_dst; v += W) {
+        const int64_t e0 = __ldg(rowptr + v), e1 = __ldg(rowptr + v + 1);
+        if (e1 - e0 > H) continue;  // a hub: its own CTA
+        alpha_row<32>(colidx, el, e0, e1, __ldg(er + v), slope, lane, alpha, red);
     }
 }
 
@@ -1739,9 +1793,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
                 g->galpha_bytes = need;
                 g->device_bytes += need;
             }
-            const int pb = (int)std::max<int64_t>(1, std::min<int64_t>((g->n_dst + 7) / 8, (int64_t)g->num_sms * 16));
-            k_gat_alpha<<<pb, 256, 0, s>>>(g->rowptr, g->colidx, g->n_dst, r.el, r.er + g->row_offset,
-                                           r.slope, g->galpha);
+            const int64_t pb = g->n_hubs + std::max<int64_t>(1, std::min<int64_t>((g->n_dst + 7) / 8, (int64_t)g->num_sms * 16));
+            k_gat_alpha<<<(unsigned)pb, 256, 0, s>>>(g->rowptr, g->colidx, g->n_dst, r.el, r.er + g->row_offset,
+                                                     r.slope, g->hub_row, g->n_hubs, g->H, g->galpha);
             g->launches += 1;
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return cuda_error(e, "k_gat_alpha launch");

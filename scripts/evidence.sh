@@ -13,7 +13,7 @@ if [ "$P" = "a" ]; then
   TLP_TRACE_CREATE=1 python bench.py > gpurun_out/$R/bench.json 2> gpurun_out/$R/bench.err
   ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/$R/launches.csv \
       python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
-  prof "_ZN3tlp5k_aggILi4ELi0E" reddit_gcn reddit
+  prof "_ZN3tlp5k_aggILi4ELi0ELi0E" reddit_gcn reddit
   # GAT on Reddit runs as k_gat_alpha + the streamed-weight sum k_agg<4, 0(GCN), 2(COEF_W), ...>
   prof "_ZN3tlp5k_aggILi4ELi0ELi2E" reddit_gat reddit
   prof "k_gat_alpha" reddit_gat_alpha reddit
