@@ -180,6 +180,10 @@ class ClockSampler:
 WORKLOADS = {
     "reddit": dict(graph="reddit", ops=OPS),
     "products": dict(graph="products", ops=("gat",)),
+    # single-op Reddit workloads (kernel experiments)
+    "reddit_gcn": dict(graph="reddit", ops=("gcn",)),
+    "reddit_gin": dict(graph="reddit", ops=("gin",)),
+    "reddit_gat": dict(graph="reddit", ops=("gat",)),
     "pubmed": dict(graph="pubmed", ops=("gat",)),
     "cora": dict(graph="cora", ops=("gcn",)),
     "rmat24": dict(graph="rmat24", ops=("gcn2",)),

@@ -1256,7 +1256,8 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
 // coefficient-free sums (GIN, SAGE, GCN NONE / RIGHT / pre-scaled BOTH) fit 64
 // registers, so they run 32 warps per SM (measured: Reddit GIN 24.0 -> 21.8
 // ms); ops with an edge coefficient (weighted, GAT) keep 85 registers (24
-// warps), where fewer registers spill into the edge loop (measured slower).
+// warps), where fewer registers spill into the edge loop (measured slower;
+// the alpha-mode GAT gather at 4 CTAs/SM: 26.9 -> 31.0 ms on Reddit).
 constexpr int min_blocks(int op, int coef, bool async) {
     return async ? TLP_MINB_ASYNC
                  : ((op == OP_GIN || op == OP_SAGE || op == OP_GCN) && coef == COEF_NONE)
@@ -1264,7 +1265,7 @@ constexpr int min_blocks(int op, int coef, bool async) {
 }
 
 template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
-__global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC)) k_agg(const AggArgs a) {
+__device__ __forceinline__ void agg_body(const AggArgs &a) {
     const int lane = threadIdx.x & 31;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (a.sched == S_HARDWARE) {  // one warp per item
@@ -1293,6 +1294,11 @@ __global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC)) k_agg(c
             __threadfence();
         }
     }
+}
+
+template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
+__global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC)) k_agg(const AggArgs a) {
+    agg_body<VEC, OP, COEF, U, ASYNC, PAIR>(a);
 }
 
 // ------------------------------------------------------------- dispatch --
