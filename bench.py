@@ -184,6 +184,14 @@ WORKLOADS = {
     "reddit_gcn": dict(graph="reddit", ops=("gcn",)),
     "reddit_gin": dict(graph="reddit", ops=("gin",)),
     "reddit_gat": dict(graph="reddit", ops=("gat",)),
+    # the paper's own measurement shape (F = 32; Table 5): context for
+    # its V100 numbers, not a BASELINE.json config
+    "reddit_f32": dict(graph="reddit", ops=OPS, F=32, ld=32,
+                       paper_v100_ms={"gcn": 6.9, "gin": 7.3, "gat": 14.6},
+                       paper_src="PAPER.md Table 5 P:1175, P:1189, P:1217 (V100 32 GB, F=32, mean of 10)"),
+    "products_f32": dict(graph="products", ops=OPS, F=32, ld=32,
+                         paper_v100_ms={"gcn": 16.1, "gin": 16.4, "gat": 28.4},
+                         paper_src="PAPER.md Table 5 P:1179, P:1193, P:1221 (V100 32 GB, F=32, mean of 10)"),
     "pubmed": dict(graph="pubmed", ops=("gat",)),
     "cora": dict(graph="cora", ops=("gcn",)),
     "rmat24": dict(graph="rmat24", ops=("gcn2",)),
@@ -212,10 +220,15 @@ def cfg_n(cfg):
 
 def make_inputs(name, device):
     import synth
-    cfg = synth.CONFIGS[WORKLOADS[name]["graph"]]
-    rp, ci = synth.dataset_graph(WORKLOADS[name]["graph"], device=device)
+    w = WORKLOADS[name]
+    cfg = synth.CONFIGS[w["graph"]]
+    rp, ci = synth.dataset_graph(w["graph"], device=device)
     n = cfg_n(cfg)
-    X = synth.dataset_features(WORKLOADS[name]["graph"], n)
+    if "F" in w:  # feature width override (the paper's F = 32 shape)
+        cfg = dict(cfg, F=w["F"], ld=w["ld"])
+        X = synth.features(n, w["F"], w["ld"], seed=synth.FEATURE_SEED_BASE + synth.CONFIG_INDEX[w["graph"]])
+    else:
+        X = synth.dataset_features(w["graph"], n)
     H = max([int(o[3:]) for o in WORKLOADS[name]["ops"] if o.startswith("gat") and o[3:].isdigit()]
             or [1])
     el = synth.normal(n * H, 1000 + synth.CONFIG_INDEX[WORKLOADS[name]["graph"]])
@@ -540,8 +553,10 @@ def run_tlp(args):
         "config": {"workload": workload_desc(name, cfg, E),
                    "graph": ("R-MAT G2 (0.57,0.19,0.19,0.05), seed %d" if name == "rmat24"
                              else "Chung-Lu G1 (SURVEY 8(d) d1), seed %d") % cfg["seed"],
-                   "l2": "inputs larger than L2 (X = %.0f MB, colidx = %.0f MB vs 126 MB L2); no flush"
-                         % (n * ld * 4 / 1e6, E * 4 / 1e6),
+                   "l2": ("inputs larger than L2 (X = %.0f MB, colidx = %.0f MB vs 126 MB L2); no flush"
+                          % (n * ld * 4 / 1e6, E * 4 / 1e6)) if n * ld * 4 > 126e6 else
+                         ("X = %.0f MB fits L2 (warm between reps); colidx = %.0f MB streams from HBM; "
+                          "--cold adds L2-flushed times" % (n * ld * 4 / 1e6, E * 4 / 1e6)),
                    "parallelism": ("rows%d (edge-balanced row ranges, X replicated, %s)" % (
                        world, "fused peer-store all-gather (NEXT-2)" if fused else
                        "grouped-broadcast all-gather of Y")) if use_dist else "single",
@@ -553,6 +568,13 @@ def run_tlp(args):
         "gpu_launches": int(n_launches),
         "clocks": clk.summary(), "e2e": e2e,
     }
+    w = WORKLOADS[name]
+    if "paper_v100_ms" in w:
+        # context only (another GPU, the paper's own F = 32 measurement)
+        result["paper_context"] = {
+            "v100_ms": w["paper_v100_ms"], "source": w["paper_src"],
+            "b200_over_v100": {o: round(w["paper_v100_ms"][o] / per_op[o]["ms_mean"], 2)
+                               for o in ops if o in w["paper_v100_ms"]}}
     if use_dist:
         result["gpu_launches_note"] = "per rank, counted by the library; NCCL's broadcast kernels not included"
     if rank == 0 and not args.no_cpu_baseline and world == 1:

@@ -235,18 +235,28 @@ __device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, un
 // order, hence bitwise-identical results.
 //
 // Lane -> edge mapping inside a 32-edge chunk, for step j, group slot k:
-//   full warp: every lane gathers edge j+k for its 4 columns (chain (j+k)&1)
-//   PAIR     : lanes 0-15 gather edge 2(j+k), lanes 16-31 edge 2(j+k)+1, over
-//              64 columns, so a warp-wide LDG.128 still moves 512 bytes while
-//              the strip of X is half as wide (each half-warp is one chain).
+//   G = 1 (full warp): every lane gathers edge j+k for its 4 columns
+//              (chain (j+k)&1);
+//   G = 2 (PAIR): lanes 0-15 gather edge 2(j+k), lanes 16-31 edge 2(j+k)+1,
+//              over 64 columns, so a warp-wide LDG.128 still moves 512 bytes
+//              while the strip of X is half as wide (each half-warp is one
+//              chain: the canonical even/odd order);
+//   G = 4, 8 (narrow rows, F <= 32 / 16): lane group g = lane / (32/G) gathers
+//              edge G(j+k)+g, so a warp instruction still moves G rows.  Group
+//              g accumulates the chain of positions = g (mod G); the chains
+//              are added by a fixed butterfly (xor 16, then 8, ...).  This
+//              order depends only on F (never on P, the schedule or the
+//              partition), so results stay bitwise reproducible and
+//              partition-invariant; G <= 2 paths are bitwise identical to each
+//              other (R10).
 
-template <int VEC, int U, bool HASC, bool PAIR, bool CLAMP>
+template <int VEC, int U, bool HASC, int G, bool CLAMP>
 __device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes, int j, int n,
-                                            int half, int u_l, float c_l, Vec<VEC> (&xv)[U],
+                                            int grp, int u_l, float c_l, Vec<VEC> (&xv)[U],
                                             float (&ck)[U]) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-        int p = PAIR ? 2 * (j + k) + half : j + k;
+        int p = G * (j + k) + grp;
         if constexpr (CLAMP) p = min(p, n - 1);  // duplicate of a line in flight
         const unsigned u = (unsigned)__shfl_sync(FULL, u_l, p);
         if constexpr (HASC) ck[k] = __shfl_sync(FULL, c_l, p);
@@ -255,15 +265,13 @@ __device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes
 }
 
 // PHASE: parity of the group's first step (the caller's j is a multiple of 2U).
-template <int VEC, int U, bool HASC, bool PAIR, bool GUARD, int PHASE>
-__device__ __forceinline__ void consume_group(int j, int n, int half, const Vec<VEC> (&xv)[U],
+template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE>
+__device__ __forceinline__ void consume_group(int j, int n, int grp, const Vec<VEC> (&xv)[U],
                                               const float (&ck)[U], Vec<VEC> (&ac)[2]) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
-        const int p = PAIR ? 2 * (j + k) + half : j + k;
-        constexpr int dummy = 0;
-        (void)dummy;
-        const int ch = PAIR ? 0 : ((PHASE + k) & 1);
+        const int p = G * (j + k) + grp;
+        const int ch = (G > 1) ? 0 : ((PHASE + k) & 1);
         if (!GUARD || p < n) {
 #pragma unroll
             for (int c = 0; c < VEC; ++c) {
@@ -388,7 +396,7 @@ __device__ __forceinline__ float ld_stream(const float *ptr) {
 //  * the gathers of a chunk are issued in double-buffered groups of U source
 //    rows: the next group is in flight while the current one is accumulated;
 //    full 32-edge chunks are fully unrolled (compile-time shuffle lanes).
-template <int VEC, int OP, int COEF, int U, bool PAIR>
+template <int VEC, int OP, int COEF, int U, int G>
 __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64_t e1,
                                              int col, bool active, float er_v, int lane,
                                              Vec<VEC> &acc, float &m, float &den,
@@ -399,8 +407,10 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     constexpr bool GB = (OP == OP_GATB);
     constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT) || GB;
     constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);  // index-dependent value
-    constexpr int STEPS = PAIR ? 16 : 32;  // gather steps of a full chunk
+    constexpr int STEPS = 32 / G;  // gather steps of a full chunk
     static_assert(STEPS % (2 * U) == 0, "U must divide the gather steps of a chunk in two groups");
+    static_assert(!GB || G <= 2, "GAT backward edge dots: full warp or PAIR only");
+    constexpr bool PAIR = (G == 2);
     // lanes past F read column 0 (a valid address); their results are never stored
     const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
     const unsigned row_bytes = (unsigned)a.ldx * 4u;
@@ -409,7 +419,7 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     const int32_t *__restrict__ ci = a.colidx + e0;
     const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
     const int len = (int)(e1 - e0);
-    const int half = PAIR ? (lane >> 4) : 0;
+    const int grp = lane / (32 / G);  // lane group (G > 1)
     Vec<VEC> ac[2];
 #pragma unroll
     for (int c = 0; c < VEC; ++c) ac[0].v[c] = ac[1].v[c] = 0.f;
@@ -468,29 +478,29 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             DotTree dt_;      // OP_GATB (full chunk): pending butterfly levels
             if (n0 == 32) {
                 // full chunk: fully unrolled, compile-time shuffle lanes, no guards
-                issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, 0, 32, half, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, G, false>(base, row_bytes, 0, 32, grp, u0, c_l, xa, ca);
 #pragma unroll
                 for (int j = 0; j < STEPS; j += 2 * U) {
-                    issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, j + U, 32, half, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, PAIR, false, 0>(j, 32, half, xa, ca, ac);
+                    issue_group<VEC, U, HASC, G, false>(base, row_bytes, j + U, 32, grp, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, G, false, 0>(j, 32, grp, xa, ca, ac);
                     if constexpr (GB) dot_tree<VEC, U, PAIR>(j, lane, xa, xu, dt_, gout + off);
                     if (j + 2 * U < STEPS)
-                        issue_group<VEC, U, HASC, PAIR, false>(base, row_bytes, j + 2 * U, 32, half, u0, c_l, xa, ca);
-                    consume_group<VEC, U, HASC, PAIR, false, U>(j + U, 32, half, xb, cb, ac);
+                        issue_group<VEC, U, HASC, G, false>(base, row_bytes, j + 2 * U, 32, grp, u0, c_l, xa, ca);
+                    consume_group<VEC, U, HASC, G, false, U>(j + U, 32, grp, xb, cb, ac);
                     if constexpr (GB) dot_tree<VEC, U, PAIR>(j + U, lane, xb, xu, dt_, gout + off);
                 }
             } else {
                 // partial chunk (n0 is warp-uniform: the guards never diverge)
-                const int steps = PAIR ? (n0 + 1) >> 1 : n0;
-                issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, 0, n0, half, u0, c_l, xa, ca);
+                const int steps = (n0 + G - 1) / G;
+                issue_group<VEC, U, HASC, G, true>(base, row_bytes, 0, n0, grp, u0, c_l, xa, ca);
                 for (int j = 0; j < steps; j += 2 * U) {
                     const bool more = j + U < steps;
-                    if (more) issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, j + U, n0, half, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, PAIR, true, 0>(j, n0, half, xa, ca, ac);
+                    if (more) issue_group<VEC, U, HASC, G, true>(base, row_bytes, j + U, n0, grp, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, G, true, 0>(j, n0, grp, xa, ca, ac);
                     if constexpr (GB) dot_group<VEC, U, PAIR, true>(j, n0, lane, xa, xu, g_l);
                     if (j + 2 * U < steps)
-                        issue_group<VEC, U, HASC, PAIR, true>(base, row_bytes, j + 2 * U, n0, half, u0, c_l, xa, ca);
-                    if (more) consume_group<VEC, U, HASC, PAIR, true, U>(j + U, n0, half, xb, cb, ac);
+                        issue_group<VEC, U, HASC, G, true>(base, row_bytes, j + 2 * U, n0, grp, u0, c_l, xa, ca);
+                    if (more) consume_group<VEC, U, HASC, G, true, U>(j + U, n0, grp, xb, cb, ac);
                     if constexpr (GB)
                         if (more) dot_group<VEC, U, PAIR, true>(j + U, n0, lane, xb, xu, g_l);
                 }
@@ -505,11 +515,18 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             d0 = d1;
         }
     }
-    // even + odd (in PAIR mode the odd chain lives in the other half-warp)
+    // even + odd (G = 2: the odd chain lives in the other half-warp); G > 2:
+    // the group chains added by a fixed butterfly
 #pragma unroll
     for (int c = 0; c < VEC; ++c) {
-        if constexpr (PAIR) acc.v[c] = ac[0].v[c] + __shfl_xor_sync(FULL, ac[0].v[c], 16);
-        else acc.v[c] = ac[0].v[c] + ac[1].v[c];
+        if constexpr (G > 1) {
+            float x = ac[0].v[c];
+#pragma unroll
+            for (int o = 16; o >= 32 / G; o >>= 1) x += __shfl_xor_sync(FULL, x, o);
+            acc.v[c] = x;
+        } else {
+            acc.v[c] = ac[0].v[c] + ac[1].v[c];
+        }
     }
 }
 
@@ -989,31 +1006,33 @@ __device__ __forceinline__ void store_out(const AggArgs &a, int64_t r, int col, 
     }
 }
 
-// Column of this lane's 4-float vector in strip s (PAIR: 64-column strips,
-// lanes l and l+16 share a column), and whether this lane stores it.
-template <int VEC, bool PAIR>
+// Column of this lane's vector in strip s (G > 1: strips of 32/G lanes x VEC
+// columns, lanes l and l + 32/G share a column; PAIR = 64-column strips), and
+// whether this lane stores it.
+template <int VEC, int G>
 __device__ __forceinline__ int strip_col(const AggArgs &a, int s, int lane) {
-    return PAIR ? s * 64 + (lane & 15) * 4 : s * a.lps * VEC + lane * VEC;
+    constexpr int LG = 32 / G;
+    return (G > 1) ? s * LG * VEC + (lane % LG) * VEC : s * a.lps * VEC + lane * VEC;
 }
 // Whether this lane's column of the strip exists (narrow strips leave lanes
 // >= lps idle; they gather column 0 of the same row, a sector already fetched).
-template <bool PAIR>
+template <int G>
 __device__ __forceinline__ bool in_strip(const AggArgs &a, int lane, int col) {
-    return (PAIR || lane < a.lps) && col < a.F;
+    return (G > 1 || lane < a.lps) && col < a.F;
 }
-template <bool PAIR>
+template <int G>
 __device__ __forceinline__ bool stores(int lane) {
-    return !PAIR || lane < 16;
+    return G == 1 || lane < 32 / G;
 }
 
 // NEXT-3: the strip's partial dots of a finished row vector with att_l, att_r
 // (per-lane fma over the vector, butterfly over the warp; lane 0 stores).
-template <int VEC, bool PAIR>
+template <int VEC, int G>
 __device__ __forceinline__ void project_row(const AggArgs &a, int64_t r, int s, int col, bool active,
                                             const Vec<VEC> &y, int lane) {
     if (a.proj == nullptr) return;
     float pl = 0.f, pr = 0.f;
-    if (active && stores<PAIR>(lane)) {
+    if (active && stores<G>(lane)) {
 #pragma unroll
         for (int c = 0; c < VEC; ++c) {
             if (col + c < a.F) {
@@ -1046,7 +1065,7 @@ __device__ __forceinline__ void gatb_self(const AggArgs &a, int64_t r, int s, in
 }
 
 // A regular work unit: whole rows [r0, r1), feature strips [s0, s1).
-template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0, int s1,
                                         int lane) {
     for (int rb = r0; rb < r1; rb += 31) {
@@ -1064,8 +1083,8 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
             const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
             const int64_t r = rb + k;
             for (int s = s0; s < s1; ++s) {
-                const int col = strip_col<VEC, PAIR>(a, s, lane);
-                const bool active = in_strip<PAIR>(a, lane, col);
+                const int col = strip_col<VEC, G>(a, s, lane);
+                const bool active = in_strip<G>(a, lane, col);
                 Vec<VEC> acc;
 #pragma unroll
                 for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
@@ -1094,12 +1113,12 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                     Vec<VEC> xu;
                     float *gout = nullptr;
                     gatb_self<VEC, OP>(a, r, s, e0, col, active, xu, gout);
-                    reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den,
+                    reduce_edges<VEC, OP, COEF, U, G>(a, e0, e1, col, active, er_v, lane, acc, m, den,
                                                          xu, gout);
                 }
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
-                if (active && stores<PAIR>(lane)) store_out<VEC>(a, r, col, y);
-                project_row<VEC, PAIR>(a, r, s, col, active, y, lane);
+                if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
+                project_row<VEC, G>(a, r, s, col, active, y, lane);
             }
         }
     }
@@ -1108,7 +1127,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
 // One C-edge chunk of hub h (a8), feature strips [s0, s1).  The last chunk of
 // the hub to finish these strips merges all its partials in chunk order and
 // writes the row.  Tickets (and GAT (m, den) pairs) are kept per panel s0.
-template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int s0, int s1,
                                              int lane) {
     const int r = __ldg(a.hub_row + h);
@@ -1125,8 +1144,8 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
     float *md = a.md + 2 * (int64_t)s0 * a.n_chunks * mdh;
     int32_t *ticket = a.hub_ticket + (int64_t)s0 * a.n_hubs + h;
     for (int s = s0; s < s1; ++s) {
-        const int col = strip_col<VEC, PAIR>(a, s, lane);
-        const bool active = in_strip<PAIR>(a, lane, col);
+        const int col = strip_col<VEC, G>(a, s, lane);
+        const bool active = in_strip<G>(a, lane, col);
         Vec<VEC> acc;
 #pragma unroll
         for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
@@ -1151,10 +1170,10 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
             Vec<VEC> xu;
             float *gout = nullptr;
             gatb_self<VEC, OP>(a, r, s, e0, col, active, xu, gout);
-            reduce_edges<VEC, OP, COEF, U, PAIR>(a, e0, e1, col, active, er_v, lane, acc, m, den, xu,
+            reduce_edges<VEC, OP, COEF, U, G>(a, e0, e1, col, active, er_v, lane, acc, m, den, xu,
                                                  gout);
         }
-        if (active && stores<PAIR>(lane)) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
+        if (active && stores<G>(lane)) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
         if constexpr (OP == OP_GAT)
             if (s == s0 && lane == 0) {
                 md[2 * (int64_t)slot] = m;
@@ -1178,8 +1197,8 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         }
     }
     for (int s = s0; s < s1; ++s) {
-        const int col = strip_col<VEC, PAIR>(a, s, lane);
-        const bool active = in_strip<PAIR>(a, lane, col);
+        const int col = strip_col<VEC, G>(a, s, lane);
+        const bool active = in_strip<G>(a, lane, col);
         // OP_GATH: the lane's (up to two) heads and their merged softmax states
         int64_t mA = 0, mB = 0;
         int split = VEC;
@@ -1229,8 +1248,8 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
         } else {
             y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
         }
-        if (active && stores<PAIR>(lane)) store_out<VEC>(a, r, col, y);
-        if constexpr (OP != OP_GATH) project_row<VEC, PAIR>(a, r, s, col, active, y, lane);
+        if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
+        if constexpr (OP != OP_GATH) project_row<VEC, G>(a, r, s, col, active, y, lane);
     }
     if (lane == 0) *ticket = 0;  // self-reset for the next launch
 }
@@ -1238,7 +1257,7 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
 // Work item i: task-major (all strips of task i) or, in panel mode, strip
 // s = i / n_tasks of task i % n_tasks, so that all warps sweep one L2-resident
 // feature panel of X at a time.
-template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
     int64_t t = i;
     int s0 = 0, s1 = a.n_strips;
@@ -1248,8 +1267,8 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
         s1 = s0 + 1;
     }
     const int2 tk = a.tasks[t];
-    if (tk.y >= 0) do_unit<VEC, OP, COEF, U, ASYNC, PAIR>(a, tk.x, tk.y, s0, s1, lane);
-    else do_hub_chunk<VEC, OP, COEF, U, ASYNC, PAIR>(a, tk.x, -tk.y - 1, s0, s1, lane);
+    if (tk.y >= 0) do_unit<VEC, OP, COEF, U, ASYNC, G>(a, tk.x, tk.y, s0, s1, lane);
+    else do_hub_chunk<VEC, OP, COEF, U, ASYNC, G>(a, tk.x, -tk.y - 1, s0, s1, lane);
 }
 
 // Resident CTAs per SM the kernel is compiled for (register budget).  The
@@ -1264,12 +1283,12 @@ constexpr int min_blocks(int op, int coef, bool async) {
                        ? TLP_MINB_LIGHT : TLP_MINB;
 }
 
-template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void agg_body(const AggArgs &a) {
     const int lane = threadIdx.x & 31;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (a.sched == S_HARDWARE) {  // one warp per item
-        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC, PAIR>(a, wid, lane);
+        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC, G>(a, wid, lane);
         if (a.n_dests > 0) __threadfence_system();
         return;
     }
@@ -1280,7 +1299,7 @@ __device__ __forceinline__ void agg_body(const AggArgs &a) {
         unsigned long long v = 0;
         if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned long long)a.step);
         const int64_t tend = min(t + a.step, a.n_items);
-        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, PAIR>(a, tt, lane);
+        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, G>(a, tt, lane);
         if (a.sched == S_DYNAMIC) t = stride + (int64_t)__shfl_sync(FULL, v, 0);
         else t += stride;
     }
@@ -1296,9 +1315,9 @@ __device__ __forceinline__ void agg_body(const AggArgs &a) {
     }
 }
 
-template <int VEC, int OP, int COEF, int U, bool ASYNC, bool PAIR>
+template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC)) k_agg(const AggArgs a) {
-    agg_body<VEC, OP, COEF, U, ASYNC, PAIR>(a);
+    agg_body<VEC, OP, COEF, U, ASYNC, G>(a);
 }
 
 // ------------------------------------------------------------- dispatch --
@@ -1307,44 +1326,49 @@ constexpr int kU = TLP_U;  // source rows per gather group (2 groups in flight)
 
 typedef void (*KernelFn)(const AggArgs);
 
-template <int VEC, bool ASYNC, bool PAIR>
+template <int VEC, bool ASYNC, int G>
 static KernelFn pick(int op, int coef) {
     if (op == OP_GCN) {
         switch (coef) {
-            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU, ASYNC, PAIR>;
-            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU, ASYNC, PAIR>;
-            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU, ASYNC, PAIR>;
-            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU, ASYNC, PAIR>;
+            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU, ASYNC, G>;
+            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU, ASYNC, G>;
+            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU, ASYNC, G>;
+            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU, ASYNC, G>;
         }
     }
     if (op == OP_GIN)
-        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC, PAIR>
-                             : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC, PAIR>;
-    if (op == OP_SAGE) return k_agg<VEC, OP_SAGE, COEF_NONE, kU, ASYNC, PAIR>;
-    if constexpr (!ASYNC)
-        if (op == OP_GATB) return k_agg<VEC, OP_GATB, COEF_W, kU, false, PAIR>;
-    return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC, PAIR>;
+        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC, G>
+                             : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC, G>;
+    if (op == OP_SAGE) return k_agg<VEC, OP_SAGE, COEF_NONE, kU, ASYNC, G>;
+    if constexpr (!ASYNC && G <= 2)
+        if (op == OP_GATB) return k_agg<VEC, OP_GATB, COEF_W, kU, false, G>;
+    return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC, G>;
 }
 
 // multi-head GAT: full-warp register path or cp.async ring
 static KernelFn pick_mh(int vec, bool async_path) {
     if (async_path)
-        return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, true, false>
-                        : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, true, false>
-                                   : k_agg<1, OP_GATH, COEF_NONE, kU, true, false>;
-    return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, false, false>
-                    : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, false, false>
-                               : k_agg<1, OP_GATH, COEF_NONE, kU, false, false>;
+        return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, true, 1>
+                        : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, true, 1>
+                                   : k_agg<1, OP_GATH, COEF_NONE, kU, true, 1>;
+    return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, false, 1>
+                    : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, false, 1>
+                               : k_agg<1, OP_GATH, COEF_NONE, kU, false, 1>;
 }
 
-// gather path: 0 register (full warp), 1 cp.async ring, 2 register half-warp PAIR (VEC = 4)
-static KernelFn pick_kernel(int path, int vec, int op, int coef) {
-    if (path == 2) return pick<4, false, true>(op, coef);
+// gather path: 0 register (full warp), 1 cp.async ring, 2 register with G
+// lane groups (G = 2: PAIR half-warps; 4, 8: narrow rows; VEC = 4)
+static KernelFn pick_kernel(int path, int vec, int op, int coef, int groups) {
+    if (path == 2) {
+        if (groups == 8) return pick<4, false, 8>(op, coef);
+        if (groups == 4) return pick<4, false, 4>(op, coef);
+        return pick<4, false, 2>(op, coef);
+    }
     if (path == 1)
-        return vec == 4 ? pick<4, true, false>(op, coef) : vec == 2 ? pick<2, true, false>(op, coef)
-                                                                   : pick<1, true, false>(op, coef);
-    return vec == 4 ? pick<4, false, false>(op, coef) : vec == 2 ? pick<2, false, false>(op, coef)
-                                                                 : pick<1, false, false>(op, coef);
+        return vec == 4 ? pick<4, true, 1>(op, coef) : vec == 2 ? pick<2, true, 1>(op, coef)
+                                                               : pick<1, true, 1>(op, coef);
+    return vec == 4 ? pick<4, false, 1>(op, coef) : vec == 2 ? pick<2, false, 1>(op, coef)
+                                                             : pick<1, false, 1>(op, coef);
 }
 
 static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
@@ -1889,7 +1913,23 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             else if (512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
         }
     }
-    const int strip_w = pair ? 64 : lps * vec;
+    // Lane groups: G = 2 for the 64-column PAIR
+    // strips; for narrow rows (F/4 vectors fill at most half a warp) G = 2, 4
+    // or 8 groups of 32/G lanes each gather their own edge, so every warp
+    // instruction still moves up to 512 bytes (F = 32: 4 rows of 128 B).
+    // TLP_GROUPS=1|2|4|8 overrides.
+    int groups = pair ? 2 : 1;
+    if (!panel && !pair && lps == 32 && vec == 4 && op != OP_GATH) {
+        const int64_t nv = (r.F + 3) / 4;
+        groups = nv <= 4 ? 8 : nv <= 8 ? 4 : nv <= 16 ? 2 : 1;
+    }
+    if (const char *e = getenv("TLP_GROUPS")) {
+        const int gq = atoi(e);
+        if ((gq == 1 || gq == 2 || gq == 4 || gq == 8) && vec == 4 && lps == 32 && op != OP_GATH)
+            groups = gq;
+    }
+    if (op == OP_GATB && groups > 2) groups = 2;  // the edge-dot trees exist for G <= 2
+    const int strip_w = groups > 1 ? (32 / groups) * vec : lps * vec;
     const int n_strips = (int)((r.F + strip_w - 1) / strip_w);
     // Few tasks for the resident warps (small graphs): split every task into its
     // strips as separate work items too, so all SMs get work.
@@ -2036,8 +2076,8 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         if (!strcmp(e, "reg")) async_path = false;
         else if (!strcmp(e, "async")) async_path = true;
     }
-    if (pair || r.op == OP_GATB) async_path = false;  // OP_GATB: register path only
-    const int path = pair ? 2 : (async_path ? 1 : 0);
+    if (groups > 1 || r.op == OP_GATB) async_path = false;  // OP_GATB: register path only
+    const int path = groups > 1 ? 2 : (async_path ? 1 : 0);
     // hot-source L2 policy: cp.async path only (rows streamed from HBM)
     if (async_path && r.op != OP_GATH && r.op != OP_GATB) {
         unsigned thr = 0;
@@ -2050,7 +2090,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             if (const char *e = getenv("TLP_HOT_COLD")) a.cold_first = atoi(e);
         }
     }
-    KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, op, coef);
+    KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, op, coef, groups);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
     size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;

@@ -1063,3 +1063,74 @@ def test_gat_alpha_mode_pubmed_all_rows(tlp, monkeypatch):
     Y = g.gat(_t(X), _t(el), _t(er), synth.SLOPE, F=cfg["F"])
     _check("pubmed alpha gat", Y, oracle.gat(rp, ci, X, el, er, synth.SLOPE, F=cfg["F"]))
     g.close()
+
+
+# ------------------------------------------- lane groups (narrow rows, G) --
+
+@pytest.mark.parametrize("groups", ["1", "2", "4", "8"])
+@pytest.mark.parametrize("F,ld", [(4, 4), (13, 16), (16, 16), (30, 32), (32, 32), (64, 64), (100, 100)])
+def test_lane_groups_parity(tlp, monkeypatch, groups, F, ld):
+    """Every lane-group count G (32/G lanes per edge, G edges per warp
+    instruction) against the oracle, all ops, hubs split, ragged chunks; F
+    wider than a group's 4(32/G) columns runs as several strips."""
+    monkeypatch.setenv("TLP_GROUPS", groups)
+    n = 700
+    deg = np.minimum((1500 / (np.arange(n) + 1) ** 0.7).astype(int) + 1, 900)
+    rp, ci = synth.power_law_rows(n, np.random.default_rng(F).permutation(deg), n, F + 7)
+    _run_all(tlp, rp, ci, n, F, ld, opts=dict(hub_threshold=100, hub_chunk=40), seed=F,
+             ops=("gcn_none", "gcn_both", "gin", "gat"))
+    _run_all(tlp, rp, ci, n, F, ld, opts=dict(hub_threshold=100, hub_chunk=40), seed=F + 1,
+             nonneg=True, ops=("gcn_right", "gat"))
+
+
+@pytest.mark.parametrize("F", [16, 32])
+def test_lane_groups_bitwise_across_schedules_and_partitions(tlp, monkeypatch, F):
+    """The automatic G for narrow rows (F = 16: 8 groups, F = 32: 4) is a
+    function of F only: every schedule, launch geometry and row partition
+    gives the same bits."""
+    n = 3000
+    rp, ci = synth.chung_lu(n, 90000, 0.55, 21, device="cpu")
+    Xh = synth.features(n, F, F, seed=9)
+    elh, erh = synth.normal(n, 1), synth.normal(n, 2)
+    X, el, er = _t(Xh), _t(elh), _t(erh)
+    opts = dict(hub_threshold=64, hub_chunk=32)
+    g = tlp.Graph(_t(rp), _t(ci), opts=opts)
+    base = {"gcn": g.gcn(X, "both").clone(), "gin": g.gin(X, 0.1).clone(), "gat": g.gat(X, el, er, 0.2).clone()}
+    _check("groups gcn", base["gcn"], oracle.gcn(rp, ci, Xh, "both"))
+    _check("groups gat", base["gat"], oracle.gat(rp, ci, Xh, elh, erh, 0.2))
+    for sched in ("static", "hardware", "dynamic", "paper"):
+        for wpc, step in ((4, 1), (8, 3), (2, 7)):
+            g.set_schedule(sched, wpc, step)
+            assert torch.equal(g.gcn(X, "both"), base["gcn"]), (sched, wpc, step)
+            assert torch.equal(g.gin(X, 0.1), base["gin"]), (sched, wpc, step)
+            assert torch.equal(g.gat(X, el, er, 0.2), base["gat"]), (sched, wpc, step)
+    b = tlp.tlp_partition_rows(rp, 4)
+    out = {k: torch.full((n, F), float("nan"), device=DEV) for k in base}
+    for k in range(4):
+        h = tlp.tlp_graph_create_rows(_t(rp), _t(ci), int(b[k]), int(b[k + 1]), opts=opts)
+        sl = tlp.Graph(None, None, handle=h)
+        r0, r1 = int(b[k]), int(b[k + 1])
+        if r1 > r0:
+            sl.gcn(X, "both", Y=out["gcn"][r0:r1])
+            sl.gin(X, 0.1, Y=out["gin"][r0:r1])
+            sl.gat(X, el, er, 0.2, Y=out["gat"][r0:r1])
+        sl.close()
+    for k in base:
+        assert torch.equal(out[k], base[k]), k
+    g.close()
+
+
+@pytest.mark.parametrize("F", [16, 32, 64])
+def test_lane_groups_gat_backward_and_epilogue(tlp, F):
+    """Narrow rows through the fused layer epilogue (bias + ELU) and the GAT
+    backward (its edge-dot trees cap G at 2) against the oracle."""
+    n = 900
+    rp, ci = synth.chung_lu(n, 20000, 0.5, 23, device="cpu")
+    Xh = synth.features(n, F, F, seed=3)
+    b = synth.normal(F, 4) * 0.5
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
+    Y = g.aggregate("gcn", _t(Xh), norm="both", bias=_t(b), act="elu", act_param=1.0, F=F)
+    ref = oracle.gcn(rp, ci, Xh, "both", F=F)
+    _check("groups gcn+elu", Y, oracle.epilogue(ref[0], ref[1], b, "elu", 1.0))
+    g.close()
+    _gat_bwd_case(tlp, rp, ci, n, F, F, seed=F)
