@@ -1880,7 +1880,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // slice fits in 60% of L2, else 128 columns (full warp, LDG.128).  The
     // reduction order is the canonical two-chain order in every case, so panel
     // mode and strip width never change a single output bit.
-    int panel = 0, pair = 0;
+    int panel = 0, pair = 0;  // pair: lane groups of a panel strip (0: none)
     int lps = 32;  // lanes per full-warp strip
     bool panel_off = false;
     {
@@ -1894,9 +1894,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             panel = 1;
         } else if (mode == 64 && vec == 4 && r.op != OP_GATH) {
             panel = 1;
-            pair = 1;
+            pair = 2;
         } else if (mode == 64 && vec == 2) {
             panel = 1;
+        } else if ((mode == 32 || mode == 16) && vec == 4 && r.op != OP_GATH) {
+            panel = 1;  // lane-group strips: 32 columns = 4 groups of 8 lanes, 16 = 8 of 4
+            pair = 128 / mode;
         } else if (mode == 32) {
             panel = 1;
             vec = 1;
@@ -1908,7 +1911,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             // keeps the wider 128-column strips (measured)
             if (op != OP_GAT && op != OP_GATH && 256.0 * g->n_src <= budget) {
                 panel = 1;
-                pair = 1;
+                pair = 2;
             }
             else if (512.0 * g->n_src <= (double)g->l2_bytes) panel = 1;
         }
@@ -1918,7 +1921,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // or 8 groups of 32/G lanes each gather their own edge, so every warp
     // instruction still moves up to 512 bytes (F = 32: 4 rows of 128 B).
     // TLP_GROUPS=1|2|4|8 overrides.
-    int groups = pair ? 2 : 1;
+    int groups = pair ? pair : 1;
     if (!panel && !pair && lps == 32 && vec == 4 && op != OP_GATH) {
         const int64_t nv = (r.F + 3) / 4;
         groups = nv <= 4 ? 8 : nv <= 8 ? 4 : nv <= 16 ? 2 : 1;

@@ -14,9 +14,14 @@ el = torch.from_numpy(synth.normal(n, 2)).cuda(); er = torch.from_numpy(synth.no
 g = tlp.Graph(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), opts=dict(hub_threshold=64, hub_chunk=32))
 for path in ("reg", "async"):
     os.environ["TLP_GATHER"] = path
-    for panel in ("0", "64", "128"):
+    for panel in ("0", "16", "32", "64", "128"):
         os.environ["TLP_PANEL"] = panel
         g.gcn(X, "both", F=150); g.gin(X, 0.1, F=150); g.gat(X, el, er, 0.2, F=150)
+# narrow rows: automatic lane groups (G = 8, 4, 2)
+os.environ.pop("TLP_GATHER"); os.environ.pop("TLP_PANEL")
+for F in (16, 32, 64):
+    Xn = torch.from_numpy(synth.features(n, F, F, seed=F)).cuda()
+    g.gcn(Xn, "both"); g.gin(Xn, 0.1); g.gat(Xn, el, er, 0.2)
 torch.cuda.synchronize()
 g.close()
 print("sanitize target ok")

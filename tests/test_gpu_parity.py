@@ -429,13 +429,20 @@ def test_panel_modes_bitwise(tlp, monkeypatch):
     el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
     g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=64, hub_chunk=32))
     outs = {}
-    for mode in ("0", "32", "64", "128", "-1"):
+    for mode in ("0", "64", "128", "-1"):
         monkeypatch.setenv("TLP_PANEL", mode)
         outs[mode] = (g.gcn(X, "both").clone(), g.gin(X, 0.1).clone(), g.gat(X, el, er, 0.2).clone())
     for mode in outs:
         for a, b in zip(outs[mode], outs["0"]):
             assert torch.equal(a, b), mode
     _check("panel gcn", outs["64"][0], oracle.gcn(rp, ci, Xh, "both"))
+    # 32 / 16-column strips run as 4 / 8 lane groups (their own fixed order)
+    elh, erh = synth.normal(n, 1), synth.normal(n, 2)
+    for mode in ("32", "16"):
+        monkeypatch.setenv("TLP_PANEL", mode)
+        _check("panel%s gcn" % mode, g.gcn(X, "both"), oracle.gcn(rp, ci, Xh, "both"))
+        _check("panel%s gin" % mode, g.gin(X, 0.1), oracle.gin(rp, ci, Xh, 0.1))
+        _check("panel%s gat" % mode, g.gat(X, el, er, 0.2), oracle.gat(rp, ci, Xh, elh, erh, 0.2))
     g.close()
 
 
@@ -1011,9 +1018,12 @@ def test_gat_alpha_mode_bitwise_across_paths(tlp, monkeypatch):
     g = tlp.Graph(_t(rp), _t(ci), opts=opts)
     base = g.gat(X, el, er, 0.2).clone()
     _check("alpha gat", base, oracle.gat(rp, ci, Xh, elh, erh, 0.2))
-    for mode in ("0", "32", "64", "128", "48"):
+    for mode in ("0", "64", "128", "48"):
         monkeypatch.setenv("TLP_PANEL", mode)
         assert torch.equal(g.gat(X, el, er, 0.2), base), mode
+    for mode in ("32", "16"):  # lane-group strips: their own fixed order
+        monkeypatch.setenv("TLP_PANEL", mode)
+        _check("alpha gat panel" + mode, g.gat(X, el, er, 0.2), oracle.gat(rp, ci, Xh, elh, erh, 0.2))
     monkeypatch.setenv("TLP_PANEL", "0")
     for path in ("reg", "async"):
         monkeypatch.setenv("TLP_GATHER", path)
