@@ -1794,17 +1794,20 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         ew = r.alpha;
         coef = COEF_W;
     }
-    // GAT edge-softmax pre-pass: when X does not fit in L2,
-    // k_gat_alpha writes every edge's alpha_e once and the aggregation becomes
-    // the streamed-weight sum sum_e alpha_e X[u_e] (the GCN-NONE kernel with
-    // COEF_W): it takes the 64-column half-warp strips (the online-softmax
-    // kernel would recompute its running state per strip) and needs no
-    // dependent el[u] gather or rescale.  Measured: Reddit 30.0 -> 27.7 ms,
-    // products 10.1 -> 9.9 ms.  TLP_GAT=online|alpha overrides.
+    // GAT edge-softmax pre-pass: when X does not fit in L2 but
+    // its 64-column strips do, k_gat_alpha writes every edge's alpha_e once and
+    // the aggregation becomes the streamed-weight sum sum_e alpha_e X[u_e] (the
+    // GCN-NONE kernel with COEF_W) on the 64-column half-warp panels (the
+    // online-softmax kernel would recompute its running state per strip, so it
+    // needs 128-column strips that do not stay in L2).  Measured: Reddit 30.0
+    // -> 27.7 ms; without panels (products: rows streamed from HBM) the online
+    // kernel stays ahead (9.67 vs 9.82 ms).  TLP_GAT=online|alpha overrides.
     int op = r.op;
     bool gat_alpha = false;
     if (r.op == OP_GAT) {
-        gat_alpha = 4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes;
+        const double budget = 0.6 * (double)g->l2_bytes;
+        gat_alpha = vec == 4 && 4.0 * (double)g->n_src * (double)r.ldx > budget &&
+                    256.0 * (double)g->n_src <= budget;
         if (const char *e = getenv("TLP_GAT")) {
             if (!strcmp(e, "online")) gat_alpha = false;
             else if (!strcmp(e, "alpha")) gat_alpha = true;

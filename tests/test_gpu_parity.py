@@ -403,7 +403,7 @@ def test_config_reddit_gat_sampled(tlp, reddit, monkeypatch, gat_mode):
     g.close()
 
 
-@pytest.mark.parametrize("gat_mode", ["auto", "online"])
+@pytest.mark.parametrize("gat_mode", ["auto", "alpha"])
 def test_config_products_gat_sampled(tlp, monkeypatch, gat_mode):
     if gat_mode != "auto":
         monkeypatch.setenv("TLP_GAT", gat_mode)
