@@ -1785,7 +1785,29 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             ew = g->ew_both;  // weighted: w_e c_out[u] streamed per edge
             coef |= COEF_W;
         } else {
-            prescale = true;  // unweighted: gather X' = c_out (.) X, no edge coefficient
+            // unweighted: when the gathered
+            // rows are L2-served (X fits, or its 64-column panels do), gather
+            // X' = c_out (.) X with no edge coefficient (GIN's register budget);
+            // when they stream from HBM, the extra pass over X (read + write of
+            // n_src x F) costs more than streaming ew_both[e] = c_out[colidx[e]]
+            // (built once per handle).  The choice depends on n_src, ldx and
+            // the L2 size only (never on P or the gather path override).
+            // TLP_BOTH=prescale|edge overrides.
+            const double budget = 0.6 * (double)g->l2_bytes;
+            bool edge = 4.0 * (double)g->n_src * (double)r.ldx > budget &&
+                        256.0 * (double)g->n_src > budget;
+            if (const char *e = getenv("TLP_BOTH")) {
+                if (!strcmp(e, "prescale")) edge = false;
+                else if (!strcmp(e, "edge")) edge = true;
+            }
+            if (edge) {
+                tlp_status st = ensure_edge_both(g, s);
+                if (st != TLP_OK) return st;
+                ew = g->ew_both;
+                coef |= COEF_W;
+            } else {
+                prescale = true;
+            }
         }
     } else if (r.op != OP_GAT && r.op != OP_GATB && g->ew) {
         coef |= COEF_W;

@@ -579,6 +579,21 @@ tlp_status build_transpose(tlp_graph g, cudaStream_t s) {
     return TLP_OK;
 }
 
+tlp_status ensure_edge_both(tlp_graph g, cudaStream_t s) {
+    if (g->ew_both || g->nnz == 0) return TLP_OK;
+    float *p = nullptr;
+    cudaError_t e = cudaMallocAsync((void **)&p, sizeof(float) * g->nnz + 16, s);
+    if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(edge BOTH coefficients)");
+    g->device_bytes += sizeof(float) * g->nnz + 16;
+    const int nsm = g->num_sms > 0 ? g->num_sms : 148;
+    k_edge_both<<<grid_for(g->nnz, nsm), 256, 0, s>>>(g->colidx, g->ew, g->c_out, g->nnz, p);
+    g->launches += 1;
+    e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "k_edge_both launch");
+    g->ew_both = p;
+    return TLP_OK;
+}
+
 tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s) {
     if (bytes <= g->scratch_bytes) return TLP_OK;
     if (g->scratch) {

@@ -103,6 +103,8 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
                              tlp_graph *out);
 
 tlp_status ensure_scratch(tlp_graph g, size_t bytes, cudaStream_t s);
+// unweighted graphs: build ew_both[e] = c_out[colidx[e]] on first use (stream-ordered)
+tlp_status ensure_edge_both(tlp_graph g, cudaStream_t s);
 tlp_status build_transpose(tlp_graph g, cudaStream_t s);
 
 // Enqueue one aggregation kernel; op: 0 GCN, 1 GIN, 2 GAT, 3 GraphSage mean,

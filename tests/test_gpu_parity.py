@@ -1144,3 +1144,34 @@ def test_lane_groups_gat_backward_and_epilogue(tlp, F):
     _check("groups gcn+elu", Y, oracle.epilogue(ref[0], ref[1], b, "elu", 1.0))
     g.close()
     _gat_bwd_case(tlp, rp, ci, n, F, F, seed=F)
+
+
+def test_gcn_both_streamed_edge_coefficients(tlp, monkeypatch):
+    """Unweighted GCN BOTH through the streamed per-edge c_out[u] (the mode
+    used when X's rows stream from HBM): oracle parity, bitwise equal to the
+    weighted path with w = 1, and partition-invariant."""
+    monkeypatch.setenv("TLP_BOTH", "edge")
+    n, F = 2500, 100
+    rp, ci = synth.chung_lu(n, 60000, 0.5, 41, device="cpu")
+    Xh = synth.features(n, F, F, seed=7)
+    X = _t(Xh)
+    opts = dict(hub_threshold=80, hub_chunk=40)
+    g = tlp.Graph(_t(rp), _t(ci), opts=opts)
+    Y = g.gcn(X, "both")
+    _check("edge both", Y, oracle.gcn(rp, ci, Xh, "both"))
+    gw = tlp.Graph(_t(rp), _t(ci), edge_weight=torch.ones(len(ci), device=DEV), opts=opts)
+    assert torch.equal(gw.gcn(X, "both"), Y)
+    for path in ("reg", "async"):
+        monkeypatch.setenv("TLP_GATHER", path)
+        assert torch.equal(g.gcn(X, "both"), Y), path
+    monkeypatch.delenv("TLP_GATHER")
+    b = tlp.tlp_partition_rows(rp, 3)
+    out = torch.full((n, F), float("nan"), device=DEV)
+    for k in range(3):
+        h = tlp.tlp_graph_create_rows(_t(rp), _t(ci), int(b[k]), int(b[k + 1]), opts=opts)
+        sl = tlp.Graph(None, None, handle=h)
+        if b[k + 1] > b[k]:
+            sl.gcn(X, "both", Y=out[int(b[k]):int(b[k + 1])])
+        sl.close()
+    assert torch.equal(out, Y)
+    g.close(); gw.close()
