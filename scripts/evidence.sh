@@ -11,6 +11,10 @@ prof() {  # <regex> <name> <workload>
 export TLP_SYNTH_CACHE=/tmp/tlp_synth
 if [ "$P" = "a" ]; then
   TLP_TRACE_CREATE=1 python bench.py > gpurun_out/$R/bench.json 2> gpurun_out/$R/bench.err
+  # the other configs and context workloads (one line each)
+  for w in products pubmed cora rmat24 reddit_f32 products_f32 reddit_sage products_gat4 reddit_bwd reddit_gat_bwd; do
+    timeout 900 python bench.py --workload $w --no-cpu-baseline > gpurun_out/$R/bench_$w.json 2> gpurun_out/$R/bench_$w.err
+  done
   ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/$R/launches.csv \
       python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
   prof "_ZN3tlp5k_aggILi4ELi0ELi0E" reddit_gcn reddit

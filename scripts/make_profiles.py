@@ -24,6 +24,26 @@ if os.path.exists(bj):
         out.append(f"* {op}: {d['ms_mean']} ms mean, {d['gather_GBs']} GB/s gather-model ({d['frac_of_8TBs']} of 8 TB/s)\n")
     out.append("\n")
 
+# bench lines of the other workloads
+import glob
+extra = sorted(glob.glob(os.path.join(src, "bench_*.json")))
+if extra:
+    out.append("## other workloads (bench.py --workload W, one line each)\n\n")
+    out.append("| workload | ms/step | per op ms (mean) | GB/s gather-model | e2e GB/s | sm MHz |\n|---|---|---|---|---|---|\n")
+    for f in extra:
+        try:
+            b = json.loads(open(f).read().strip().splitlines()[-1])
+        except Exception:
+            continue
+        wl = os.path.basename(f)[6:-5]
+        json.dump(b, open(os.path.join(dst, f"{R}_bench_{wl}.json"), "w"), indent=1)
+        ops = ", ".join(f"{k} {v['ms_mean']}" for k, v in b.get("ops", {}).items())
+        e2e = (b.get("e2e") or {}).get("value")
+        out.append(f"| {wl} | {b['ms_per_step']} | {ops} | {b['value']} | {e2e} | {b['clocks']['sm_mhz']} |\n")
+        if b.get("paper_context"):
+            out.append(f"| ↳ paper V100 (F=32) | | {b['paper_context']['v100_ms']} | B200/V100 {b['paper_context']['b200_over_v100']} | | |\n")
+    out.append("\n")
+
 # launch list: share of each kernel in the step
 lc = os.path.join(src, "launches.csv")
 if os.path.exists(lc):
