@@ -300,7 +300,7 @@ def dataset_graph(name, device=None):
     cdir = _cache_dir()
     if cdir:
         p = os.path.join(cdir, f"{name}_seed{cfg['seed']}")
-        if os.path.exists(p + "_rowptr.npy"):
+        if os.path.exists(p + "_rowptr.npy") and os.path.exists(p + "_colidx.npy"):
             return np.load(p + "_rowptr.npy"), np.load(p + "_colidx.npy")
     if name == "rmat24":
         g = rmat(cfg["scale"], cfg["edge_factor"], cfg["seed"], device=device)
@@ -308,8 +308,12 @@ def dataset_graph(name, device=None):
         g = chung_lu(cfg["n"], cfg["e"], cfg["alpha"], cfg["seed"], device=device)
     if cdir:
         os.makedirs(cdir, exist_ok=True)
-        np.save(p + "_rowptr.npy", g[0])
-        np.save(p + "_colidx.npy", g[1])
+        # atomic per file (several ranks may generate the same graph at once);
+        # colidx lands last, and readers require both files
+        for suffix, arr in (("_rowptr.npy", g[0]), ("_colidx.npy", g[1])):
+            tmp = "%s%s.%d.tmp.npy" % (p, suffix, os.getpid())
+            np.save(tmp, arr)
+            os.replace(tmp, p + suffix)
     return g
 
 
