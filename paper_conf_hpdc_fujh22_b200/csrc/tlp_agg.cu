@@ -1544,92 +1544,206 @@ __global__ void __launch_bounds__(256) k_gat_alpha(const int64_t *__restrict__ r
 //    per-strip dots g_e = dY[v_e] . X[u], one gather of dY per edge;
 //  k_gatb_edges (transposed rows u): dt_e = alpha_e (g_e - S_v) LeakyReLU'(t_e),
 //    del[u] = sum_e dt_e;  k_gatb_der (forward rows v): der[v] = sum_e dt_e.
-// Warp per row, lane-strided edges, butterfly reductions: deterministic.
-__global__ void k_gatb_stats(const int64_t *__restrict__ rowptr, const int32_t *__restrict__ colidx,
-                             int64_t n_dst, const float *__restrict__ el, const float *__restrict__ er,
-                             float slope, const float *__restrict__ dY, int64_t lddy,
-                             const float *__restrict__ Y, int64_t ldy, int64_t F,
-                             float4 *__restrict__ vstat) {
-    const int lane = threadIdx.x & 31;
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n_dst; v += W) {
-        const int64_t e0 = rowptr[v], e1 = rowptr[v + 1];
-        const float er_v = er[v];
+// Row-parallel scalar passes: hub rows (degree > H of the handle whose CSR is
+// walked) get one 256-thread CTA each (blocks [0, n_hubs)), the other rows a
+// warp each; edges are lane-strided with GB_UN independent loads in flight per
+// thread.  Sums use a fixed tree (warp butterfly, then warps in order), so
+// every pass is deterministic.
+constexpr int GB_UN = 4;
+
+template <int NT>
+__device__ __forceinline__ float group_sum(float v, float *red, int tid) {
+    v = warp_sum(v);
+    if constexpr (NT > 32) {
+        __syncthreads();  // red is reused by consecutive reductions
+        if ((tid & 31) == 0) red[tid >> 5] = v;
+        __syncthreads();
+        v = ((tid & 31) < NT / 32) ? red[tid & 31] : 0.f;
+        v = warp_sum(v);
+    }
+    return v;
+}
+template <int NT>
+__device__ __forceinline__ void group_max_sum(float &m, float &z, float *red, int tid) {
+    float M = warp_max(m);
+    float Z = warp_sum(m == -INFINITY ? 0.f : z * __expf(m - M));
+    if constexpr (NT > 32) {
+        __syncthreads();
+        if ((tid & 31) == 0) { red[tid >> 5] = M; red[8 + (tid >> 5)] = Z; }
+        __syncthreads();
+        const float mw = ((tid & 31) < NT / 32) ? red[tid & 31] : -INFINITY;
+        const float zw = ((tid & 31) < NT / 32) ? red[8 + (tid & 31)] : 0.f;
+        M = warp_max(mw);
+        Z = warp_sum(mw == -INFINITY ? 0.f : zw * __expf(mw - M));
+    }
+    m = M;
+    z = Z;
+}
+
+// Dispatch of a row body over the hub CTAs and the warp-per-row blocks.
+#define TLP_ROWS(ROWPTR, NROWS, HUBROW, NHUBS, H, BODY)                                         \
+    do {                                                                                          \
+        __shared__ float red_[16];                                                                \
+        if ((int64_t)blockIdx.x < (NHUBS)) {                                                      \
+            const int64_t row_ = __ldg((HUBROW) + blockIdx.x);                                    \
+            BODY<256>(row_, __ldg((ROWPTR) + row_), __ldg((ROWPTR) + row_ + 1), threadIdx.x, red_); \
+            return;                                                                               \
+        }                                                                                         \
+        const int64_t W_ = ((int64_t)(gridDim.x - (NHUBS)) * blockDim.x) >> 5;                   \
+        for (int64_t v_ = (((int64_t)blockIdx.x - (NHUBS)) * blockDim.x + threadIdx.x) >> 5;      \
+             v_ < (NROWS); v_ += W_) {                                                            \
+            const int64_t a_ = __ldg((ROWPTR) + v_), b_ = __ldg((ROWPTR) + v_ + 1);               \
+            if (b_ - a_ > (H)) continue;                                                          \
+            BODY<32>(v_, a_, b_, threadIdx.x & 31, red_);                                         \
+        }                                                                                         \
+    } while (0)
+
+struct GatbStats {
+    const int32_t *colidx;
+    const float *el, *er, *dY, *Y;
+    float slope;
+    int64_t lddy, ldy, F;
+    float4 *vstat;
+    template <int NT>
+    __device__ __forceinline__ void operator()(int64_t v, int64_t e0, int64_t e1, int tid, float *red) const {
+        const float er_v = __ldg(er + v);
         float m = -INFINITY, z = 0.f;
-        for (int64_t e = e0 + lane; e < e1; e += 32) {
-            const float t = el[colidx[e]] + er_v;
-            const float sc = t >= 0.f ? t : slope * t;
-            if (sc > m) {
-                z = fmaf(z, __expf(m - sc), 1.f);
-                m = sc;
-            } else {
-                z += __expf(sc - m);
+        for (int64_t b = e0 + tid; b < e1; b += (int64_t)NT * GB_UN) {
+            float sc[GB_UN];
+            float mk = -INFINITY;
+#pragma unroll
+            for (int k = 0; k < GB_UN; ++k) {
+                sc[k] = -INFINITY;
+                if (b + k * NT < e1) {
+                    const float t = __ldg(el + __ldg(colidx + b + k * NT)) + er_v;
+                    sc[k] = t >= 0.f ? t : slope * t;
+                }
+                mk = fmaxf(mk, sc[k]);
             }
+            if (mk > m) {
+                z *= __expf(m - mk);
+                m = mk;
+            }
+#pragma unroll
+            for (int k = 0; k < GB_UN; ++k) z += __expf(sc[k] - m);
         }
-        const float M = warp_max(m);
-        const float Z = warp_sum(m == -INFINITY ? 0.f : z * __expf(m - M));
+        group_max_sum<NT>(m, z, red, tid);
         float S = 0.f;
-        for (int64_t f = lane; f < F; f += 32) S = fmaf(dY[v * lddy + f], Y[v * ldy + f], S);
-        S = warp_sum(S);
-        if (lane == 0) vstat[v] = make_float4(er_v, M, Z > 0.f ? 1.0f / Z : 0.f, S);
+        for (int64_t f = tid; f < F; f += NT) S = fmaf(__ldg(dY + v * lddy + f), __ldg(Y + v * ldy + f), S);
+        S = group_sum<NT>(S, red, tid);
+        if (tid == 0) vstat[v] = make_float4(er_v, m, z > 0.f ? 1.0f / z : 0.f, S);
     }
-}
-
-__global__ void k_gatb_alpha(const int64_t *__restrict__ t_rowptr, const int32_t *__restrict__ t_colidx,
-                             int64_t n_src, const float *__restrict__ el,
-                             const float4 *__restrict__ vstat, float slope,
-                             float *__restrict__ alpha) {
-    const int lane = threadIdx.x & 31;
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t u = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; u < n_src; u += W) {
-        const int64_t e0 = t_rowptr[u], e1 = t_rowptr[u + 1];
-        const float el_u = el[u];
-        for (int64_t e = e0 + lane; e < e1; e += 32) {
-            const float4 q = vstat[t_colidx[e]];
-            const float t = el_u + q.x;
-            const float sc = t >= 0.f ? t : slope * t;
-            alpha[e] = __expf(sc - q.y) * q.z;
+};
+struct GatbAlpha {
+    const int32_t *t_colidx;
+    const float *el;
+    const float4 *vstat;
+    float slope;
+    float *alpha;
+    template <int NT>
+    __device__ __forceinline__ void operator()(int64_t u, int64_t e0, int64_t e1, int tid, float *) const {
+        const float el_u = __ldg(el + u);
+        for (int64_t b = e0 + tid; b < e1; b += (int64_t)NT * GB_UN) {
+            float4 q[GB_UN];
+#pragma unroll
+            for (int k = 0; k < GB_UN; ++k)
+                if (b + k * NT < e1) q[k] = __ldg(vstat + __ldg(t_colidx + b + k * NT));
+#pragma unroll
+            for (int k = 0; k < GB_UN; ++k)
+                if (b + k * NT < e1) {
+                    const float t = el_u + q[k].x;
+                    const float sc = t >= 0.f ? t : slope * t;
+                    alpha[b + k * NT] = __expf(sc - q[k].y) * q[k].z;
+                }
         }
     }
-}
-
-__global__ void k_gatb_edges(const int64_t *__restrict__ t_rowptr, const int32_t *__restrict__ t_colidx,
-                             int64_t n_src, const float *__restrict__ el,
-                             const float4 *__restrict__ vstat, const float *__restrict__ alpha,
-                             float slope, const float *__restrict__ gbuf, int n_strips,
-                             int64_t gstride, float *__restrict__ dt, float *__restrict__ del) {
-    const int lane = threadIdx.x & 31;
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t u = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; u < n_src; u += W) {
-        const int64_t e0 = t_rowptr[u], e1 = t_rowptr[u + 1];
-        const float el_u = el[u];
+};
+struct GatbEdges {
+    const int32_t *t_colidx;
+    const float *el;
+    const float4 *vstat;
+    const float *alpha;
+    float slope;
+    const float *gbuf;
+    int n_strips;
+    int64_t gstride;
+    float *dt, *del;
+    template <int NT>
+    __device__ __forceinline__ void operator()(int64_t u, int64_t e0, int64_t e1, int tid, float *red) const {
+        const float el_u = __ldg(el + u);
         float acc = 0.f;
-        for (int64_t e = e0 + lane; e < e1; e += 32) {
-            const float4 q = vstat[t_colidx[e]];
-            const float t = el_u + q.x;
-            float g = 0.f;
-            for (int k = 0; k < n_strips; ++k) g += gbuf[(int64_t)k * gstride + e];
-            const float d = alpha[e] * (g - q.w) * (t >= 0.f ? 1.f : slope);
-            dt[e] = d;
-            acc += d;
+        for (int64_t b = e0 + tid; b < e1; b += (int64_t)NT * GB_UN) {
+            float4 q[GB_UN];
+            float g[GB_UN], al[GB_UN];
+#pragma unroll
+            for (int k = 0; k < GB_UN; ++k) {
+                g[k] = 0.f;
+                if (b + k * NT < e1) {
+                    q[k] = __ldg(vstat + __ldg(t_colidx + b + k * NT));
+                    al[k] = __ldg(alpha + b + k * NT);
+                }
+            }
+            for (int s = 0; s < n_strips; ++s) {  // strip order (deterministic)
+                const float *gs = gbuf + (int64_t)s * gstride;
+#pragma unroll
+                for (int k = 0; k < GB_UN; ++k)
+                    if (b + k * NT < e1) g[k] += __ldcs(gs + b + k * NT);
+            }
+#pragma unroll
+            for (int k = 0; k < GB_UN; ++k)
+                if (b + k * NT < e1) {
+                    const float t = el_u + q[k].x;
+                    const float d = al[k] * (g[k] - q[k].w) * (t >= 0.f ? 1.f : slope);
+                    dt[b + k * NT] = d;
+                    acc += d;
+                }
         }
-        acc = warp_sum(acc);
-        if (lane == 0) del[u] = acc;
+        acc = group_sum<NT>(acc, red, tid);
+        if (tid == 0) del[u] = acc;
     }
-}
-
-__global__ void k_gatb_der(const int64_t *__restrict__ rowptr, int64_t n_dst,
-                           const int32_t *__restrict__ tpos, const float *__restrict__ dt,
-                           float *__restrict__ der) {
-    const int lane = threadIdx.x & 31;
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t v = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; v < n_dst; v += W) {
+};
+struct GatbDer {
+    const int32_t *tpos;
+    const float *dt;
+    float *der;
+    template <int NT>
+    __device__ __forceinline__ void operator()(int64_t v, int64_t e0, int64_t e1, int tid, float *red) const {
         float acc = 0.f;
-        for (int64_t e = rowptr[v] + lane; e < rowptr[v + 1]; e += 32) acc += dt[tpos[e]];
-        acc = warp_sum(acc);
-        if (lane == 0) der[v] = acc;
+        for (int64_t b = e0 + tid; b < e1; b += (int64_t)NT * GB_UN * 2) {
+            float d[2 * GB_UN];
+#pragma unroll
+            for (int k = 0; k < 2 * GB_UN; ++k)
+                d[k] = (b + k * NT < e1) ? __ldcg(dt + __ldg(tpos + b + k * NT)) : 0.f;
+#pragma unroll
+            for (int k = 0; k < 2 * GB_UN; ++k) acc += d[k];
+        }
+        acc = group_sum<NT>(acc, red, tid);
+        if (tid == 0) der[v] = acc;
     }
+};
+
+#define TLP_BODY(F) F.template operator()
+__global__ void __launch_bounds__(256) k_gatb_stats(GatbStats p, const int64_t *__restrict__ rowptr,
+                                                    int64_t n, const int32_t *__restrict__ hub_row,
+                                                    int64_t n_hubs, int64_t H) {
+    TLP_ROWS(rowptr, n, hub_row, n_hubs, H, TLP_BODY(p));
 }
+__global__ void __launch_bounds__(256) k_gatb_alpha(GatbAlpha p, const int64_t *__restrict__ rowptr,
+                                                    int64_t n, const int32_t *__restrict__ hub_row,
+                                                    int64_t n_hubs, int64_t H) {
+    TLP_ROWS(rowptr, n, hub_row, n_hubs, H, TLP_BODY(p));
+}
+__global__ void __launch_bounds__(256) k_gatb_edges(GatbEdges p, const int64_t *__restrict__ rowptr,
+                                                    int64_t n, const int32_t *__restrict__ hub_row,
+                                                    int64_t n_hubs, int64_t H) {
+    TLP_ROWS(rowptr, n, hub_row, n_hubs, H, TLP_BODY(p));
+}
+__global__ void __launch_bounds__(256) k_gatb_der(GatbDer p, const int64_t *__restrict__ rowptr,
+                                                  int64_t n, const int32_t *__restrict__ hub_row,
+                                                  int64_t n_hubs, int64_t H) {
+    TLP_ROWS(rowptr, n, hub_row, n_hubs, H, TLP_BODY(p));
+}
+#undef TLP_BODY
 
 // ---- hot-source L2 policy ----------------
 // Out-degree class of a source: 0 for d <= 1, else min(31, floor(2 log2 d))
@@ -2249,8 +2363,9 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
     float *alpha = reinterpret_cast<float *>((char *)g->bwd + vbytes + ebytes);
     const int nsm = g->num_sms > 0 ? g->num_sms : 148;
     if (n_dst) {
-        k_gatb_stats<<<nsm * 8, 256, 0, s>>>(g->rowptr, g->colidx, n_dst, el, er, slope, dY, lddy, Y,
-                                             ldy, F, vstat);
+        GatbStats p{g->colidx, el, er, dY, Y, slope, lddy, ldy, F, vstat};
+        k_gatb_stats<<<(unsigned)(g->n_hubs + nsm * 8), 256, 0, s>>>(p, g->rowptr, n_dst, g->hub_row,
+                                                                   g->n_hubs, g->H);
         g->launches += 1;
         TLP_CUDA_TRY(cudaGetLastError());
     }
@@ -2258,7 +2373,11 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
         if (n_dst) TLP_CUDA_TRY(cudaMemsetAsync(der, 0, sizeof(float) * n_dst, s));
         return TLP_OK;
     }
-    k_gatb_alpha<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, slope, alpha);
+    {
+        GatbAlpha p{g->t->colidx, el, vstat, slope, alpha};
+        k_gatb_alpha<<<(unsigned)(g->t->n_hubs + nsm * 8), 256, 0, s>>>(p, g->t->rowptr, n_src,
+                                                                      g->t->hub_row, g->t->n_hubs, g->t->H);
+    }
     g->launches += 1;
     TLP_CUDA_TRY(cudaGetLastError());
     AggRequest r;
@@ -2272,12 +2391,17 @@ tlp_status tlp_gat_backward(tlp_graph g, const float *X, int64_t F, int64_t ldx,
     r.n_strips_out = &n_strips;
     tlp_status st = aggregate(g->t, r, s);
     if (st != TLP_OK) return st;
-    k_gatb_edges<<<nsm * 8, 256, 0, s>>>(g->t->rowptr, g->t->colidx, n_src, el, vstat, alpha, slope,
-                                         gbuf, n_strips, nnz, dt, del);
+    {
+        GatbEdges p{g->t->colidx, el, vstat, alpha, slope, gbuf, n_strips, nnz, dt, del};
+        k_gatb_edges<<<(unsigned)(g->t->n_hubs + nsm * 8), 256, 0, s>>>(p, g->t->rowptr, n_src,
+                                                                      g->t->hub_row, g->t->n_hubs, g->t->H);
+    }
     g->launches += 1;
     TLP_CUDA_TRY(cudaGetLastError());
     if (n_dst) {
-        k_gatb_der<<<nsm * 8, 256, 0, s>>>(g->rowptr, n_dst, g->tpos, dt, der);
+        GatbDer p{g->tpos, dt, der};
+        k_gatb_der<<<(unsigned)(g->n_hubs + nsm * 8), 256, 0, s>>>(p, g->rowptr, n_dst, g->hub_row,
+                                                                 g->n_hubs, g->H);
         g->launches += 1;
         TLP_CUDA_TRY(cudaGetLastError());
     }
