@@ -2243,7 +2243,10 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (sched == S_HARDWARE) {
         blocks = (a.n_items + wpc - 1) / wpc;
     } else {
-        blocks = (int64_t)occupancy_blocks(fn, threads, smem) * g->num_sms;
+        int per_sm = occupancy_blocks(fn, threads, smem);
+        if (const char *e = getenv("TLP_CTAS"))  // measurement: cap resident CTAs per SM
+            if (atoi(e) > 0) per_sm = std::min(per_sm, atoi(e));
+        blocks = (int64_t)per_sm * g->num_sms;
         int64_t need = (a.n_items + (int64_t)wpc * step - 1) / ((int64_t)wpc * step);
         if (blocks > need) blocks = need;  // tiny graphs: do not launch idle warps
     }
