@@ -250,7 +250,24 @@ __device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, un
 //              partition-invariant; G <= 2 paths are bitwise identical to each
 //              other (R10).
 
-template <int VEC, int U, bool HASC, int G, bool CLAMP>
+// Edge coefficients of lane-group gathers (G > 1) live in shared memory: the
+// chunk's 32 coefficients are written once per chunk and read (broadcast) at
+// consume time, so no coefficient register is held across the gather latency
+// and the streamed-weight sums (GAT alpha mode, weighted GCN/GIN) fit 64
+// registers, i.e. 4 CTAs / 32 warps per SM like the coefficient-free sums
+// (measured: Reddit GAT 26.46 -> 24.42 ms; at 3 CTAs/SM 25.65 ms).
+#ifndef TLP_SMEMC
+#define TLP_SMEMC 1
+#endif
+#ifndef TLP_MINB_SMC
+#define TLP_MINB_SMC 4   // resident CTAs for the shared-memory-coefficient kernels
+#endif
+__device__ __forceinline__ float *chunk_coef_smem() {
+    __shared__ float tlp_cw[TLP_MAXT / 32][32];
+    return tlp_cw[threadIdx.x >> 5];
+}
+
+template <int VEC, int U, bool HASC, int G, bool CLAMP, bool SMC = false>
 __device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes, int j, int n,
                                             int grp, int u_l, float c_l, Vec<VEC> (&xv)[U],
                                             float (&ck)[U]) {
@@ -259,23 +276,26 @@ __device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes
         int p = G * (j + k) + grp;
         if constexpr (CLAMP) p = min(p, n - 1);  // duplicate of a line in flight
         const unsigned u = (unsigned)__shfl_sync(FULL, u_l, p);
-        if constexpr (HASC) ck[k] = __shfl_sync(FULL, c_l, p);
+        if constexpr (HASC && !SMC) ck[k] = __shfl_sync(FULL, c_l, p);
         xv[k] = ld_vec<VEC>(row_ptr(base, u, row_bytes));
     }
 }
 
 // PHASE: parity of the group's first step (the caller's j is a multiple of 2U).
-template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE>
+template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE, bool SMC = false>
 __device__ __forceinline__ void consume_group(int j, int n, int grp, const Vec<VEC> (&xv)[U],
-                                              const float (&ck)[U], Vec<VEC> (&ac)[2]) {
+                                              const float (&ck)[U], Vec<VEC> (&ac)[2],
+                                              const float *cw = nullptr) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
         const int p = G * (j + k) + grp;
         const int ch = (G > 1) ? 0 : ((PHASE + k) & 1);
         if (!GUARD || p < n) {
+            float cv = 0.f;
+            if constexpr (HASC) cv = SMC ? cw[p] : ck[k];
 #pragma unroll
             for (int c = 0; c < VEC; ++c) {
-                if constexpr (HASC) ac[ch].v[c] = fmaf(ck[k], xv[k].v[c], ac[ch].v[c]);
+                if constexpr (HASC) ac[ch].v[c] = fmaf(cv, xv[k].v[c], ac[ch].v[c]);
                 else ac[ch].v[c] += xv[k].v[c];
             }
         }
@@ -411,6 +431,8 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     static_assert(STEPS % (2 * U) == 0, "U must divide the gather steps of a chunk in two groups");
     static_assert(!GB || G <= 2, "GAT backward edge dots: full warp or PAIR only");
     constexpr bool PAIR = (G == 2);
+    constexpr bool SMC = TLP_SMEMC && HASC && (G > 1) && !GB;
+    float *cw = SMC ? chunk_coef_smem() : nullptr;
     // lanes past F read column 0 (a valid address); their results are never stored
     const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
     const unsigned row_bytes = (unsigned)a.ldx * 4u;
@@ -472,35 +494,40 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
                 if constexpr (COEF & COEF_COUT) c_l = d0;
                 if constexpr (COEF & COEF_W) c_l *= w0;
             }
+            if constexpr (SMC) {
+                __syncwarp();  // the previous chunk's coefficients are consumed
+                cw[lane] = c_l;
+                __syncwarp();
+            }
             Vec<VEC> xa[U], xb[U];
             float ca[U], cb[U];
             float g_l = 0.f;  // OP_GATB (partial chunk): this strip's dot of edge `lane`
             DotTree dt_;      // OP_GATB (full chunk): pending butterfly levels
             if (n0 == 32) {
                 // full chunk: fully unrolled, compile-time shuffle lanes, no guards
-                issue_group<VEC, U, HASC, G, false>(base, row_bytes, 0, 32, grp, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, 0, 32, grp, u0, c_l, xa, ca);
 #pragma unroll
                 for (int j = 0; j < STEPS; j += 2 * U) {
-                    issue_group<VEC, U, HASC, G, false>(base, row_bytes, j + U, 32, grp, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, G, false, 0>(j, 32, grp, xa, ca, ac);
+                    issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, j + U, 32, grp, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, G, false, 0, SMC>(j, 32, grp, xa, ca, ac, cw);
                     if constexpr (GB) dot_tree<VEC, U, PAIR>(j, lane, xa, xu, dt_, gout + off);
                     if (j + 2 * U < STEPS)
-                        issue_group<VEC, U, HASC, G, false>(base, row_bytes, j + 2 * U, 32, grp, u0, c_l, xa, ca);
-                    consume_group<VEC, U, HASC, G, false, U>(j + U, 32, grp, xb, cb, ac);
+                        issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, j + 2 * U, 32, grp, u0, c_l, xa, ca);
+                    consume_group<VEC, U, HASC, G, false, U, SMC>(j + U, 32, grp, xb, cb, ac, cw);
                     if constexpr (GB) dot_tree<VEC, U, PAIR>(j + U, lane, xb, xu, dt_, gout + off);
                 }
             } else {
                 // partial chunk (n0 is warp-uniform: the guards never diverge)
                 const int steps = (n0 + G - 1) / G;
-                issue_group<VEC, U, HASC, G, true>(base, row_bytes, 0, n0, grp, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, 0, n0, grp, u0, c_l, xa, ca);
                 for (int j = 0; j < steps; j += 2 * U) {
                     const bool more = j + U < steps;
-                    if (more) issue_group<VEC, U, HASC, G, true>(base, row_bytes, j + U, n0, grp, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, G, true, 0>(j, n0, grp, xa, ca, ac);
+                    if (more) issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, j + U, n0, grp, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, G, true, 0, SMC>(j, n0, grp, xa, ca, ac, cw);
                     if constexpr (GB) dot_group<VEC, U, PAIR, true>(j, n0, lane, xa, xu, g_l);
                     if (j + 2 * U < steps)
-                        issue_group<VEC, U, HASC, G, true>(base, row_bytes, j + 2 * U, n0, grp, u0, c_l, xa, ca);
-                    if (more) consume_group<VEC, U, HASC, G, true, U>(j + U, n0, grp, xb, cb, ac);
+                        issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, j + 2 * U, n0, grp, u0, c_l, xa, ca);
+                    if (more) consume_group<VEC, U, HASC, G, true, U, SMC>(j + U, n0, grp, xb, cb, ac, cw);
                     if constexpr (GB)
                         if (more) dot_group<VEC, U, PAIR, true>(j + U, n0, lane, xb, xu, g_l);
                 }
@@ -1277,8 +1304,9 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
 // ms); ops with an edge coefficient (weighted, GAT) keep 85 registers (24
 // warps), where fewer registers spill into the edge loop (measured slower;
 // the alpha-mode GAT gather at 4 CTAs/SM: 26.9 -> 31.0 ms on Reddit).
-constexpr int min_blocks(int op, int coef, bool async) {
+constexpr int min_blocks(int op, int coef, bool async, int G = 1) {
     return async ? TLP_MINB_ASYNC
+         : (TLP_SMEMC && G > 1 && coef != COEF_NONE && (op == OP_GCN || op == OP_GIN)) ? TLP_MINB_SMC
                  : ((op == OP_GIN || op == OP_SAGE || op == OP_GCN) && coef == COEF_NONE)
                        ? TLP_MINB_LIGHT : TLP_MINB;
 }
@@ -1316,7 +1344,7 @@ __device__ __forceinline__ void agg_body(const AggArgs &a) {
 }
 
 template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC)) k_agg(const AggArgs a) {
+__global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC, G)) k_agg(const AggArgs a) {
     agg_body<VEC, OP, COEF, U, ASYNC, G>(a);
 }
 
