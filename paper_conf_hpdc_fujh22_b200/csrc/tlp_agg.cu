@@ -255,7 +255,8 @@ __device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, un
 // consume time, so no coefficient register is held across the gather latency
 // and the streamed-weight sums (GAT alpha mode, weighted GCN/GIN) fit 64
 // registers, i.e. 4 CTAs / 32 warps per SM like the coefficient-free sums
-// (measured: Reddit GAT 26.46 -> 24.42 ms; at 3 CTAs/SM 25.65 ms).
+// (measured: Reddit GAT 26.46 -> 24.42 ms, at 3 CTAs/SM 25.65 ms; GAT
+// backward 36.3 -> 34.4 ms).
 #ifndef TLP_SMEMC
 #define TLP_SMEMC 1
 #endif
@@ -431,7 +432,7 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     static_assert(STEPS % (2 * U) == 0, "U must divide the gather steps of a chunk in two groups");
     static_assert(!GB || G <= 2, "GAT backward edge dots: full warp or PAIR only");
     constexpr bool PAIR = (G == 2);
-    constexpr bool SMC = TLP_SMEMC && HASC && (G > 1) && !GB;
+    constexpr bool SMC = TLP_SMEMC && HASC && (G > 1);
     float *cw = SMC ? chunk_coef_smem() : nullptr;
     // lanes past F read column 0 (a valid address); their results are never stored
     const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
@@ -1306,7 +1307,8 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
 // the alpha-mode GAT gather at 4 CTAs/SM: 26.9 -> 31.0 ms on Reddit).
 constexpr int min_blocks(int op, int coef, bool async, int G = 1) {
     return async ? TLP_MINB_ASYNC
-         : (TLP_SMEMC && G > 1 && coef != COEF_NONE && (op == OP_GCN || op == OP_GIN)) ? TLP_MINB_SMC
+         : (TLP_SMEMC && G > 1 && coef != COEF_NONE && (op == OP_GCN || op == OP_GIN || op == OP_GATB))
+               ? TLP_MINB_SMC
                  : ((op == OP_GIN || op == OP_SAGE || op == OP_GCN) && coef == COEF_NONE)
                        ? TLP_MINB_LIGHT : TLP_MINB;
 }
