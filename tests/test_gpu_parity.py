@@ -1175,3 +1175,26 @@ def test_gcn_both_streamed_edge_coefficients(tlp, monkeypatch):
         sl.close()
     assert torch.equal(out, Y)
     g.close(); gw.close()
+
+
+def test_launch_counter(tlp, monkeypatch):
+    """tlp_graph_info.launches counts every kernel a handle enqueues: one gather
+    per aggregation, plus the X pre-scale of unweighted GCN BOTH and the
+    edge-softmax pass of GAT alpha mode (bench.py reports this count)."""
+    n = 500
+    rp, ci = synth.chung_lu(n, 8000, 0.5, 3, device="cpu")
+    X = _t(synth.features(n, 64, 64, seed=1))
+    el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
+    g = tlp.Graph(_t(rp), _t(ci))
+
+    def count(f):
+        l0 = tlp.tlp_graph_info_get(g.handle)["launches"]
+        f()
+        return tlp.tlp_graph_info_get(g.handle)["launches"] - l0
+    assert count(lambda: g.gin(X, 0.1)) == 1
+    assert count(lambda: g.gcn(X, "none")) == 1
+    assert count(lambda: g.gcn(X, "both")) == 2
+    assert count(lambda: g.gat(X, el, er, 0.2)) == 1
+    monkeypatch.setenv("TLP_GAT", "alpha")
+    assert count(lambda: g.gat(X, el, er, 0.2)) == 2
+    g.close()
