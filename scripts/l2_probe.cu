@@ -62,6 +62,18 @@ int main() {
         run<256, 8>(tab, tb, sms, out);
         run<512, 4>(tab, tb, sms, out);
     }
+    // large tables (HBM random-row gathers vs table size: address-translation
+    // reach; R-MAT-24's X is 8.6 GB)
+    if (getenv("PROBE_BIG")) {
+        float4 *big = nullptr;
+        const int64_t bb = int64_t(9) << 30;
+        if (cudaMalloc(&big, bb) == cudaSuccess) {
+            cudaMemset(big, 0, bb);
+            for (int64_t tb : {int64_t(1) << 30, int64_t(2) << 30, int64_t(4) << 30, int64_t(8) << 30})
+                run<512, 4>(big, tb, sms, out);
+            cudaFree(big);
+        }
+    }
     // narrow rows (narrow feature panels for X >> L2, e.g. products F = 100):
     // 16..128-byte random rows from an L2-resident table
     if (getenv("PROBE_NARROW"))
