@@ -1,5 +1,7 @@
-"""R-MAT-24 one-layer GCN(BOTH) under scheduling / gather knobs (CUDA events,
-median of N reps after warm-up).  Kernel experiment, not a bench line."""
+"""One aggregation of a pre-registered workload graph (default R-MAT-24
+GCN(BOTH); `reddit gin` etc.) under scheduling / gather knobs (CUDA events,
+median of N reps after warm-up).  Kernel experiment, not a bench line.
+usage: python scripts/rmat_probe.py [reps] [workload] [op]"""
 import os, sys, statistics
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -7,7 +9,8 @@ import paper_conf_hpdc_fujh22_b200 as tlp
 import synth
 
 reps = int(sys.argv[1]) if len(sys.argv) > 1 else 8
-name = "rmat24"
+name = sys.argv[2] if len(sys.argv) > 2 else "rmat24"
+op = sys.argv[3] if len(sys.argv) > 3 else "gcn"
 cfg = synth.CONFIGS[name]
 rp, ci = synth.dataset_graph(name, device="cuda")
 rp = torch.as_tensor(rp).cuda()
@@ -16,6 +19,16 @@ n = rp.numel() - 1
 F, ld = cfg["F"], cfg["ld"]
 X = torch.randn((n, ld), device="cuda")
 Y = torch.empty((n, ld), device="cuda")
+el = torch.randn(n, device="cuda")
+er = torch.randn(n, device="cuda")
+
+
+def call(g, out=None):
+    if op == "gin":
+        return g.gin(X, 0.1, Y=out, F=F)
+    if op == "gat":
+        return g.gat(X, el, er, 0.2, Y=out, F=F)
+    return g.gcn(X, "both", Y=out, F=F)
 
 
 def timeit(f):
@@ -36,7 +49,7 @@ def run(tag, g, env=None, sched=None):
     if sched:
         tlp.tlp_graph_set_schedule(g.handle, **sched)
     try:
-        print(tag, timeit(lambda: g.gcn(X, "both", Y=Y, F=F)), flush=True)
+        print(tag, timeit(lambda: call(g, Y)), flush=True)
     finally:
         for k, v in old.items():
             if v is None:
@@ -49,12 +62,14 @@ def run(tag, g, env=None, sched=None):
 
 g = tlp.Graph(rp, ci)
 print("info", {k: g.info[k] for k in ("n_units", "n_tasks", "n_hubs", "unit_edges")}, flush=True)
-ref = g.gcn(X, "both", F=F).clone()
+ref = call(g).clone()
 run("default", g)
 for h in ("0", "0.25", "0.75"):
     run("TLP_HOT=" + h, g, {"TLP_HOT": h})
 run("TLP_HOT_COLD=0", g, {"TLP_HOT_COLD": "0"})
 run("TLP_GATHER=reg", g, {"TLP_GATHER": "reg"})
+run("TLP_GATHER=async", g, {"TLP_GATHER": "async"})
+run("TLP_CTAS=3", g, {"TLP_CTAS": "3"})
 run("TLP_CTAS=2", g, {"TLP_CTAS": "2"})
 for st in (1, 2, 8, 32):
     run(f"step={st}", g, sched=dict(step=st))
@@ -63,9 +78,9 @@ for w in (4, 16):
 run("TLP_BOTH=prescale", g, {"TLP_BOTH": "prescale"})
 del g
 torch.cuda.empty_cache()
-for ue in (32, 64, 256, 512):
+for ue in (16, 32, 64, 256):
     g = tlp.Graph(rp, ci, opts=dict(unit_edges=ue))
-    Yv = g.gcn(X, "both", F=F)
+    Yv = call(g)
     same = bool(torch.equal(Yv[:, :F], ref[:, :F]))
     run(f"unit_edges={ue} (bitwise same {same})", g)
     del g, Yv
