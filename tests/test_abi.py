@@ -89,6 +89,17 @@ def test_no_cpu_fallback_for_features():
         tlp._vec_cuda(torch.zeros(4), "el")
 
 
+def test_missing_library_fails_loudly(tmp_path):
+    """Without libtlp.so the package does not import (no silent fallback)."""
+    import subprocess
+    import sys
+    env = dict(os.environ, TLP_LIB_PATH=str(tmp_path / "absent" / "libtlp.so"))
+    r = subprocess.run([sys.executable, "-c", "import paper_conf_hpdc_fujh22_b200"], cwd=ROOT,
+                       env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode != 0
+    assert "ImportError" in r.stderr
+
+
 def test_product_package_does_not_import_oracle():
     """The product path never touches oracle/ (and vice versa)."""
     pkg = os.path.join(ROOT, "paper_conf_hpdc_fujh22_b200")
