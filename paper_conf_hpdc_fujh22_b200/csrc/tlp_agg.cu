@@ -1,1404 +1,28 @@
-// tlp_agg.cu -- the aggregation kernels and their C ABI.
-//
-// One kernel launch per aggregation call (Observation III) that
-// fuses, per destination row: index staging (a5), the coefficient/score of
-// every edge, the gather-accumulate of the source rows (a6, a7), the hub
-// split-and-merge (a8) and the epilogue store (a9).
-//
-// Mapping (prior art: TLPGNN's two-level parallelism; kept where
-// it still holds on sm_100a, changed where it does not -- DESIGN.md):
-//  * a WARP owns a task (a run of whole destination rows, or one chunk of a
-//    hub row): no atomics on data (Observation I), no divergence.
-//  * lanes cover consecutive 16-byte (VEC=4) feature vectors of one source
-//    row (feature parallelism, Fig. 5b): a warp-wide gather of a
-//    row strip is 32 x LDG.128 = 512 contiguous bytes, fully coalesced
-//    (Observation II).  Rows wider than 128 floats are processed
-//    as 128-float strips, so the register footprint does not grow with F.
-//  * edge indices are loaded 32 at a time by the lanes (one coalesced LDG)
-//    and broadcast with shuffles; U source rows are in flight per warp.
-//  * fp32 accumulators live in registers; Y is written once per row (register
-//    caching).
-//  * GAT: LeakyReLU score, online softmax (running max / denominator rescaled
-//    once per 32-edge chunk) and the weighted gather in the same pass; scores
-//    never leave registers (kernel fusion).
-//  * scheduling: persistent grid, static first wave + atomic counter fetching
-//    `step` tasks (Alg. 1); hub rows (deg > H) are split into
-//    C-edge chunks whose partials are merged in chunk order by the last
-//    arriving warp (ticket), so results are bitwise deterministic.
-#include <cuda_runtime.h>
-#include <math.h>
-
+// tlp_agg.cu -- aggregation dispatch, the scalar passes around the gather
+// kernels (repack / pre-scale, GAT edge softmax, GAT backward passes, hot
+// tags, projection sums) and the C ABI of the aggregations.  The gather kernel
+// templates live in tlp_agg_kernels.cuh (see its header comment for the
+// mapping of TLPGNN's two-level parallelism onto sm_100a).
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
 
-#include "tlp_internal.h"
+#include "tlp_agg_kernels.cuh"
 
 namespace tlp {
 
-// OP_SAGE: GraphSage mean (optionally with the self row); OP_GATH: multi-head
-// GAT.
-// OP_GATB: GAT backward on the transposed graph (NEXT-4, tlp_gat_backward).
-enum Op : int { OP_GCN = 0, OP_GIN = 1, OP_GAT = 2, OP_SAGE = 3, OP_GATH = 4, OP_GATB = 5 };
-enum Coef : int { COEF_NONE = 0, COEF_COUT = 1, COEF_W = 2, COEF_W_COUT = 3 };
-enum Sched : int { S_DYNAMIC = 0, S_STATIC = 1, S_HARDWARE = 2 };
-
-constexpr unsigned FULL = 0xffffffffu;
-
-// Compile-time tuning knobs: source rows per
-// gather group (two groups in flight per warp) and the launch bounds.
-#ifndef TLP_U
-#define TLP_U 2        // register path: rows per gather group (2 groups in flight)
-#endif
-#ifndef TLP_MAXT
-#define TLP_MAXT 256   // threads per CTA at most (8 warps)
-#endif
-#ifndef TLP_MINB
-#define TLP_MINB 3     // register path: 3 CTAs/SM -> <= 85 registers, 24 warps/SM
-#endif
-#ifndef TLP_MHB
-#define TLP_MHB 4      // multi-head GAT: heads scored together per pass
-#endif
-#ifndef TLP_HINTS
-#define TLP_HINTS 0    // 1: L2 evict_first policy on per-edge streams and Y stores (measured: no gain)
-#endif
-#ifndef TLP_MINB_LIGHT
-#define TLP_MINB_LIGHT 4  // register path, no edge coefficient (GIN, SAGE): <= 64 registers, 32 warps/SM
-#endif
-#ifndef TLP_MINB_ASYNC
-#define TLP_MINB_ASYNC 3  // async path: 3 CTAs/SM (ring = 3 x 64 KB of shared memory)
-#endif
-
-struct AggArgs {
-    const int64_t *__restrict__ rowptr;
-    const int32_t *__restrict__ colidx;
-    const float *__restrict__ ew;
-    const float *__restrict__ c_out;
-    const float *__restrict__ X;
-    float *__restrict__ Y;
-    const float *__restrict__ el;
-    const float *__restrict__ er;
-    const int2 *__restrict__ tasks;
-    const int32_t *__restrict__ hub_row;
-    const int32_t *__restrict__ hub_off;
-    int32_t *hub_ticket;
-    float *scratch;  // hub partial vectors [n_chunks x ldp]
-    float *md;       // GAT hub (m, den) pairs [n_chunks x 2]
-    unsigned long long *ctr;
-    unsigned int *done;
-    int64_t ldx, ldy, ldp, row_offset, n_tasks, n_items, n_hubs, n_chunks, C;
-    int F, n_strips, norm, step, sched, panel;
-    int lps;  // lanes per strip (full-warp strips: lps * VEC columns, lps <= 32)
-    float eps1, slope;
-    int sage_self;  // OP_SAGE: include X[v] in the mean
-    const float *bias;  // layer epilogue (NEXT-3): y = act(y + bias)
-    int act;
-    float act_param;
-    int heads, fh;  // OP_GATH: H heads of fh columns each (F = heads * fh)
-    // NEXT-2 fused all-gather: when n_dests > 0 every output row is stored to
-    // dests[i] + (row_offset + r) * ldy for each destination (the Y_full of every
-    // rank, mapped over NVLink) instead of to Y.
-    float *const *dests;
-    int n_dests;
-    // hot-source L2 policy: when hot_thr != 0
-    // colidx carries the source's out-degree class in bits 27-31; sources with
-    // tag >= hot_thr are gathered with L2 evict_last, the rest with cold_first ?
-    // evict_first : evict_normal.  A cache policy only: no value changes.
-    unsigned hot_thr;
-    int cold_first;
-    // OP_GATB: forward X (the transposed row's own features) and the per-strip
-    // edge dot products gbuf[s * gstride + e] = sum over strip s of
-    // dY[v_e] . X[u] (transposed edge e).
-    const float *xself;
-    int64_t ldxs;
-    // NEXT-3 epilogue projections: per strip s and local row r, the strip's
-    // partial dots proj[(s * n_dst + r) * 2 + {0,1}] of the finished output
-    // row with att_l / att_r (NULL proj: off)
-    const float *att_l, *att_r;
-    float *proj;
-    int64_t n_dst;
-    float *gbuf;
-    int64_t gstride;
-};
-
-constexpr unsigned kIdxMask = (1u << 27) - 1u;
-
-// Per-thread L2 policies for tagged gathers (createpolicy once per task).
-struct GPol {
-    unsigned thr;
-    unsigned long long hot, cold;
-};
-__device__ __forceinline__ GPol make_gpol(const AggArgs &a) {
-    GPol g;
-    g.thr = a.hot_thr;
-    g.hot = g.cold = 0;
-    if (g.thr) {
-        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(g.hot));
-        if (a.cold_first) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(g.cold));
-        else asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(g.cold));
-    }
-    return g;
-}
-
-template <int VEC>
-struct Vec {
-    float v[VEC];
-};
-
-template <int VEC>
-__device__ __forceinline__ Vec<VEC> ld_vec(const float *p) {
-    Vec<VEC> r;
-    if constexpr (VEC == 4) {
-        float4 t = __ldg(reinterpret_cast<const float4 *>(p));
-        r.v[0] = t.x; r.v[1] = t.y; r.v[2] = t.z; r.v[3] = t.w;
-    } else if constexpr (VEC == 2) {
-        float2 t = __ldg(reinterpret_cast<const float2 *>(p));
-        r.v[0] = t.x; r.v[1] = t.y;
-    } else {
-        r.v[0] = __ldg(p);
-    }
-    return r;
-}
-
-// L2-coherent load (data written by another SM during this launch).
-template <int VEC>
-__device__ __forceinline__ Vec<VEC> ld_vec_cg(const float *p) {
-    Vec<VEC> r;
-    if constexpr (VEC == 4) {
-        float4 t = __ldcg(reinterpret_cast<const float4 *>(p));
-        r.v[0] = t.x; r.v[1] = t.y; r.v[2] = t.z; r.v[3] = t.w;
-    } else if constexpr (VEC == 2) {
-        float2 t = __ldcg(reinterpret_cast<const float2 *>(p));
-        r.v[0] = t.x; r.v[1] = t.y;
-    } else {
-        r.v[0] = __ldcg(p);
-    }
-    return r;
-}
-
-template <int VEC>
-__device__ __forceinline__ void st_vec(float *p, const Vec<VEC> &x) {
-    if constexpr (VEC == 4) {
-#if TLP_HINTS
-        unsigned long long pol;
-        asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
-                     ::"l"(p), "f"(x.v[0]), "f"(x.v[1]), "f"(x.v[2]), "f"(x.v[3]), "l"(pol) : "memory");
-#else
-        *reinterpret_cast<float4 *>(p) = make_float4(x.v[0], x.v[1], x.v[2], x.v[3]);
-#endif
-    } else if constexpr (VEC == 2) {
-        *reinterpret_cast<float2 *>(p) = make_float2(x.v[0], x.v[1]);
-    } else {
-        *p = x.v[0];
-    }
-}
-
-// Store only columns < F (the tail vector of a row may straddle F).
-template <int VEC>
-__device__ __forceinline__ void st_row(float *row, int col, int F, const Vec<VEC> &x) {
-    if (col + VEC <= F) {
-        st_vec<VEC>(row + col, x);
-    } else {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c)
-            if (col + c < F) row[col + c] = x.v[c];
-    }
-}
-
-__device__ __forceinline__ float warp_max(float v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(FULL, v, o));
-    return v;
-}
-
-// Butterfly sum: every lane ends with the bitwise-same value (commutativity).
-__device__ __forceinline__ float warp_sum(float v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
-    return v;
-}
-
-// Gather address of source row u: base + u * row_bytes, one IMAD.WIDE.U32
-// (32x32 -> 64-bit multiply-add); base = X + column (a byte pointer).
-__device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, unsigned row_bytes) {
-    return reinterpret_cast<const float *>(base + (unsigned long long)u * row_bytes);
-}
-
-// ---- canonical reduction order ---------------------------------------------
-// Every path reduces a row (or a hub chunk) as TWO interleaved chains: the
-// edges at even and at odd positions (relative to the row / chunk start, in
-// CSR order), each accumulated sequentially with fmaf, then added as
-// even + odd.  Hub chunks start at even offsets (C is even) and are merged in
-// chunk order.  The register path (full warp or half-warp PAIR), the cp.async
-// path, every strip width, scheduler and partition produce exactly this
-// order, hence bitwise-identical results.
-//
-// Lane -> edge mapping inside a 32-edge chunk, for step j, group slot k:
-//   G = 1 (full warp): every lane gathers edge j+k for its 4 columns
-//              (chain (j+k)&1);
-//   G = 2 (PAIR): lanes 0-15 gather edge 2(j+k), lanes 16-31 edge 2(j+k)+1,
-//              over 64 columns, so a warp-wide LDG.128 still moves 512 bytes
-//              while the strip of X is half as wide (each half-warp is one
-//              chain: the canonical even/odd order);
-//   G = 4, 8 (narrow rows, F <= 32 / 16): lane group g = lane / (32/G) gathers
-//              edge G(j+k)+g, so a warp instruction still moves G rows.  Group
-//              g accumulates the chain of positions = g (mod G); the chains
-//              are added by a fixed butterfly (xor 16, then 8, ...).  This
-//              order depends only on F (never on P, the schedule or the
-//              partition), so results stay bitwise reproducible and
-//              partition-invariant; G <= 2 paths are bitwise identical to each
-//              other (R10).
-
-// Edge coefficients of lane-group gathers (G > 1) live in shared memory: the
-// chunk's 32 coefficients are written once per chunk and read (broadcast) at
-// consume time, so no coefficient register is held across the gather latency
-// and the streamed-weight sums (GAT alpha mode, weighted GCN/GIN) fit 64
-// registers, i.e. 4 CTAs / 32 warps per SM like the coefficient-free sums
-// (measured: Reddit GAT 26.46 -> 24.42 ms, at 3 CTAs/SM 25.65 ms; GAT
-// backward 36.3 -> 34.4 ms).
-#ifndef TLP_SMEMC
-#define TLP_SMEMC 1
-#endif
-#ifndef TLP_MINB_SMC
-#define TLP_MINB_SMC 4   // resident CTAs for the shared-memory-coefficient kernels
-#endif
-__device__ __forceinline__ float *chunk_coef_smem() {
-    __shared__ float tlp_cw[TLP_MAXT / 32][32];
-    return tlp_cw[threadIdx.x >> 5];
-}
-
-template <int VEC, int U, bool HASC, int G, bool CLAMP, bool SMC = false>
-__device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes, int j, int n,
-                                            int grp, int u_l, float c_l, Vec<VEC> (&xv)[U],
-                                            float (&ck)[U]) {
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-        int p = G * (j + k) + grp;
-        if constexpr (CLAMP) p = min(p, n - 1);  // duplicate of a line in flight
-        const unsigned u = (unsigned)__shfl_sync(FULL, u_l, p);
-        if constexpr (HASC && !SMC) ck[k] = __shfl_sync(FULL, c_l, p);
-        xv[k] = ld_vec<VEC>(row_ptr(base, u, row_bytes));
-    }
-}
-
-// PHASE: parity of the group's first step (the caller's j is a multiple of 2U).
-template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE, bool SMC = false>
-__device__ __forceinline__ void consume_group(int j, int n, int grp, const Vec<VEC> (&xv)[U],
-                                              const float (&ck)[U], Vec<VEC> (&ac)[2],
-                                              const float *cw = nullptr) {
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-        const int p = G * (j + k) + grp;
-        const int ch = (G > 1) ? 0 : ((PHASE + k) & 1);
-        if (!GUARD || p < n) {
-            float cv = 0.f;
-            if constexpr (HASC) cv = SMC ? cw[p] : ck[k];
-#pragma unroll
-            for (int c = 0; c < VEC; ++c) {
-                if constexpr (HASC) ac[ch].v[c] = fmaf(cv, xv[k].v[c], ac[ch].v[c]);
-                else ac[ch].v[c] += xv[k].v[c];
-            }
-        }
-    }
-}
-
-// OP_GATB: per-edge dot products dY[v_e] . X[u] over this lane's columns,
-// reduced across the lanes that share the edge (butterfly: the same bits in
-// every lane); lane p keeps the dot of edge p of the chunk in g_l.
-template <int VEC, int U, bool PAIR, bool GUARD>
-__device__ __forceinline__ void dot_group(int j, int n, int lane, const Vec<VEC> (&xv)[U],
-                                          const Vec<VEC> &xu, float &g_l) {
-    const int half = PAIR ? (lane >> 4) : 0;
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-        const int p = PAIR ? 2 * (j + k) + half : j + k;
-        float d = 0.f;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) d = fmaf(xv[k].v[c], xu.v[c], d);
-        if (GUARD && p >= n) d = 0.f;
-        if constexpr (PAIR) {
-#pragma unroll
-            for (int o = 8; o > 0; o >>= 1) d += __shfl_xor_sync(FULL, d, o);
-            const float other = __shfl_xor_sync(FULL, d, 16);
-            const int t2 = 2 * (j + k);
-            if (lane == t2) g_l = half == 0 ? d : other;
-            if (lane == t2 + 1) g_l = half == 1 ? d : other;
-        } else {
-            d = warp_sum(d);
-            if (lane == p) g_l = d;
-        }
-    }
-}
-
-// OP_GATB, full 32-edge chunks: the per-step lane partials are reduced by a
-// streaming transposed butterfly.  Steps t are the gather steps of the chunk
-// (PAIR: 16 steps of two edges, one per half-warp, 4 levels xor 8,4,2,1; full
-// warp: 32 steps, 5 levels xor 16..1).  At level k a lane keeps the step whose
-// bit matches its lane bit and adds its partner's partial of that step, so one
-// shuffle reduces two steps; after the last level lane l holds the whole dot of
-// step bitreverse(l) (PAIR: of edge 2*rev4(l & 15) + half).  15 (PAIR) or 31
-// shuffles per 32 edges instead of 4-5 per edge.  t is a compile-time constant
-// in the unrolled full-chunk loop, so the level logic folds away.
-struct DotTree {
-    float lv[5];
-};
-template <bool PAIR>
-__device__ __forceinline__ void dot_push(DotTree &tr, float d, int t, int lane, float *gout) {
-    constexpr int L = PAIR ? 4 : 5;
-#pragma unroll
-    for (int k = 0; k < L; ++k) {
-        const int bitmask = (PAIR ? 8 : 16) >> k;  // lane bit of level k
-        if (((t >> k) & 1) == 0) {  // first of the pair at this level: park it
-            tr.lv[k] = d;
-            return;
-        }
-        const bool hi = (lane & bitmask) != 0;
-        const float keep = hi ? d : tr.lv[k];
-        const float send = hi ? tr.lv[k] : d;
-        d = keep + __shfl_xor_sync(FULL, send, bitmask);
-    }
-    // all levels done (t = last step): lane holds the dot of step rev(lane)
-    const int l = PAIR ? (lane & 15) : lane;
-    const int rv = PAIR ? (int)(__brev((unsigned)l) >> 28) : (int)(__brev((unsigned)l) >> 27);
-    const int e = PAIR ? 2 * rv + (lane >> 4) : rv;
-    gout[e] = d;
-}
-template <int VEC, int U, bool PAIR>
-__device__ __forceinline__ void dot_tree(int j, int lane, const Vec<VEC> (&xv)[U],
-                                         const Vec<VEC> &xu, DotTree &tr, float *gout) {
-#pragma unroll
-    for (int k = 0; k < U; ++k) {
-        float d = 0.f;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) d = fmaf(xv[k].v[c], xu.v[c], d);
-        dot_push<PAIR>(tr, d, j + k, lane, gout);
-    }
-}
-
-// ---- L2 residency hints -------------------------------------------------------
-// Per-edge streams (colidx, edge coefficients) and Y are touched once per strip:
-// with TLP_HINTS they are loaded / stored with an L2 evict_first policy so they
-// do not evict the L2-resident panel of X that every edge gathers from.
-__device__ __forceinline__ unsigned long long policy_evict_first() {
-    unsigned long long p;
-    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-__device__ __forceinline__ int ld_stream(const int32_t *ptr) {
-#if TLP_HINTS
-    int v;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
-                 : "=r"(v) : "l"(ptr), "l"(policy_evict_first()));
-    return v;
-#else
-    return __ldg(ptr);
-#endif
-}
-__device__ __forceinline__ float ld_stream(const float *ptr) {
-#if TLP_HINTS
-    float v;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
-                 : "=f"(v) : "l"(ptr), "l"(policy_evict_first()));
-    return v;
-#else
-    return __ldg(ptr);
-#endif
-}
-
-// Reduce the edges [e0, e1) of one destination row for the feature vector at
-// `col` (a6 / a7).  GCN/GIN: acc = sum_e c_e X[u_e] (two-chain order above).
-// GAT: online softmax state (m, den, acc = sum_e exp(s_e - m) X[u_e]).
-//
-// Latency hiding (the kernel is bound by bytes in flight, not by arithmetic):
-//  * edge indices are loaded 32 at a time by the lanes two chunks ahead, and
-//    the index-dependent values (c_out[u] or el[u]) one chunk ahead, so the
-//    gathers of a chunk never wait on an index load;
-//  * the gathers of a chunk are issued in double-buffered groups of U source
-//    rows: the next group is in flight while the current one is accumulated;
-//    full 32-edge chunks are fully unrolled (compile-time shuffle lanes).
-template <int VEC, int OP, int COEF, int U, int G>
-__device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64_t e1,
-                                             int col, bool active, float er_v, int lane,
-                                             Vec<VEC> &acc, float &m, float &den,
-                                             const Vec<VEC> &xu, float *gout) {
-    // OP_GATB: the coefficient of transposed edge u -> v is alpha_e, streamed
-    // (COEF_W) from the k_gatb_alpha pass; the strip's dot dY[v].X[u] of every
-    // edge is reduced across lanes and stored to gout
-    constexpr bool GB = (OP == OP_GATB);
-    constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT) || GB;
-    constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);  // index-dependent value
-    constexpr int STEPS = 32 / G;  // gather steps of a full chunk
-    static_assert(STEPS % (2 * U) == 0, "U must divide the gather steps of a chunk in two groups");
-    static_assert(!GB || G <= 2, "GAT backward edge dots: full warp or PAIR only");
-    constexpr bool PAIR = (G == 2);
-    constexpr bool SMC = TLP_SMEMC && HASC && (G > 1);
-    float *cw = SMC ? chunk_coef_smem() : nullptr;
-    // lanes past F read column 0 (a valid address); their results are never stored
-    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
-    const unsigned row_bytes = (unsigned)a.ldx * 4u;
-    const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
-    // 32-bit edge offsets relative to e0 (a row or hub chunk has < 2^31 edges)
-    const int32_t *__restrict__ ci = a.colidx + e0;
-    const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
-    const int len = (int)(e1 - e0);
-    const int grp = lane / (32 / G);  // lane group (G > 1)
-    Vec<VEC> ac[2];
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) ac[0].v[c] = ac[1].v[c] = 0.f;
-    if (len > 0) {
-        int off = 0;
-        int n0 = min(32, len);
-        int n1 = min(32, len - 32);
-        int u0 = 0, u1 = 0;
-        float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
-        if (lane < n0) {
-            u0 = ld_stream(ci + lane);
-            if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane);
-        }
-        if (lane < n1) {
-            u1 = ld_stream(ci + 32 + lane);
-            if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
-        }
-        if constexpr (DEP)
-            if (lane < n0) d0 = __ldg(dep + u0);
-        while (true) {
-            // two chunks ahead: indices; one chunk ahead: index-dependent values
-            const int n2 = min(32, len - off - 64);
-            int u2 = 0;
-            float w2 = 1.f;
-            if (lane < n2) {
-                u2 = ld_stream(ci + off + 64 + lane);
-                if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
-            }
-            if constexpr (DEP)
-                if (lane < n1) d1 = __ldg(dep + u1);
-            // coefficients of the current chunk
-            float c_l = 1.f;
-            if constexpr (OP == OP_GAT) {
-                float s = -INFINITY;
-                if (lane < n0) {
-                    const float t = d0 + er_v;
-                    s = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
-                }
-                const float m_new = fmaxf(m, warp_max(s));
-                const float scale = __expf(m - m_new);  // m = -inf -> 0
-                c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
-                den = fmaf(den, scale, warp_sum(c_l));
-#pragma unroll
-                for (int c = 0; c < VEC; ++c) {
-                    ac[0].v[c] *= scale;
-                    ac[1].v[c] *= scale;
-                }
-                m = m_new;
-            } else {
-                if constexpr (COEF & COEF_COUT) c_l = d0;
-                if constexpr (COEF & COEF_W) c_l *= w0;
-            }
-            if constexpr (SMC) {
-                __syncwarp();  // the previous chunk's coefficients are consumed
-                cw[lane] = c_l;
-                __syncwarp();
-            }
-            Vec<VEC> xa[U], xb[U];
-            float ca[U], cb[U];
-            float g_l = 0.f;  // OP_GATB (partial chunk): this strip's dot of edge `lane`
-            DotTree dt_;      // OP_GATB (full chunk): pending butterfly levels
-            if (n0 == 32) {
-                // full chunk: fully unrolled, compile-time shuffle lanes, no guards
-                issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, 0, 32, grp, u0, c_l, xa, ca);
-#pragma unroll
-                for (int j = 0; j < STEPS; j += 2 * U) {
-                    issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, j + U, 32, grp, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, G, false, 0, SMC>(j, 32, grp, xa, ca, ac, cw);
-                    if constexpr (GB) dot_tree<VEC, U, PAIR>(j, lane, xa, xu, dt_, gout + off);
-                    if (j + 2 * U < STEPS)
-                        issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, j + 2 * U, 32, grp, u0, c_l, xa, ca);
-                    consume_group<VEC, U, HASC, G, false, U, SMC>(j + U, 32, grp, xb, cb, ac, cw);
-                    if constexpr (GB) dot_tree<VEC, U, PAIR>(j + U, lane, xb, xu, dt_, gout + off);
-                }
-            } else {
-                // partial chunk (n0 is warp-uniform: the guards never diverge)
-                const int steps = (n0 + G - 1) / G;
-                issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, 0, n0, grp, u0, c_l, xa, ca);
-                for (int j = 0; j < steps; j += 2 * U) {
-                    const bool more = j + U < steps;
-                    if (more) issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, j + U, n0, grp, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, G, true, 0, SMC>(j, n0, grp, xa, ca, ac, cw);
-                    if constexpr (GB) dot_group<VEC, U, PAIR, true>(j, n0, lane, xa, xu, g_l);
-                    if (j + 2 * U < steps)
-                        issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, j + 2 * U, n0, grp, u0, c_l, xa, ca);
-                    if (more) consume_group<VEC, U, HASC, G, true, U, SMC>(j + U, n0, grp, xb, cb, ac, cw);
-                    if constexpr (GB)
-                        if (more) dot_group<VEC, U, PAIR, true>(j + U, n0, lane, xb, xu, g_l);
-                }
-            }
-            if constexpr (GB)
-                if (n0 < 32 && lane < n0) gout[off + lane] = g_l;  // partial chunk
-            if (n1 <= 0) break;
-            off += 32;
-            n0 = n1; n1 = n2;
-            u0 = u1; u1 = u2;
-            w0 = w1; w1 = w2;
-            d0 = d1;
-        }
-    }
-    // even + odd (G = 2: the odd chain lives in the other half-warp); G > 2:
-    // the group chains added by a fixed butterfly
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) {
-        if constexpr (G > 1) {
-            float x = ac[0].v[c];
-#pragma unroll
-            for (int o = 16; o >= 32 / G; o >>= 1) x += __shfl_xor_sync(FULL, x, o);
-            acc.v[c] = x;
-        } else {
-            acc.v[c] = ac[0].v[c] + ac[1].v[c];
-        }
-    }
-}
-
-// ---- asynchronous-copy path ------------------------------------------------
-// The gathered rows land in a per-warp shared-memory ring through cp.async
-// (LDGSTS, L2 -> SMEM, bypassing L1 and the register file), D edges deep.  Bytes
-// in flight then cost no registers, so occupancy and depth are decoupled.
-#ifndef TLP_DEPTH
-#define TLP_DEPTH 16   // edges in flight per warp on the async path
-#endif
-
-template <int VEC>
-__device__ __forceinline__ void cp_async_vec(float *dst_smem, const float *src, bool pred) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
-    const int bytes = pred ? 4 * VEC : 0;  // src-size 0 => zero fill, no global read
-    if constexpr (VEC == 4)
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
-    else if constexpr (VEC == 2)
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
-    else
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
-}
-// cp.async of source row u (possibly tagged) with the hot/cold L2 policy.
-template <int VEC>
-__device__ __forceinline__ void cp_async_x(float *dst_smem, const char *base, unsigned u,
-                                           unsigned row_bytes, const GPol &gp, bool pred) {
-    const float *src = reinterpret_cast<const float *>(
-        base + (unsigned long long)(u & kIdxMask) * row_bytes);
-    if (gp.thr == 0 || VEC != 4) {
-        cp_async_vec<VEC>(dst_smem, src, pred);
-        return;
-    }
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
-    const int bytes = pred ? 16 : 0;
-    const unsigned long long pol = u >= gp.thr ? gp.hot : gp.cold;
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;\n"
-                 ::"r"(d), "l"(src), "r"(bytes), "l"(pol));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
-
-template <int VEC>
-__device__ __forceinline__ float *warp_ring() {
-    extern __shared__ __align__(16) float tlp_smem[];
-    const int w = threadIdx.x >> 5;
-    return tlp_smem + (size_t)w * TLP_DEPTH * 32 * VEC;
-}
-
-template <int VEC, bool HASC>
-__device__ __forceinline__ void acc_from_smem(const float *src, float cj, Vec<VEC> &acc) {
-    if constexpr (VEC == 4) {
-        const float4 x = *reinterpret_cast<const float4 *>(src);
-        if constexpr (HASC) {
-            acc.v[0] = fmaf(cj, x.x, acc.v[0]); acc.v[1] = fmaf(cj, x.y, acc.v[1]);
-            acc.v[2] = fmaf(cj, x.z, acc.v[2]); acc.v[3] = fmaf(cj, x.w, acc.v[3]);
-        } else {
-            acc.v[0] += x.x; acc.v[1] += x.y; acc.v[2] += x.z; acc.v[3] += x.w;
-        }
-    } else {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) {
-            if constexpr (HASC) acc.v[c] = fmaf(cj, src[c], acc.v[c]);
-            else acc.v[c] += src[c];
-        }
-    }
-}
-
-template <int VEC, int OP, int COEF, int U>
-__device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0, int64_t e1,
-                                                   int col, bool active, float er_v, int lane,
-                                                   Vec<VEC> &acc, float &m, float &den) {
-    constexpr int D = TLP_DEPTH;
-    constexpr bool HASC = (COEF != COEF_NONE) || (OP == OP_GAT);
-    constexpr bool DEP = (COEF & COEF_COUT) || (OP == OP_GAT);
-    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
-    const unsigned row_bytes = (unsigned)a.ldx * 4u;
-    const float *__restrict__ dep = (OP == OP_GAT) ? a.el : a.c_out;
-    const GPol gp = make_gpol(a);
-    const int32_t *__restrict__ ci = a.colidx + e0;
-    const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
-    const int len = (int)(e1 - e0);
-    Vec<VEC> ae, ao;  // even / odd chains (canonical order)
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) ae.v[c] = ao.v[c] = 0.f;
-    if (len > 0) {
-        float *ring = warp_ring<VEC>() + lane * VEC;
-        int off = 0;
-        int n0 = min(32, len);
-        int n1 = min(32, len - 32);
-        int u0 = 0, u1 = 0;
-        float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
-        if (lane < n0) {
-            u0 = ld_stream(ci + lane);
-            if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane);
-        }
-        if (lane < n1) {
-            u1 = ld_stream(ci + 32 + lane);
-            if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
-        }
-        if constexpr (DEP)
-            if (lane < n0) d0 = __ldg(dep + (u0 & kIdxMask));
-        // prologue: edges 0 .. D-2 in flight
-#pragma unroll
-        for (int k = 0; k < D - 1; ++k) {
-            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
-            cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active && k < len);
-            cp_async_commit();
-        }
-        int slot = 0;  // ring slot of edge `off + j`
-        while (true) {
-            const int n2 = min(32, len - off - 64);
-            int u2 = 0;
-            float w2 = 1.f;
-            if (lane < n2) {
-                u2 = ld_stream(ci + off + 64 + lane);
-                if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
-            }
-            if constexpr (DEP)
-                if (lane < n1) d1 = __ldg(dep + (u1 & kIdxMask));
-            float c_l = 1.f;
-            if constexpr (OP == OP_GAT) {
-                float s = -INFINITY;
-                if (lane < n0) {
-                    const float t = d0 + er_v;
-                    s = t >= 0.f ? t : a.slope * t;
-                }
-                const float m_new = fmaxf(m, warp_max(s));
-                const float scale = __expf(m - m_new);
-                c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
-                den = fmaf(den, scale, warp_sum(c_l));
-#pragma unroll
-                for (int c = 0; c < VEC; ++c) {
-                    ae.v[c] *= scale;
-                    ao.v[c] *= scale;
-                }
-                m = m_new;
-            } else {
-                if constexpr (COEF & COEF_COUT) c_l = d0;
-                if constexpr (COEF & COEF_W) c_l *= w0;
-            }
-            for (int j = 0; j < n0; ++j) {
-                // issue edge j + D - 1 (in this chunk or the next one)
-                const int jj = j + D - 1;
-                const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
-                const bool valid = (off + jj) < len;
-                int ws = slot + D - 1;
-                if (ws >= D) ws -= D;
-                cp_async_x<VEC>(ring + ws * 32 * VEC, base, (unsigned)ui, row_bytes, gp, active && valid);
-                cp_async_commit();
-                cp_async_wait<D - 1>();
-                const float cj = __shfl_sync(FULL, c_l, j);
-                // chunks start at even offsets: the parity of j is the edge's parity
-                if (j & 1) acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, cj, ao);
-                else acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, cj, ae);
-                if (++slot == D) slot = 0;
-            }
-            if (n1 <= 0) break;
-            off += 32;
-            n0 = n1; n1 = n2;
-            u0 = u1; u1 = u2;
-            w0 = w1; w1 = w2;
-            d0 = d1;
-        }
-        cp_async_wait<0>();  // drain the (empty) tail groups before the ring is reused
-    }
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
-}
-
-// ---- multi-head GAT (NEXT-1) -----------------------------------------------
-// Head h owns columns [h*fh, (h+1)*fh) (fh a multiple of VEC, so a lane's
-// vector lies in one head).  A strip of 32*VEC columns spans heads
-// [h_lo, h_lo+nh).  Per 32-edge chunk the warp computes, head by head, the
-// LeakyReLU scores, the online-softmax update (running max M, denominator D,
-// rescale S) and the weights p[j], kept in a per-warp shared-memory block;
-// each lane then gathers with the weights of its own head.  Scores never
-// leave the SM.  Reduction order: the canonical two chains per head.
-constexpr int kMhMaxHeads = 33;  // heads one strip can touch (fh >= VEC)
-constexpr int kMhWarpFloats = kMhMaxHeads * 32 + 3 * kMhMaxHeads + 1;  // P, M, D, S (+pad)
-
-__device__ __forceinline__ float *mh_warp_smem() {
-    extern __shared__ __align__(16) float tlp_smem[];
-    return tlp_smem + (size_t)(threadIdx.x >> 5) * kMhWarpFloats;
-}
-
-// Scores, online-softmax update and weights of one 32-edge chunk for the heads
-// [h_lo, h_lo+nh) of a strip (lane j holds edge j with source u_l).  Heads are
-// processed TLP_MHB at a time so their el loads and warp reductions overlap.
-__device__ __forceinline__ void mh_chunk_scores(const AggArgs &a, int u_l, int n0, int H, int h_lo,
-                                                int nh, const float *__restrict__ erv, int lane,
-                                                float *P, float *M, float *D, float *S) {
-    constexpr int B = TLP_MHB;
-    const float *__restrict__ elu = a.el + (size_t)((unsigned)u_l) * H + h_lo;
-    for (int hb = 0; hb < nh; hb += B) {
-        float sv[B], mo[B], mn[B], sm[B];
-#pragma unroll
-        for (int k = 0; k < B; ++k) {
-            sv[k] = -INFINITY;
-            if (hb + k < nh && lane < n0) {
-                const float t = __ldg(elu + hb + k) + __ldg(erv + hb + k);
-                sv[k] = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
-            }
-        }
-#pragma unroll
-        for (int k = 0; k < B; ++k) {
-            if (hb + k < nh) {  // warp-uniform
-                mo[k] = M[hb + k];
-                mn[k] = fmaxf(mo[k], warp_max(sv[k]));
-                const float p = (lane < n0) ? __expf(sv[k] - mn[k]) : 0.f;
-                sm[k] = warp_sum(p);
-                P[(hb + k) * 32 + lane] = p;
-            }
-        }
-        __syncwarp();
-        if (lane == 0) {
-#pragma unroll
-            for (int k = 0; k < B; ++k)
-                if (hb + k < nh) {
-                    const float scale = __expf(mo[k] - mn[k]);
-                    M[hb + k] = mn[k];
-                    D[hb + k] = fmaf(D[hb + k], scale, sm[k]);
-                    S[hb + k] = scale;
-                }
-        }
-        __syncwarp();
-    }
-}
-
-// A lane's VEC columns [col, col+VEC) lie in at most two heads (fh >= VEC):
-// head slot hl for components c < split, hl + 1 for the rest.
-template <int VEC, int U>
-__device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, int64_t e1, int s,
-                                                int col, bool active, int64_t rglob, int lane,
-                                                Vec<VEC> &acc, float *&Mh, float *&Dh, int &h_lo,
-                                                int &nh, int &hl, int &split) {
-    float *P = mh_warp_smem();
-    float *M = P + kMhMaxHeads * 32;
-    float *D = M + kMhMaxHeads;
-    float *S = D + kMhMaxHeads;
-    Mh = M;
-    Dh = D;
-    const int H = a.heads, fh = a.fh;
-    const int c_lo = s * 32 * VEC;
-    const int c_hi = min(a.F, c_lo + 32 * VEC) - 1;
-    h_lo = c_lo / fh;
-    nh = c_hi / fh - h_lo + 1;
-    const int cc = active ? col : c_lo;
-    hl = cc / fh - h_lo;
-    split = (hl + h_lo + 1) * fh - cc;                 // components in head hl
-    const int hl2 = min(hl + (split < VEC ? 1 : 0), nh - 1);
-    for (int hh = lane; hh < nh; hh += 32) {
-        M[hh] = -INFINITY;
-        D[hh] = 0.f;
-    }
-    __syncwarp();
-    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
-    const unsigned row_bytes = (unsigned)a.ldx * 4u;
-    const int32_t *__restrict__ ci = a.colidx + e0;
-    const float *__restrict__ erv = a.er + rglob * H + h_lo;
-    const int len = (int)(e1 - e0);
-    Vec<VEC> ac[2];
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) ac[0].v[c] = ac[1].v[c] = 0.f;
-    for (int off = 0; off < len; off += 32) {
-        const int n0 = min(32, len - off);
-        const int u_l = (lane < n0) ? __ldg(ci + off + lane) : 0;
-        mh_chunk_scores(a, u_l, n0, H, h_lo, nh, erv, lane, P, M, D, S);
-        const float sA = S[hl], sB = S[hl2];
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) {
-            const float sc = (c < split) ? sA : sB;
-            ac[0].v[c] *= sc;
-            ac[1].v[c] *= sc;
-        }
-        const float *pa = P + hl * 32;
-        const float *pb = P + hl2 * 32;
-        for (int j = 0; j < n0; j += 2 * U) {
-            Vec<VEC> xv[2 * U];
-            float ca[2 * U], cb[2 * U];
-#pragma unroll
-            for (int k = 0; k < 2 * U; ++k) {
-                const int jj = min(j + k, n0 - 1);
-                const unsigned u = (unsigned)__shfl_sync(FULL, u_l, jj);
-                ca[k] = pa[jj];
-                cb[k] = pb[jj];
-                xv[k] = ld_vec<VEC>(row_ptr(base, u, row_bytes));
-            }
-#pragma unroll
-            for (int k = 0; k < 2 * U; ++k)
-                if (j + k < n0) {
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c)
-                        ac[k & 1].v[c] = fmaf(c < split ? ca[k] : cb[k], xv[k].v[c], ac[k & 1].v[c]);
-                }
-        }
-        __syncwarp();  // P, S are rewritten by the next chunk
-    }
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) acc.v[c] = ac[0].v[c] + ac[1].v[c];
-}
-
-// Multi-head GAT with the cp.async ring (gathers that stream from HBM): the
-// per-warp shared memory holds the head block followed by a D-deep ring.
-template <int VEC>
-__device__ __forceinline__ float *mh_warp_ring() {
-    extern __shared__ __align__(16) float tlp_smem[];
-    constexpr int stride = kMhWarpFloats + TLP_DEPTH * 32 * VEC;
-    return tlp_smem + (size_t)(threadIdx.x >> 5) * stride + kMhWarpFloats;
-}
-template <int VEC>
-__device__ __forceinline__ float *mh_warp_smem_async() {
-    extern __shared__ __align__(16) float tlp_smem[];
-    constexpr int stride = kMhWarpFloats + TLP_DEPTH * 32 * VEC;
-    return tlp_smem + (size_t)(threadIdx.x >> 5) * stride;
-}
-
-template <int VEC>
-__device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t e0, int64_t e1,
-                                                      int s, int col, bool active, int64_t rglob,
-                                                      int lane, Vec<VEC> &acc, float *&Mh,
-                                                      float *&Dh, int &h_lo, int &nh, int &hl,
-                                                      int &split) {
-    constexpr int DD = TLP_DEPTH;
-    float *P = mh_warp_smem_async<VEC>();
-    float *M = P + kMhMaxHeads * 32;
-    float *Dn = M + kMhMaxHeads;
-    float *S = Dn + kMhMaxHeads;
-    Mh = M;
-    Dh = Dn;
-    const int H = a.heads, fh = a.fh;
-    const int c_lo = s * 32 * VEC;
-    const int c_hi = min(a.F, c_lo + 32 * VEC) - 1;
-    h_lo = c_lo / fh;
-    nh = c_hi / fh - h_lo + 1;
-    const int cc = active ? col : c_lo;
-    hl = cc / fh - h_lo;
-    split = (hl + h_lo + 1) * fh - cc;
-    const int hl2 = min(hl + (split < VEC ? 1 : 0), nh - 1);
-    for (int hh = lane; hh < nh; hh += 32) {
-        M[hh] = -INFINITY;
-        Dn[hh] = 0.f;
-    }
-    __syncwarp();
-    const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
-    const unsigned row_bytes = (unsigned)a.ldx * 4u;
-    const int32_t *__restrict__ ci = a.colidx + e0;
-    const float *__restrict__ erv = a.er + rglob * H + h_lo;
-    const int len = (int)(e1 - e0);
-    Vec<VEC> ae, ao;
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) ae.v[c] = ao.v[c] = 0.f;
-    if (len > 0) {
-        float *ring = mh_warp_ring<VEC>() + lane * VEC;
-        int n0 = min(32, len), n1 = min(32, len - 32);
-        int u0 = (lane < n0) ? __ldg(ci + lane) : 0;
-        int u1 = (lane < n1) ? __ldg(ci + 32 + lane) : 0;
-#pragma unroll
-        for (int k = 0; k < DD - 1; ++k) {
-            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
-            cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
-            cp_async_commit();
-        }
-        int slot = 0, off = 0;
-        while (true) {
-            const int n2 = min(32, len - off - 64);
-            const int u2 = (lane < n2) ? __ldg(ci + off + 64 + lane) : 0;
-            mh_chunk_scores(a, u0, n0, H, h_lo, nh, erv, lane, P, M, Dn, S);
-            const float sA = S[hl], sB = S[hl2];
-#pragma unroll
-            for (int c = 0; c < VEC; ++c) {
-                const float sc = (c < split) ? sA : sB;
-                ae.v[c] *= sc;
-                ao.v[c] *= sc;
-            }
-            const float *pa = P + hl * 32;
-            const float *pb = P + hl2 * 32;
-            for (int j = 0; j < n0; ++j) {
-                const int jj = j + DD - 1;
-                const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
-                int ws = slot + DD - 1;
-                if (ws >= DD) ws -= DD;
-                cp_async_vec<VEC>(ring + ws * 32 * VEC, row_ptr(base, (unsigned)ui, row_bytes),
-                                  active && (off + jj) < len);
-                cp_async_commit();
-                cp_async_wait<DD - 1>();
-                const float ca = pa[j], cb = pb[j];
-                const float *src = ring + slot * 32 * VEC;
-                Vec<VEC> &ac = (j & 1) ? ao : ae;
-#pragma unroll
-                for (int c = 0; c < VEC; ++c) ac.v[c] = fmaf(c < split ? ca : cb, src[c], ac.v[c]);
-                if (++slot == DD) slot = 0;
-            }
-            __syncwarp();  // P, S are rewritten by the next chunk
-            if (n1 <= 0) break;
-            off += 32;
-            n0 = n1; n1 = n2;
-            u0 = u1; u1 = u2;
-        }
-        cp_async_wait<0>();
-    }
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
-}
-
-// Layer epilogue (NEXT-3, Eq. 2): y = act(y + bias), per element, so it never
-// changes with strip width or gather path.
-template <int VEC>
-__device__ __forceinline__ void apply_layer_epilogue(const AggArgs &a, int col, Vec<VEC> &y) {
-    if (a.bias) {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c)
-            if (col + c < a.F) y.v[c] += __ldg(a.bias + col + c);
-    }
-    if (a.act == TLP_ACT_RELU) {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = y.v[c] > 0.f ? y.v[c] : 0.f;
-    } else if (a.act == TLP_ACT_LEAKY_RELU) {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = y.v[c] >= 0.f ? y.v[c] : a.act_param * y.v[c];
-    } else if (a.act == TLP_ACT_ELU) {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = y.v[c] > 0.f ? y.v[c] : a.act_param * expm1f(y.v[c]);
-    }
-}
-
-// Epilogue (a9) for a full row reduction.
-template <int VEC, int OP>
-__device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_t deg, int col,
-                                             bool active, const Vec<VEC> &acc, float den) {
-    Vec<VEC> y;
-    if constexpr (OP == OP_GATB) {
-        y = acc;  // dX[u] = sum_e alpha_e dY[v_e]
-    } else if constexpr (OP == OP_GCN) {
-        float cin = 1.f;
-        const float dc = (float)(deg > 1 ? deg : 1);
-        if (a.norm == TLP_NORM_RIGHT) cin = 1.0f / dc;
-        else if (a.norm == TLP_NORM_BOTH) cin = 1.0f / sqrtf(dc);
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] * cin;
-    } else if constexpr (OP == OP_GIN) {
-        Vec<VEC> xs;
-        if (active) xs = ld_vec<VEC>(a.X + (a.row_offset + r) * a.ldx + col);
-        else {
-#pragma unroll
-            for (int c = 0; c < VEC; ++c) xs.v[c] = 0.f;
-        }
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = fmaf(a.eps1, xs.v[c], acc.v[c]);
-    } else if constexpr (OP == OP_SAGE) {
-        // mean over N(v) (+ v itself when sage_self): (X[v] + sum) / (deg + 1)
-        const int64_t cnt = deg + a.sage_self;
-        const float inv = 1.0f / (float)(cnt > 1 ? cnt : 1);
-        Vec<VEC> xs;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) xs.v[c] = 0.f;
-        if (a.sage_self && active) xs = ld_vec<VEC>(a.X + (a.row_offset + r) * a.ldx + col);
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = (xs.v[c] + acc.v[c]) * inv;
-    } else {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = deg > 0 ? acc.v[c] / den : 0.f;
-    }
-    apply_layer_epilogue<VEC>(a, col, y);
-    return y;
-}
-
-// Store a finished output vector of local row r: to Y, or (fused all-gather)
-// to the same global row of every destination buffer.
-template <int VEC>
-__device__ __forceinline__ void store_out(const AggArgs &a, int64_t r, int col, const Vec<VEC> &y) {
-    if (a.n_dests == 0) {
-        st_row<VEC>(a.Y + r * a.ldy, col, a.F, y);
-    } else {
-        const int64_t off = (a.row_offset + r) * a.ldy;
-        for (int i = 0; i < a.n_dests; ++i) st_row<VEC>(a.dests[i] + off, col, a.F, y);
-    }
-}
-
-// Column of this lane's vector in strip s (G > 1: strips of 32/G lanes x VEC
-// columns, lanes l and l + 32/G share a column; PAIR = 64-column strips), and
-// whether this lane stores it.
-template <int VEC, int G>
-__device__ __forceinline__ int strip_col(const AggArgs &a, int s, int lane) {
-    constexpr int LG = 32 / G;
-    return (G > 1) ? s * LG * VEC + (lane % LG) * VEC : s * a.lps * VEC + lane * VEC;
-}
-// Whether this lane's column of the strip exists (narrow strips leave lanes
-// >= lps idle; they gather column 0 of the same row, a sector already fetched).
-template <int G>
-__device__ __forceinline__ bool in_strip(const AggArgs &a, int lane, int col) {
-    return (G > 1 || lane < a.lps) && col < a.F;
-}
-template <int G>
-__device__ __forceinline__ bool stores(int lane) {
-    return G == 1 || lane < 32 / G;
-}
-
-// NEXT-3: the strip's partial dots of a finished row vector with att_l, att_r
-// (per-lane fma over the vector, butterfly over the warp; lane 0 stores).
-template <int VEC, int G>
-__device__ __forceinline__ void project_row(const AggArgs &a, int64_t r, int s, int col, bool active,
-                                            const Vec<VEC> &y, int lane) {
-    if (a.proj == nullptr) return;
-    float pl = 0.f, pr = 0.f;
-    if (active && stores<G>(lane)) {
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) {
-            if (col + c < a.F) {
-                if (a.att_l) pl = fmaf(y.v[c], __ldg(a.att_l + col + c), pl);
-                if (a.att_r) pr = fmaf(y.v[c], __ldg(a.att_r + col + c), pr);
-            }
-        }
-    }
-    pl = warp_sum(pl);
-    pr = warp_sum(pr);
-    if (lane == 0) {
-        float *p = a.proj + ((int64_t)s * a.n_dst + r) * 2;
-        p[0] = pl;
-        p[1] = pr;
-    }
-}
-
-
-// OP_GATB: the transposed row's own forward features X[u] for this lane's
-// columns of strip s, and where the strip's edge dot products go.
-template <int VEC, int OP>
-__device__ __forceinline__ void gatb_self(const AggArgs &a, int64_t r, int s, int64_t e0, int col,
-                                          bool active, Vec<VEC> &xu, float *&gout) {
-#pragma unroll
-    for (int c = 0; c < VEC; ++c) xu.v[c] = 0.f;
-    if constexpr (OP == OP_GATB) {
-        if (active) xu = ld_vec<VEC>(a.xself + r * a.ldxs + col);
-        gout = a.gbuf + (int64_t)s * a.gstride + e0;
-    }
-}
-
-// A regular work unit: whole rows [r0, r1), feature strips [s0, s1).
-template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0, int s1,
-                                        int lane) {
-    for (int rb = r0; rb < r1; rb += 31) {
-        const int nr = min(31, r1 - rb);
-        // lanes fetch the row offsets of up to 31 rows at once (register caching
-        // of the index boundary, Fig. 7a)
-        int64_t rp = 0;
-        if (lane <= nr) rp = __ldg(a.rowptr + rb + lane);
-        float erl = 0.f;
-        if constexpr (OP == OP_GAT)
-            if (lane < nr) erl = __ldg(a.er + a.row_offset + rb + lane);
-        for (int k = 0; k < nr; ++k) {
-            const int64_t e0 = __shfl_sync(FULL, rp, k);
-            const int64_t e1 = __shfl_sync(FULL, rp, k + 1);
-            const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
-            const int64_t r = rb + k;
-            for (int s = s0; s < s1; ++s) {
-                const int col = strip_col<VEC, G>(a, s, lane);
-                const bool active = in_strip<G>(a, lane, col);
-                Vec<VEC> acc;
-#pragma unroll
-                for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
-                float m = -INFINITY, den = 0.f;
-                if constexpr (OP == OP_GATH) {
-                    float *Mh, *Dh;
-                    int h_lo, nh, hl, split;
-                    if constexpr (ASYNC)
-                        reduce_edges_mh_async<VEC>(a, e0, e1, s, col, active, a.row_offset + r, lane,
-                                                   acc, Mh, Dh, h_lo, nh, hl, split);
-                    else
-                        reduce_edges_mh<VEC, U>(a, e0, e1, s, col, active, a.row_offset + r, lane, acc,
-                                                Mh, Dh, h_lo, nh, hl, split);
-                    const float dA = Dh[hl], dB = Dh[min(hl + 1, nh - 1)];
-                    __syncwarp();  // the head state is reset by the next strip / row
-                    Vec<VEC> y;
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c)
-                        y.v[c] = (e1 > e0) ? acc.v[c] / (c < split ? dA : dB) : 0.f;
-                    apply_layer_epilogue<VEC>(a, col, y);
-                    if (active) store_out<VEC>(a, r, col, y);
-                    continue;
-                } else if constexpr (ASYNC) {
-                    reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
-                } else {
-                    Vec<VEC> xu;
-                    float *gout = nullptr;
-                    gatb_self<VEC, OP>(a, r, s, e0, col, active, xu, gout);
-                    reduce_edges<VEC, OP, COEF, U, G>(a, e0, e1, col, active, er_v, lane, acc, m, den,
-                                                         xu, gout);
-                }
-                Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
-                if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
-                project_row<VEC, G>(a, r, s, col, active, y, lane);
-            }
-        }
-    }
-}
-
-// One C-edge chunk of hub h (a8), feature strips [s0, s1).  The last chunk of
-// the hub to finish these strips merges all its partials in chunk order and
-// writes the row.  Tickets (and GAT (m, den) pairs) are kept per panel s0.
-template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int s0, int s1,
-                                             int lane) {
-    const int r = __ldg(a.hub_row + h);
-    const int off = __ldg(a.hub_off + h);
-    const int nch = __ldg(a.hub_off + h + 1) - off;
-    const int64_t eb = __ldg(a.rowptr + r), ee = __ldg(a.rowptr + r + 1);
-    const int64_t e0 = eb + (int64_t)j * a.C;
-    const int64_t e1 = min(e0 + a.C, ee);
-    float er_v = 0.f;
-    if constexpr (OP == OP_GAT) er_v = __ldg(a.er + a.row_offset + r);
-    const int slot = off + j;
-    // this panel's (m, den) pairs: [n_chunks][heads] (heads = 1 unless OP_GATH)
-    const int mdh = (OP == OP_GATH) ? a.heads : 1;
-    float *md = a.md + 2 * (int64_t)s0 * a.n_chunks * mdh;
-    int32_t *ticket = a.hub_ticket + (int64_t)s0 * a.n_hubs + h;
-    for (int s = s0; s < s1; ++s) {
-        const int col = strip_col<VEC, G>(a, s, lane);
-        const bool active = in_strip<G>(a, lane, col);
-        Vec<VEC> acc;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
-        float m = -INFINITY, den = 0.f;
-        if constexpr (OP == OP_GATH) {
-            float *Mh, *Dh;
-            int h_lo, nh, hl, split;
-            if constexpr (ASYNC)
-                reduce_edges_mh_async<VEC>(a, e0, e1, s, col, active, a.row_offset + r, lane, acc, Mh,
-                                           Dh, h_lo, nh, hl, split);
-            else
-                reduce_edges_mh<VEC, U>(a, e0, e1, s, col, active, a.row_offset + r, lane, acc, Mh, Dh,
-                                        h_lo, nh, hl, split);
-            for (int hh = lane; hh < nh; hh += 32) {
-                md[2 * ((int64_t)slot * mdh + h_lo + hh)] = Mh[hh];
-                md[2 * ((int64_t)slot * mdh + h_lo + hh) + 1] = Dh[hh];
-            }
-            __syncwarp();
-        } else if constexpr (ASYNC) {
-            reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
-        } else {
-            Vec<VEC> xu;
-            float *gout = nullptr;
-            gatb_self<VEC, OP>(a, r, s, e0, col, active, xu, gout);
-            reduce_edges<VEC, OP, COEF, U, G>(a, e0, e1, col, active, er_v, lane, acc, m, den, xu,
-                                                 gout);
-        }
-        if (active && stores<G>(lane)) st_vec<VEC>(a.scratch + (int64_t)slot * a.ldp + col, acc);
-        if constexpr (OP == OP_GAT)
-            if (s == s0 && lane == 0) {
-                md[2 * (int64_t)slot] = m;
-                md[2 * (int64_t)slot + 1] = den;
-            }
-    }
-    __threadfence();
-    __syncwarp();
-    int last = 0;
-    if (lane == 0) last = (atomicAdd(ticket, 1) == nch - 1);
-    last = __shfl_sync(FULL, last, 0);
-    if (!last) return;
-    __threadfence();
-    float M = -INFINITY, D = 0.f;
-    if constexpr (OP == OP_GAT) {
-        for (int q = 0; q < nch; ++q) M = fmaxf(M, __ldcg(md + 2 * (int64_t)(off + q)));
-        for (int q = 0; q < nch; ++q) {
-            const float mq = __ldcg(md + 2 * (int64_t)(off + q));
-            const float dq = __ldcg(md + 2 * (int64_t)(off + q) + 1);
-            D = fmaf(dq, __expf(mq - M), D);
-        }
-    }
-    for (int s = s0; s < s1; ++s) {
-        const int col = strip_col<VEC, G>(a, s, lane);
-        const bool active = in_strip<G>(a, lane, col);
-        // OP_GATH: the lane's (up to two) heads and their merged softmax states
-        int64_t mA = 0, mB = 0;
-        int split = VEC;
-        float MA = -INFINITY, DA = 0.f, MB = -INFINITY, DB = 0.f;
-        if constexpr (OP == OP_GATH) {
-            const int cc = active ? col : s * a.lps * VEC;
-            mA = cc / a.fh;
-            split = (int)((mA + 1) * a.fh - cc);
-            mB = min(mA + (split < VEC ? 1 : 0), (int64_t)a.heads - 1);
-            for (int q = 0; q < nch; ++q) {
-                MA = fmaxf(MA, __ldcg(md + 2 * ((int64_t)(off + q) * mdh + mA)));
-                MB = fmaxf(MB, __ldcg(md + 2 * ((int64_t)(off + q) * mdh + mB)));
-            }
-            for (int q = 0; q < nch; ++q) {
-                const float *pa = md + 2 * ((int64_t)(off + q) * mdh + mA);
-                const float *pb = md + 2 * ((int64_t)(off + q) * mdh + mB);
-                DA = fmaf(__ldcg(pa + 1), __expf(__ldcg(pa) - MA), DA);
-                DB = fmaf(__ldcg(pb + 1), __expf(__ldcg(pb) - MB), DB);
-            }
-        }
-        Vec<VEC> acc;
-#pragma unroll
-        for (int c = 0; c < VEC; ++c) acc.v[c] = 0.f;
-        if (active) {
-            for (int q = 0; q < nch; ++q) {
-                Vec<VEC> p = ld_vec_cg<VEC>(a.scratch + (int64_t)(off + q) * a.ldp + col);
-                if constexpr (OP == OP_GATH) {
-                    const float wA = __expf(__ldcg(md + 2 * ((int64_t)(off + q) * mdh + mA)) - MA);
-                    const float wB = __expf(__ldcg(md + 2 * ((int64_t)(off + q) * mdh + mB)) - MB);
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) acc.v[c] = fmaf(c < split ? wA : wB, p.v[c], acc.v[c]);
-                } else if constexpr (OP == OP_GAT) {
-                    const float w = __expf(__ldcg(md + 2 * (int64_t)(off + q)) - M);
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) acc.v[c] = fmaf(w, p.v[c], acc.v[c]);
-                } else {
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) acc.v[c] += p.v[c];
-                }
-            }
-        }
-        Vec<VEC> y;
-        if constexpr (OP == OP_GATH) {
-#pragma unroll
-            for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] / (c < split ? DA : DB);
-            apply_layer_epilogue<VEC>(a, col, y);
-        } else {
-            y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
-        }
-        if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
-        if constexpr (OP != OP_GATH) project_row<VEC, G>(a, r, s, col, active, y, lane);
-    }
-    if (lane == 0) *ticket = 0;  // self-reset for the next launch
-}
-
-// Work item i: task-major (all strips of task i) or, in panel mode, strip
-// s = i / n_tasks of task i % n_tasks, so that all warps sweep one L2-resident
-// feature panel of X at a time.
-template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
-    int64_t t = i;
-    int s0 = 0, s1 = a.n_strips;
-    if (a.panel) {
-        s0 = (int)(i / a.n_tasks);
-        t = i - (int64_t)s0 * a.n_tasks;
-        s1 = s0 + 1;
-    }
-    const int2 tk = a.tasks[t];
-    if (tk.y >= 0) do_unit<VEC, OP, COEF, U, ASYNC, G>(a, tk.x, tk.y, s0, s1, lane);
-    else do_hub_chunk<VEC, OP, COEF, U, ASYNC, G>(a, tk.x, -tk.y - 1, s0, s1, lane);
-}
-
-// Resident CTAs per SM the kernel is compiled for (register budget).  The
-// coefficient-free sums (GIN, SAGE, GCN NONE / RIGHT / pre-scaled BOTH) fit 64
-// registers, so they run 32 warps per SM (measured: Reddit GIN 24.0 -> 21.8
-// ms); ops with an edge coefficient (weighted, GAT) keep 85 registers (24
-// warps), where fewer registers spill into the edge loop (measured slower;
-// the alpha-mode GAT gather at 4 CTAs/SM: 26.9 -> 31.0 ms on Reddit).
-constexpr int min_blocks(int op, int coef, bool async, int G = 1) {
-    return async ? TLP_MINB_ASYNC
-         : (TLP_SMEMC && G > 1 && coef != COEF_NONE && (op == OP_GCN || op == OP_GIN || op == OP_GATB))
-               ? TLP_MINB_SMC
-                 : ((op == OP_GIN || op == OP_SAGE || op == OP_GCN) && coef == COEF_NONE)
-                       ? TLP_MINB_LIGHT : TLP_MINB;
-}
-
-template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__device__ __forceinline__ void agg_body(const AggArgs &a) {
-    const int lane = threadIdx.x & 31;
-    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (a.sched == S_HARDWARE) {  // one warp per item
-        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC, G>(a, wid, lane);
-        if (a.n_dests > 0) __threadfence_system();
-        return;
-    }
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t stride = W * a.step;
-    int64_t t = wid * a.step;  // static first wave
-    while (t < a.n_items) {
-        unsigned long long v = 0;
-        if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned long long)a.step);
-        const int64_t tend = min(t + a.step, a.n_items);
-        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, G>(a, tt, lane);
-        if (a.sched == S_DYNAMIC) t = stride + (int64_t)__shfl_sync(FULL, v, 0);
-        else t += stride;
-    }
-    if (a.n_dests > 0) __threadfence_system();  // peer stores visible before the barrier
-    if (a.sched == S_DYNAMIC && lane == 0) {
-        // last warp out resets the counter: no memset launch between calls
-        __threadfence();
-        if (atomicAdd(a.done, 1u) == (unsigned)(W - 1)) {
-            *a.ctr = 0ull;
-            *a.done = 0u;
-            __threadfence();
-        }
-    }
-}
-
-template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__global__ void __launch_bounds__(TLP_MAXT, min_blocks(OP, COEF, ASYNC, G)) k_agg(const AggArgs a) {
-    agg_body<VEC, OP, COEF, U, ASYNC, G>(a);
-}
-
 // ------------------------------------------------------------- dispatch --
-
-constexpr int kU = TLP_U;  // source rows per gather group (2 groups in flight)
-
-typedef void (*KernelFn)(const AggArgs);
-
-template <int VEC, bool ASYNC, int G>
-static KernelFn pick(int op, int coef) {
-    if (op == OP_GCN) {
-        switch (coef) {
-            case COEF_NONE: return k_agg<VEC, OP_GCN, COEF_NONE, kU, ASYNC, G>;
-            case COEF_COUT: return k_agg<VEC, OP_GCN, COEF_COUT, kU, ASYNC, G>;
-            case COEF_W: return k_agg<VEC, OP_GCN, COEF_W, kU, ASYNC, G>;
-            default: return k_agg<VEC, OP_GCN, COEF_W_COUT, kU, ASYNC, G>;
-        }
-    }
-    if (op == OP_GIN)
-        return coef & COEF_W ? k_agg<VEC, OP_GIN, COEF_W, kU, ASYNC, G>
-                             : k_agg<VEC, OP_GIN, COEF_NONE, kU, ASYNC, G>;
-    if (op == OP_SAGE) return k_agg<VEC, OP_SAGE, COEF_NONE, kU, ASYNC, G>;
-    if constexpr (!ASYNC && G <= 2)
-        if (op == OP_GATB) return k_agg<VEC, OP_GATB, COEF_W, kU, false, G>;
-    return k_agg<VEC, OP_GAT, COEF_NONE, kU, ASYNC, G>;
-}
-
-// multi-head GAT: full-warp register path or cp.async ring
-static KernelFn pick_mh(int vec, bool async_path) {
-    if (async_path)
-        return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, true, 1>
-                        : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, true, 1>
-                                   : k_agg<1, OP_GATH, COEF_NONE, kU, true, 1>;
-    return vec == 4 ? k_agg<4, OP_GATH, COEF_NONE, kU, false, 1>
-                    : vec == 2 ? k_agg<2, OP_GATH, COEF_NONE, kU, false, 1>
-                               : k_agg<1, OP_GATH, COEF_NONE, kU, false, 1>;
-}
 
 // gather path: 0 register (full warp), 1 cp.async ring, 2 register with G
 // lane groups (G = 2: PAIR half-warps; 4, 8: narrow rows; VEC = 4)
 static KernelFn pick_kernel(int path, int vec, int op, int coef, int groups) {
     if (path == 2) {
-        if (groups == 8) return pick<4, false, 8>(op, coef);
-        if (groups == 4) return pick<4, false, 4>(op, coef);
-        return pick<4, false, 2>(op, coef);
+        if (groups == 8) return pick_g8(op, coef);
+        if (groups == 4) return pick_g4(op, coef);
+        return pick_g2(op, coef);
     }
-    if (path == 1)
-        return vec == 4 ? pick<4, true, 1>(op, coef) : vec == 2 ? pick<2, true, 1>(op, coef)
-                                                               : pick<1, true, 1>(op, coef);
-    return vec == 4 ? pick<4, false, 1>(op, coef) : vec == 2 ? pick<2, false, 1>(op, coef)
-                                                             : pick<1, false, 1>(op, coef);
+    if (path == 1) return vec == 4 ? pick_async_v4(op, coef) : pick_async_v21(vec, op, coef);
+    return vec == 4 ? pick_reg_v4(op, coef) : pick_reg_v21(vec, op, coef);
 }
 
 static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
@@ -1426,19 +50,23 @@ static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
 
 static bool aligned(const void *p, size_t a) { return ((uintptr_t)p % a) == 0; }
 
-// X'[u, f] = c_out[u] * X[u, f] for f < F (unweighted GCN BOTH); the pad
-// columns of the last vector are zeroed (gathered, never stored to Y).
+// Gather copy of X: out[u, f] = c_out[u] * X[u, f]
+// (unweighted GCN BOTH pre-scaling; c_out = NULL copies) for f < F, written
+// row-major with leading dimension out_ld, or (pw > 0) panel-major: column f
+// of row u at out + (f / pw) * gps + u * pw + f % pw.  The pad columns of the
+// last vector are zeroed (they are gathered, never stored to Y).
 template <int VEC>
-__global__ void k_prescale(const float *__restrict__ X, const float *__restrict__ c_out, int64_t n,
-                           int64_t F, int64_t ldx, int64_t nvec, float *__restrict__ Xs) {
+__global__ void k_repack(const float *__restrict__ X, const float *__restrict__ c_out, int64_t n,
+                         int64_t F, int64_t ldx, int64_t nvec, float *__restrict__ out,
+                         int64_t out_ld, int pw, int64_t gps) {
     const int64_t tot = n * nvec;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < tot;
          i += (int64_t)gridDim.x * blockDim.x) {
         const int64_t u = i / nvec;
         const int64_t c = (i - u * nvec) * VEC;
-        const float cu = __ldg(c_out + u);
+        const float cu = c_out ? __ldg(c_out + u) : 1.0f;
         const float *src = X + u * ldx + c;
-        float *dst = Xs + u * ldx + c;
+        float *dst = pw ? out + (c / pw) * gps + u * pw + (c % pw) : out + u * out_ld + c;
         if constexpr (VEC == 4) {
             if (c + 4 <= F) {
                 const float4 x = __ldg(reinterpret_cast<const float4 *>(src));
@@ -1452,8 +80,6 @@ __global__ void k_prescale(const float *__restrict__ X, const float *__restrict_
                 continue;
             }
         }
-        // the ragged last vector: columns [F, c + VEC) lie inside ldx (vec was
-        // chosen from ldx % VEC) and are read by the gathers, so define them
         for (int k = 0; k < VEC; ++k) dst[k] = (c + k < F) ? cu * __ldg(src + k) : 0.f;
     }
 }
@@ -2006,41 +632,6 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             ew = g->galpha;
         }
     }
-    // Unweighted GCN BOTH (DESIGN.md "GCN BOTH pre-scaling"): one pass writes
-    // X'[u] = c_out[u] X[u] (each term rounded once, as the oracle's product),
-    // then every gather path sums X' rows with no per-edge coefficient, i.e.
-    // the register budget and instruction count of GIN.  Same bits on every
-    // path, schedule and partition (every path gathers the same X').
-    const float *Xg = r.X;
-    if (prescale) {
-        const size_t need = sizeof(float) * ((size_t)g->n_src * (size_t)r.ldx) + 64;
-        if (need > g->xs_bytes) {
-            if (g->xs) {
-                cudaFreeAsync(g->xs, s);
-                g->device_bytes -= g->xs_bytes;
-                g->xs = nullptr;
-                g->xs_bytes = 0;
-            }
-            cudaError_t e = cudaMallocAsync((void **)&g->xs, need, s);
-            if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(prescaled X)");
-            g->xs_bytes = need;
-            g->device_bytes += need;
-        }
-        const int64_t nvec = (r.F + vec - 1) / vec;
-        const int64_t tot = g->n_src * nvec;
-        const int pb = (int)std::max<int64_t>(1, std::min<int64_t>((tot + 255) / 256, (int64_t)g->num_sms * 16));
-        if (vec == 4)
-            k_prescale<4><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
-        else if (vec == 2)
-            k_prescale<2><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
-        else
-            k_prescale<1><<<pb, 256, 0, s>>>(r.X, g->c_out, g->n_src, r.F, r.ldx, nvec, g->xs);
-        g->launches += 1;
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return cuda_error(e, "k_prescale launch");
-        Xg = g->xs;
-    }
-
     // Feature panels: when X is much larger than
     // L2, sweep the graph once per column strip so the strip of X being
     // gathered (n_src x strip width x 4 bytes) stays L2-resident while every
@@ -2108,12 +699,85 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (!panel && !panel_off && n_strips > 1 && g->n_tasks < (int64_t)g->num_sms * 32 * 4) panel = 1;
     if (n_strips < 2) panel = 0;
 
+    // Gather layout.  In panel mode every edge
+    // gathers one strip of a source row from L2; a strip that is not 128-byte
+    // aligned touches one more cache line and one more sector per gather and
+    // inflates the L2 footprint of the panel (measured on Reddit, F = 602:
+    // ld 604 -> 608 cut DRAM reads 50 -> 22 GB per launch, GIN 21.5 -> 17.8
+    // ms).  So when the caller's rows are not 128-byte aligned, the gathers read
+    // a copy of X written by one streaming pass (read + write of n_src x F,
+    // ~1 % of a Reddit launch): padded rows (ld rounded up to 32 floats) or
+    // panel-major blocks of strip_w columns.  The unweighted GCN-BOTH
+    // pre-scale writes its X' in the same layout at no extra cost.  Values are
+    // copied bit for bit (or scaled exactly as before), so no output bit changes.
+    // TLP_LAYOUT=caller|padded|panel overrides.
+    int layout = 0;  // 0 caller, 1 padded rows, 2 panel-major
+    if (panel && vec == 4 && op != OP_GATH &&
+        4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes) {
+        const bool misaligned = (r.ldx % 32) != 0 || !aligned(r.X, 128);
+        layout = misaligned ? 1 : 0;
+        if (const char *e = getenv("TLP_LAYOUT")) {
+            if (!strcmp(e, "caller")) layout = 0;
+            else if (!strcmp(e, "padded")) layout = 1;
+            else if (!strcmp(e, "panel")) layout = 2;
+        }
+        if (layout == 2 && strip_w % 4 != 0) layout = 1;
+    }
+    // Unweighted GCN BOTH (DESIGN.md "GCN BOTH pre-scaling"): one pass writes
+    // X'[u] = c_out[u] X[u] (each term rounded once, as the oracle's product),
+    // then every gather path sums X' rows with no per-edge coefficient, i.e.
+    // the register budget and instruction count of GIN.  Same bits on every
+    // path, schedule and partition (every path gathers the same X').
+    const float *Xg = r.X;
+    int64_t ldg = r.ldx, gps = 0;
+    if (prescale || layout != 0) {
+        if (layout == 1) ldg = (r.F + 31) / 32 * 32;
+        if (layout == 2) {
+            ldg = strip_w;
+            gps = g->n_src * (int64_t)strip_w;
+        }
+        const size_t need = sizeof(float) * (layout == 2 ? (size_t)n_strips * (size_t)gps
+                                                           : (size_t)g->n_src * (size_t)ldg) + 256;
+        if (need > g->xs_bytes) {
+            if (g->xs) {
+                cudaFreeAsync(g->xs, s);
+                g->device_bytes -= g->xs_bytes;
+                g->xs = nullptr;
+                g->xs_bytes = 0;
+            }
+            cudaError_t e = cudaMallocAsync((void **)&g->xs, need, s);
+            if (e != cudaSuccess) return cuda_error(e, "cudaMallocAsync(prescaled X)");
+            g->xs_bytes = need;
+            g->device_bytes += need;
+        }
+        const int64_t nvec = (r.F + vec - 1) / vec;
+        const int64_t tot = g->n_src * nvec;
+        const int pb = (int)std::max<int64_t>(1, std::min<int64_t>((tot + 255) / 256, (int64_t)g->num_sms * 16));
+        const float *cs = prescale ? g->c_out : nullptr;
+        const int pw = layout == 2 ? strip_w : 0;
+        if (vec == 4)
+            k_repack<4><<<pb, 256, 0, s>>>(r.X, cs, g->n_src, r.F, r.ldx, nvec, g->xs, ldg, pw, gps);
+        else if (vec == 2)
+            k_repack<2><<<pb, 256, 0, s>>>(r.X, cs, g->n_src, r.F, r.ldx, nvec, g->xs, ldg, pw, gps);
+        else
+            k_repack<1><<<pb, 256, 0, s>>>(r.X, cs, g->n_src, r.F, r.ldx, nvec, g->xs, ldg, pw, gps);
+        g->launches += 1;
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "k_repack launch");
+        Xg = g->xs;
+    }
+
+
     AggArgs a;
     a.rowptr = g->rowptr;
     a.colidx = g->colidx;
     a.ew = ew;
     a.c_out = cvec;
     a.X = Xg;
+    a.xown = r.X;
+    a.ldown = r.ldx;
+    a.gps = gps;
+    a.pw = strip_w;
     a.Y = r.Y;
     a.el = r.el;
     a.er = r.er;
@@ -2122,7 +786,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.hub_off = g->hub_off;
     a.ctr = reinterpret_cast<unsigned long long *>(g->ctr);
     a.done = g->ctr + 2;
-    a.ldx = r.ldx;
+    a.ldx = ldg;
     a.ldy = r.ldy;
     a.ldp = (r.F + 3) / 4 * 4;
     a.row_offset = g->row_offset;

@@ -1,0 +1,10 @@
+// tlp_k_g8.cu -- one family of aggregation kernel specialisations (see
+// tlp_agg_kernels.cuh); a separate translation unit so the library builds in
+// parallel.
+#include "tlp_agg_kernels.cuh"
+
+namespace tlp {
+
+KernelFn pick_g8(int op, int coef) { return pick<4, false, 8>(op, coef); }
+
+}  // namespace tlp
