@@ -71,25 +71,32 @@ def gather_bytes(op, n_rows, n_edges, F):
     raise ValueError(op)
 
 
-def l2_gather_peak():
-    """Measured L2-resident random-row gather bandwidth (256-byte rows, the
-    largest table that still fits L2 like a 64-column panel), or None."""
-    p = os.path.join(ROOT, "profiles", "l2_gather_probe.jsonl")
-    try:
-        rows, mhz = [], None
-        for line in open(p):
-            line = line.strip()
-            if line.startswith("{"):
-                rows.append(json.loads(line))
-            elif line.endswith("MHz"):
-                mhz = line.split()[0]
-        cands = [r for r in rows if r["row_bytes"] == 256 and r["table_MB"] < 80]
-        best = max(cands, key=lambda r: r["table_MB"] * 1e6 + r["GBs"])
-        best = max([r for r in cands if r["table_MB"] == best["table_MB"]], key=lambda r: r["GBs"])
-        best["sm_mhz"] = mhz
-        return best
-    except (OSError, ValueError, KeyError):
+def l2_gather_ceiling(table_bytes, iters=600):
+    """In-run L2 random-row gather ceiling (bench_probe/l2_ceiling.cu, built by
+    __graft_entry__.build()): GB/s of 256-byte random-row gathers from an
+    L2-resident table of `table_bytes` (one panel-major strip block), or None."""
+    import ctypes
+    p = os.path.join(ROOT, "bench_probe", "libl2c.so")
+    if not os.path.exists(p):
         return None
+    lib = ctypes.CDLL(p)
+    lib.l2c_run.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.POINTER(ctypes.c_float),
+                            ctypes.POINTER(ctypes.c_double)]
+    ms, by = ctypes.c_float(), ctypes.c_double()
+    if lib.l2c_run(int(table_bytes), int(iters), ctypes.byref(ms), ctypes.byref(by)) != 0:
+        return None
+    return {"GBs": round(by.value / (ms.value * 1e-3) / 1e9, 1), "ms": round(ms.value, 3),
+            "table_MB": round(table_bytes / 1e6, 1)}
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def peak_hbm():
@@ -123,7 +130,7 @@ class ClockSampler:
 
     def __init__(self, gpu_index, period_ms=None):
         self.gpu = gpu_index
-        self.period = int(period_ms or os.environ.get("TLP_CLOCK_MS", "500"))
+        self.period = int(period_ms or os.environ.get("TLP_CLOCK_MS", "50"))
         self.proc = None
         self.lines = []
 
@@ -265,9 +272,21 @@ def run_tlp(args):
     rp_d = torch.from_numpy(rp).to(dev)
     ci_d = torch.from_numpy(ci).to(dev)
     comm = None
+    if use_dist:
+        # the driver counts ranks from NCCL's init log
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        comm = tlp.comm_from_torch()
+    # first create of the process: includes loading the library's create
+    # kernels (CUDA lazy module loading); then the warm create of the real
+    # graph (SURVEY 8(a) a1 target: create < 1 % of one aggregation)
+    t0 = time.perf_counter()
+    tiny = tlp.Graph(torch.tensor([0, 1], device=dev), torch.tensor([0], dtype=torch.int32, device=dev))
+    torch.cuda.synchronize()
+    first_create_ms = (time.perf_counter() - t0) * 1e3
+    tiny.close()
     t0 = time.perf_counter()
     if use_dist:
-        comm = tlp.comm_from_torch()
         g = tlp.Graph.dist(comm, rp_d, ci_d)
     else:
         g = tlp.Graph(rp_d, ci_d)
@@ -504,6 +523,45 @@ def run_tlp(args):
         for op in Yp:
             assert torch.equal(Yp[op][:64].to(dev), last[op][:64])
 
+    # ---- dist: the local aggregation and the all-gather timed separately ----
+    dist_split = None
+    if use_dist and not fused and graphs is None and all(o in ("gcn", "gin", "gat", "sage") for o in ops):
+        b = tlp.tlp_dist_bounds(g.handle, world)
+        lo, hi = int(b[rank]), int(b[rank + 1])
+        comp = {op: [] for op in ops}
+        gath = {op: [] for op in ops}
+        dist.barrier()
+        torch.cuda.synchronize()
+        for _ in range(max(3, min(args.steps, 10))):
+            for op in ops:
+                ys = Y[op][lo:hi]
+                a1, a2, a3 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                a1.record(stream)
+                if op in ("gcn", "gcn2"):
+                    g.gcn(X, "both", Y=ys, F=F)
+                elif op == "gin":
+                    g.gin(X, synth.EPS, Y=ys, F=F)
+                elif op == "sage":
+                    g.sage(X, True, Y=ys, F=F)
+                else:
+                    g.gat(X, el, er, synth.SLOPE, Y=ys, F=F)
+                a2.record(stream)
+                tlp.tlp_dist_allgather_rows(g.handle, comm, Y[op], stream=stream)
+                a3.record(stream)
+                comp[op].append((a1, a2))
+                gath[op].append((a2, a3))
+        torch.cuda.synchronize()
+        dist_split = {}
+        for op in ops:
+            tc = torch.tensor([statistics.median([x.elapsed_time(y) for x, y in comp[op]]),
+                               statistics.median([x.elapsed_time(y) for x, y in gath[op]])], device=dev)
+            dist.all_reduce(tc, op=dist.ReduceOp.MAX)
+            ybytes = n * ld * 4
+            dist_split[op] = {"compute_ms": round(float(tc[0]), 4), "allgather_ms": round(float(tc[1]), 4),
+                              "allgather_bytes": int(ybytes),
+                              "allgather_busbw_GBs": round(ybytes * (world - 1) / world
+                                                           / (float(tc[1]) * 1e-3) / 1e9, 1)}
+
     # ---- roofline of the dominant kernel ----
     peak, peak_src = peak_hbm()
     per_op = {}
@@ -523,27 +581,38 @@ def run_tlp(args):
     dom = max(ops, key=lambda o: per_op[o]["ms_mean"])
     traffic = load_traffic(name).get(dom)
     achieved = per_op[dom]["gather_GBs"]
-    roofline = {"bound": "hbm", "kernel": f"k_agg ({dom})", "achieved": achieved,
-                "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4),
-                "traffic": traffic, "peak_source": peak_src,
+    # L2-panel mode (X larger than L2, a 64-column strip block fits): the
+    # gathered rows are L2 hits, so the bound is the L2 random-row gather rate,
+    # measured in this run by the probe (same clocks, same box)
+    panel = n * ld * 4 > 0.6 * 126e6 and n * 256 <= 0.6 * 126e6 and F > 64
+    roofline = {"kernel": f"k_agg ({dom})", "achieved": achieved, "unit": "GB/s",
                 "bytes_per_launch": per_op[dom]["gather_bytes"],
-                "bytes_model": "gather model: per edge 4F+4 colidx+4 coef/el; per row Y, rowptr (+self/er)"}
+                "bytes_model": "gather model (SURVEY 8(d) d2): per edge 4F + 4 colidx + 4 coef/el; "
+                               "per row Y, rowptr (+self/er); time = the op's mean CUDA-event "
+                               "duration over the timed region (all of its launches)",
+                "traffic": traffic,
+                "traffic_source": "profiles/ncu_traffic.json (dram__bytes_read.sum + "
+                                  "dram__bytes_write.sum per launch, ncu --set full of this round's kernels)"}
+    probe = None
+    if panel and rank == 0:
+        with ClockSampler(local) as pclk:
+            probe = l2_gather_ceiling(n * 256)
+        if probe:
+            probe["clocks"] = pclk.summary()
+    if probe:
+        roofline.update({"bound": "l2", "peak": probe["GBs"], "frac": round(achieved / probe["GBs"], 4),
+                         "peak_source": "measured in this run: bench_probe/l2_ceiling.cu, random "
+                                        "256-byte rows of a %.0f MB L2-resident table (one strip "
+                                        "block), persistent grid at the kernel's occupancy" % probe["table_MB"],
+                         "probe": probe})
+    else:
+        roofline.update({"bound": "hbm", "peak": peak, "frac": round(achieved / peak, 4),
+                         "peak_source": peak_src})
     if traffic:
-        # DRAM bytes the ncu capture measured per launch, over this run's launch time:
-        # what actually crossed HBM (the rest of the gather model is served by L2)
-        roofline["traffic_GBs"] = round(traffic / (per_op[dom]["ms_mean"] * 1e-3) / 1e9, 1)
-        roofline["traffic_frac_of_peak"] = round(roofline["traffic_GBs"] / peak, 4)
-        roofline["note"] = ("frac > 1: feature panels keep the gathered slice of X in L2, so most of "
-                            "the gather-model bytes are L2 hits; traffic_GBs is the HBM rate")
-    l2 = l2_gather_peak()
-    if l2:
-        # the ceiling that binds when the gathered rows are L2-resident (panel mode):
-        # random-row L2 gather bandwidth measured by scripts/l2_probe.cu on a B200
-        roofline["l2_gather"] = {"peak": l2["GBs"], "unit": "GB/s",
-                                 "frac": round(achieved / l2["GBs"], 4),
-                                 "source": "profiles/l2_gather_probe.jsonl (%d-byte rows, %.0f MB "
-                                           "table, sm clock at measurement %s)"
-                                           % (l2["row_bytes"], l2["table_MB"], l2.get("sm_mhz"))}
+        # DRAM bytes per launch over this run's launch time: the HBM rate
+        roofline["hbm"] = {"achieved": round(traffic / (per_op[dom]["ms_mean"] * 1e-3) / 1e9, 1),
+                           "peak": peak, "peak_source": peak_src, "unit": "GB/s"}
+        roofline["hbm"]["frac"] = round(roofline["hbm"]["achieved"] / peak, 4)
 
     result = {
         "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
@@ -562,12 +631,15 @@ def run_tlp(args):
                        "grouped-broadcast all-gather of Y")) if use_dist else "single",
                    "frac_of_8TBs": round(value / NOMINAL_HBM_GBS, 4)},
         "ops": per_op, "create_ms": round(create_ms, 1),
+        "create_first_ms": round(first_create_ms, 1),
         "plan": {k: info[k] for k in ("n_hubs", "n_hub_chunks", "n_units", "n_tasks",
                                       "hub_threshold", "hub_chunk", "max_in_degree")},
         "roofline": roofline,
         "gpu_launches": int(n_launches),
         "clocks": clk.summary(), "e2e": e2e,
     }
+    if dist_split:
+        result["dist"] = dist_split
     w = WORKLOADS[name]
     if "paper_v100_ms" in w:
         # context only (another GPU, the paper's own F = 32 measurement)
@@ -636,13 +708,69 @@ def _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds, seed=0):
     return np.sort(perm[:k])
 
 
+def _pool_worker(job):
+    """One process of the all-core oracle run: its chunk of rows, inputs
+    memory-mapped from the shared directory (no copies)."""
+    d, name, F, rows = job
+    rp = np.load(os.path.join(d, "rp.npy"), mmap_mode="r")
+    ci = np.load(os.path.join(d, "ci.npy"), mmap_mode="r")
+    Xh = np.load(os.path.join(d, "X.npy"), mmap_mode="r")
+    elh = np.load(os.path.join(d, "el.npy"), mmap_mode="r")
+    erh = np.load(os.path.join(d, "er.npy"), mmap_mode="r")
+    cfg = {"F": F}
+    t0 = time.perf_counter()
+    by, _ = _oracle_rows(name, cfg, np.asarray(rp), ci, Xh, elh, erh, rows)
+    return by, time.perf_counter() - t0
+
+
+def oracle_all_cores(name, cfg, rp, ci, Xh, elh, erh, rows, cores):
+    """The oracle as it stands, on `cores` processes over disjoint row chunks
+    (rows are independent, so every output is the single-threaded one, bit for
+    bit).  Returns (bytes, wall seconds)."""
+    import multiprocessing as mp
+    import shutil
+    import tempfile
+    base = "/dev/shm" if os.path.isdir("/dev/shm") else None
+    d = tempfile.mkdtemp(prefix="tlp_oracle_", dir=base)
+    try:
+        for nm, arr in (("rp", rp), ("ci", ci), ("X", Xh), ("el", elh), ("er", erh)):
+            np.save(os.path.join(d, nm + ".npy"), np.ascontiguousarray(arr))
+        chunks = [c for c in np.array_split(rows, cores) if len(c)]
+        ctx = mp.get_context("spawn")
+        with ctx.Pool(len(chunks)) as pool:
+            pool.map(_pool_worker, [(d, name, cfg["F"], chunks[0][:2])] * len(chunks))  # warm (imports)
+            t0 = time.perf_counter()
+            res = pool.map(_pool_worker, [(d, name, cfg["F"], c) for c in chunks])
+            wall = time.perf_counter() - t0
+        return sum(r[0] for r in res), wall
+    finally:
+        shutil.rmtree(d, ignore_errors=True)
+
+
 def cpu_baseline(name, cfg, rp, ci, Xh, elh, erh, seconds):
-    rows = _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds)
-    by, dt = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows)
-    return {"value": round(by / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"{len(rows)} of {cfg_n(cfg)} destination rows (uniform random, seed 0), "
-                      f"all ops of the step, {dt:.1f} s single-threaded fp64",
-            "host_cores_available": len(os.sched_getaffinity(0))}
+    """The fp64 oracle, untuned, on the host: single-threaded on a calibrated
+    row sample, then on all cores (one process per core, disjoint row chunks)
+    on a sample `cores` times larger."""
+    cores = len(os.sched_getaffinity(0))
+    rows = _calibrated_rows(name, cfg, rp, ci, Xh, elh, erh, seconds / 3)
+    by1, dt1 = _oracle_rows(name, cfg, rp, ci, Xh, elh, erh, rows)
+    out = {"kind": "oracle", "unit": "GB/s", "cpu_model": cpu_model(),
+           "host_cores_available": cores,
+           "single_thread": {"value": round(by1 / dt1 / 1e9, 4), "cores": 1,
+                             "sample": f"{len(rows)} of {cfg_n(cfg)} destination rows, {dt1:.1f} s"}}
+    try:
+        rng = np.random.default_rng(1)
+        k = int(min(cfg_n(cfg), len(rows) * cores * 0.5))
+        big = np.sort(rng.permutation(cfg_n(cfg))[:k])
+        byn, dtn = oracle_all_cores(name, cfg, rp, ci, Xh, elh, erh, big, cores)
+        out.update({"value": round(byn / dtn / 1e9, 4), "cores": cores,
+                    "sample": f"{len(big)} of {cfg_n(cfg)} destination rows (uniform random, seed 1), "
+                              f"all ops of the step, {dtn:.1f} s wall on {cores} processes "
+                              f"(~{dtn * cores:.0f} s of CPU), fp64 oracle"})
+    except Exception as e:  # noqa: BLE001 -- keep the single-thread figure
+        out.update({"value": out["single_thread"]["value"], "cores": 1,
+                    "sample": out["single_thread"]["sample"], "all_cores_error": repr(e)[:200]})
+    return out
 
 
 def run_reference(args):
@@ -699,13 +827,67 @@ def main():
                     help="with --dist/torchrun: NEXT-2 fused compute + all-gather over NVLink peer memory")
     ap.add_argument("--dist", action="store_true",
                     help="use the NCCL dist API even at world size 1 (exercises the N>1 path)")
+    ap.add_argument("--selftest", action="store_true",
+                    help="CPU check of the multi-rank launcher (gloo, no GPU): ranks partition "
+                         "the Reddit-shaped rows with libtlp's host partition and reduce a time")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: the contract wants >= 3 warm-up steps", file=sys.stderr)
-    if args.impl == "reference":
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is None and args.gpus > 1:
+        # --gpus N without a launcher: start N ranks ourselves (one process per
+        # GPU, torchrun over 127.0.0.1), forwarding the same arguments
+        sys.exit(launch_ranks(args.gpus, sys.argv[1:]))
+    if world_env is not None and int(world_env) != args.gpus:
+        print(f"error: --gpus {args.gpus} but WORLD_SIZE={world_env}", file=sys.stderr)
+        sys.exit(2)
+    if args.selftest:
+        run_selftest(args)
+    elif args.impl == "reference":
         run_reference(args)
     else:
         run_tlp(args)
+
+
+def launch_ranks(n, argv):
+    """Re-run this script under torch.distributed.run with n ranks on this node."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + list(argv)
+    return subprocess.call(cmd)
+
+
+def run_selftest(args):
+    """Launcher self-test on CPU (gloo): every rank computes the edge-balanced
+    row bounds with libtlp's host partition (tlp_partition_rows), checks them
+    against the oracle's rule, and the max-over-ranks reduction of a time runs
+    as in run_tlp; rank 0 prints one JSON line."""
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import oracle
+    import paper_conf_hpdc_fujh22_b200 as tlp
+    import synth
+    rp, _ = synth.chung_lu(3000, 60000, 0.4, 9, device="cpu")
+    b = tlp.tlp_partition_rows(rp, world)
+    ok = bool(np.array_equal(b, oracle.partition(rp, world)))
+    my_edges = int(rp[b[rank + 1]] - rp[b[rank]])
+    t = torch.tensor([float(my_edges)])
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    tot = torch.tensor([float(my_edges)])
+    dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+    okt = torch.tensor([1 if ok else 0])
+    dist.all_reduce(okt, op=dist.ReduceOp.MIN)
+    if rank == 0:
+        print(json.dumps({"selftest": "launcher", "n_gpus": world, "bounds_match_oracle": bool(okt.item()),
+                          "edges_total": int(tot.item()), "edges_max_rank": int(t.item()),
+                          "nnz": int(rp[-1])}))
+    dist.destroy_process_group()
 
 
 if __name__ == "__main__":

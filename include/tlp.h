@@ -348,6 +348,21 @@ tlp_status tlp_comm_create(const uint8_t id[128], int world, int rank,
                            tlp_comm *out);
 tlp_status tlp_comm_destroy(tlp_comm c);
 
+/* Failure detection (the paper is single-GPU, so this
+ * follows NCCL's own error model).  tlp_comm_async_error polls the
+ * communicator's asynchronous error state without blocking: *nccl_result =
+ * the ncclResult_t (0 = ncclSuccess, 7 = ncclInProgress); returns
+ * TLP_ERR_NCCL when it is an error.  tlp_comm_abort tears the communicator
+ * down without waiting for peers (ncclCommAbort); afterwards only
+ * tlp_comm_destroy may be called on it, and dist calls return TLP_ERR_NCCL.
+ * tlp_comm_wait blocks until `stream` has drained, polling the error state
+ * every ~0.2 ms; on an error, or after timeout_s seconds (<= 0: no limit), it
+ * aborts the communicator and returns TLP_ERR_NCCL -- a dead or hung peer
+ * cannot hang this rank forever. */
+tlp_status tlp_comm_async_error(tlp_comm c, int *nccl_result);
+tlp_status tlp_comm_abort(tlp_comm c);
+tlp_status tlp_comm_wait(tlp_comm c, void *stream, double timeout_s);
+
 /* Every rank passes the FULL square CSR (n x n, device or host).  The handle
  * holds this rank's row slice [b_k, b_{k+1}) (row_offset = b_k) with
  * out-degrees taken over the full CSR. */
@@ -392,9 +407,11 @@ tlp_status tlp_dist_gat_aggregate(tlp_graph local, tlp_comm c,
 /* NEXT-2 fused compute + all-gather: desc->Y must be a symmetric buffer
  * (tlp_comm_alloc_symmetric) holding Y_full [n x ldy].  ONE kernel computes this
  * rank's rows and stores each finished row vector into Y_full on every rank
- * over NVLink, overlapping the exchange with the gather; a one-element NCCL
- * all-reduce then orders `stream` after every rank's kernel.  Same result,
- * bit for bit, as tlp_dist_aggregate. */
+ * over NVLink, overlapping the exchange with the gather.  A one-element NCCL
+ * all-reduce on `stream` before the kernel (no rank stores into a peer's
+ * Y_full while that peer's earlier work may still read it) and one after it
+ * (every rank's stores have landed) order the call.  Same result, bit for
+ * bit, as tlp_dist_aggregate. */
 tlp_status tlp_dist_aggregate_fused(tlp_graph local, tlp_comm c,
                                     const tlp_agg_desc *desc, void *stream);
 

@@ -99,6 +99,9 @@ _sig = {
     "tlp_comm_get_unique_id": ([_P], _I),
     "tlp_comm_create": ([_P, _I, _I, ctypes.POINTER(_P)], _I),
     "tlp_comm_destroy": ([_P], _I),
+    "tlp_comm_async_error": ([_P, ctypes.POINTER(_I)], _I),
+    "tlp_comm_abort": ([_P], _I),
+    "tlp_comm_wait": ([_P, _P, ctypes.c_double], _I),
     "tlp_dist_graph_create": ([_P, _I64, _I64, _P, _P, _P, ctypes.POINTER(tlp_create_opts), _P,
                                ctypes.POINTER(_P)], _I),
     "tlp_dist_bounds": ([_P, _P], _I),
@@ -204,11 +207,34 @@ def _out(Y, n, F, like):
     return Y, F, ldy
 
 
-def _vec_cuda(v, name):
+def _vec_cuda(v, name, n=None):
+    """A float32 CUDA vector of at least n elements.  A non-contiguous input is
+    copied; the copy is registered with the launch stream by _keep_alive so the
+    caching allocator cannot recycle it while the kernel is queued."""
     torch = _torch()
     if not isinstance(v, torch.Tensor) or not v.is_cuda or v.dtype != torch.float32:
         raise TypeError(f"{name} must be a float32 CUDA tensor")
+    if n is not None and v.numel() < n:
+        raise ValueError(f"{name} has {v.numel()} elements, the call reads {n}")
     return v.contiguous()
+
+
+def _keep_alive(stream_handle, *tensors):
+    """Tie temporaries passed to a kernel to the stream the kernel was enqueued
+    on (no-op when that is torch's current stream: the allocator already
+    orders reuse on it)."""
+    torch = _torch()
+    for t in tensors:
+        if t is None or not isinstance(t, torch.Tensor) or not t.is_cuda:
+            continue
+        if stream_handle is None or stream_handle == torch.cuda.current_stream(t.device).cuda_stream:
+            continue
+        t.record_stream(torch.cuda.ExternalStream(stream_handle, device=t.device))
+
+
+def _need_rows(T, n, name):
+    if T.shape[0] < n:
+        raise ValueError(f"{name} has {T.shape[0]} rows, the graph needs {n}")
 
 
 # ------------------------------------------------------------------ graph ----
@@ -221,6 +247,8 @@ def tlp_graph_create(rowptr, colidx, n_src=None, edge_weight=None, opts=None, st
     ew = None if edge_weight is None else _as_index(edge_weight, np.float32)
     n_dst = int(rowptr.shape[0]) - 1
     nnz = int(colidx.shape[0])
+    if ew is not None and int(ew.shape[0]) != nnz:
+        raise ValueError(f"edge_weight has {int(ew.shape[0])} entries, colidx has {nnz}")
     if n_src is None:
         n_src = n_dst
     out = _P()
@@ -300,37 +328,55 @@ def tlp_graph_build_transpose(g, stream=None):
 
 # ------------------------------------------------------------ aggregations ---
 
+def _info(g, info=None):
+    return tlp_graph_info_get(g) if info is None else info
+
+
 def _n_dst(g):
     return tlp_graph_info_get(g)["n_dst"]
 
 
-def tlp_gcn_aggregate(g, X, norm="both", Y=None, F=None, stream=None, n_dst=None):
+def _fwd_args(g, X, Y, F, info):
+    """Shape checks of a forward aggregation (the C ABI gets raw pointers and
+    cannot check them): X has the graph's n_src rows, Y (if given) n_dst."""
+    info = _info(g, info)
     X, F, ldx = _feat(X, F)
-    n = _n_dst(g) if n_dst is None else n_dst
-    Y, F, ldy = _out(Y, n, F, X)
+    _need_rows(X, info["n_src"], "X")
+    if Y is not None:
+        Y0, _, _ = _feat(Y, F)
+        _need_rows(Y0, info["n_dst"], "Y")
+    Y, F, ldy = _out(Y, info["n_dst"], F, X)
+    return info, X, F, ldx, Y, ldy
+
+
+def _gat_vecs(info, el, er, heads=1):
+    el = _vec_cuda(el, "el", info["n_src"] * heads)
+    er = _vec_cuda(er, "er", (info["row_offset"] + info["n_dst"]) * heads)
+    return el, er
+
+
+def tlp_gcn_aggregate(g, X, norm="both", Y=None, F=None, stream=None, n_dst=None, info=None):
+    info, X, F, ldx, Y, ldy = _fwd_args(g, X, Y, F, info)
     nm = NORMS[norm] if isinstance(norm, str) else int(norm)
     _check(_lib.tlp_gcn_aggregate(g, _ptr(X), F, ldx, nm, _ptr(Y), ldy, _stream(stream, X.device)),
            "tlp_gcn_aggregate")
     return Y
 
 
-def tlp_gin_aggregate(g, X, eps=0.0, Y=None, F=None, stream=None, n_dst=None):
-    X, F, ldx = _feat(X, F)
-    n = _n_dst(g) if n_dst is None else n_dst
-    Y, F, ldy = _out(Y, n, F, X)
+def tlp_gin_aggregate(g, X, eps=0.0, Y=None, F=None, stream=None, n_dst=None, info=None):
+    info, X, F, ldx, Y, ldy = _fwd_args(g, X, Y, F, info)
     _check(_lib.tlp_gin_aggregate(g, _ptr(X), F, ldx, float(eps), _ptr(Y), ldy,
                                   _stream(stream, X.device)), "tlp_gin_aggregate")
     return Y
 
 
-def tlp_gat_aggregate(g, X, el, er, slope=0.2, Y=None, F=None, stream=None, n_dst=None):
-    X, F, ldx = _feat(X, F)
-    el = _vec_cuda(el, "el")
-    er = _vec_cuda(er, "er")
-    n = _n_dst(g) if n_dst is None else n_dst
-    Y, F, ldy = _out(Y, n, F, X)
+def tlp_gat_aggregate(g, X, el, er, slope=0.2, Y=None, F=None, stream=None, n_dst=None, info=None):
+    info, X, F, ldx, Y, ldy = _fwd_args(g, X, Y, F, info)
+    el, er = _gat_vecs(info, el, er)
+    sh = _stream(stream, X.device)
     _check(_lib.tlp_gat_aggregate(g, _ptr(X), F, ldx, _ptr(el), _ptr(er), float(slope), _ptr(Y),
-                                  ldy, _stream(stream, X.device)), "tlp_gat_aggregate")
+                                  ldy, sh), "tlp_gat_aggregate")
+    _keep_alive(sh, el, er)
     return Y
 
 
@@ -342,101 +388,117 @@ def _desc(op, X, Y, F, ldx, ldy, norm="both", eps=0.0, el=None, er=None, slope=0
     d.X, d.F, d.ldx, d.Y, d.ldy = _ptr(X), int(F), int(ldx), _ptr(Y), int(ldy)
     d.norm = NORMS[norm] if isinstance(norm, str) else int(norm)
     d.eps, d.slope, d.heads = float(eps), float(slope), int(heads)
-    d.el = _ptr(None if el is None else _vec_cuda(el, "el"))
-    d.er = _ptr(None if er is None else _vec_cuda(er, "er"))
+    d.el = _ptr(el)
+    d.er = _ptr(er)
     d.include_self = int(bool(include_self))
-    d.bias = _ptr(None if bias is None else _vec_cuda(bias, "bias"))
+    d.bias = _ptr(bias)
     d.act = ACTS[act] if isinstance(act, str) else int(act)
     d.act_param = float(act_param)
-    d.att_l = _ptr(None if att_l is None else _vec_cuda(att_l, "att_l"))
-    d.att_r = _ptr(None if att_r is None else _vec_cuda(att_r, "att_r"))
-    d.el_out = _ptr(None if el_out is None else _vec_cuda(el_out, "el_out"))
-    d.er_out = _ptr(None if er_out is None else _vec_cuda(er_out, "er_out"))
+    d.att_l = _ptr(att_l)
+    d.att_r = _ptr(att_r)
+    d.el_out = _ptr(el_out)
+    d.er_out = _ptr(er_out)
     return d
 
 
-def tlp_aggregate(g, op, X, Y=None, F=None, stream=None, n_dst=None, **kw):
+def _desc_vectors(info, op, F, kw, n_rows_global=None):
+    """Check and make contiguous the vector arguments of a descriptor call;
+    returns the (possibly copied) tensors to keep alive."""
+    heads = int(kw.get("heads", 1) or 1)
+    n_src = info["n_src"]
+    n_er = n_rows_global if n_rows_global is not None else info["row_offset"] + info["n_dst"]
+    sizes = {"el": n_src * heads, "er": n_er * heads, "bias": F, "att_l": F, "att_r": F}
+    keep = []
+    for k, n in sizes.items():
+        if kw.get(k) is not None:
+            kw[k] = _vec_cuda(kw[k], k, n)
+            keep.append(kw[k])
+    return keep
+
+
+def tlp_aggregate(g, op, X, Y=None, F=None, stream=None, n_dst=None, info=None, **kw):
     """Descriptor API: op in {gcn, gin, gat, sage, gat_mh}; keyword arguments of
     tlp_agg_desc (norm, eps, el, er, slope, heads, include_self) plus the fused
     layer epilogue bias=[F] tensor, act in {none, relu, leaky_relu, elu}, act_param,
     and the next layer's attention projections att_l / att_r ([F]) written to
     el_out / er_out ([n_dst] float32 CUDA tensors, contiguous)."""
-    X, F, ldx = _feat(X, F)
-    n = _n_dst(g) if n_dst is None else n_dst
-    Y, F, ldy = _out(Y, n, F, X)
+    info, X, F, ldx, Y, ldy = _fwd_args(g, X, Y, F, info)
+    n = info["n_dst"]
     for k in ("el_out", "er_out"):
         o = kw.get(k)
         if o is not None and (not o.is_contiguous() or o.numel() != n):
             raise ValueError(f"{k} must be a contiguous float32 CUDA tensor of n_dst elements")
-    keep = [kw.get(k) for k in ("el", "er", "bias", "att_l", "att_r")]  # keep copies alive
-    for k in ("el", "er", "bias", "att_l", "att_r"):
-        if kw.get(k) is not None:
-            kw[k] = _vec_cuda(kw[k], k)
+    keep = _desc_vectors(info, op, F, kw)
     d = _desc(op, X, Y, F, ldx, ldy, **kw)
-    _check(_lib.tlp_aggregate(g, ctypes.byref(d), _stream(stream, X.device)), "tlp_aggregate")
-    del keep
+    sh = _stream(stream, X.device)
+    _check(_lib.tlp_aggregate(g, ctypes.byref(d), sh), "tlp_aggregate")
+    _keep_alive(sh, *keep)
     return Y
 
 
-def tlp_sage_aggregate(g, X, include_self=False, Y=None, F=None, stream=None, n_dst=None):
+def tlp_sage_aggregate(g, X, include_self=False, Y=None, F=None, stream=None, n_dst=None, info=None):
     """GraphSage mean over N(v) (or N(v) + v with include_self)."""
-    X, F, ldx = _feat(X, F)
-    n = _n_dst(g) if n_dst is None else n_dst
-    Y, F, ldy = _out(Y, n, F, X)
+    info, X, F, ldx, Y, ldy = _fwd_args(g, X, Y, F, info)
     _check(_lib.tlp_sage_aggregate(g, _ptr(X), F, ldx, int(bool(include_self)), _ptr(Y), ldy,
                                    _stream(stream, X.device)), "tlp_sage_aggregate")
     return Y
 
 
-def tlp_gat_mh_aggregate(g, X, el, er, heads, slope=0.2, Y=None, F=None, stream=None, n_dst=None):
+def tlp_gat_mh_aggregate(g, X, el, er, heads, slope=0.2, Y=None, F=None, stream=None, n_dst=None,
+                         info=None):
     """Multi-head GAT; el: [n_src, heads], er: [n_dst (+row_offset), heads] CUDA fp32."""
-    X, F, ldx = _feat(X, F)
-    el = _vec_cuda(el, "el")
-    er = _vec_cuda(er, "er")
-    n = _n_dst(g) if n_dst is None else n_dst
-    Y, F, ldy = _out(Y, n, F, X)
+    info, X, F, ldx, Y, ldy = _fwd_args(g, X, Y, F, info)
+    el, er = _gat_vecs(info, el, er, int(heads))
+    sh = _stream(stream, X.device)
     _check(_lib.tlp_gat_mh_aggregate(g, _ptr(X), int(heads), F, ldx, _ptr(el), _ptr(er),
-                                     float(slope), _ptr(Y), ldy, _stream(stream, X.device)),
-           "tlp_gat_mh_aggregate")
+                                     float(slope), _ptr(Y), ldy, sh), "tlp_gat_mh_aggregate")
+    _keep_alive(sh, el, er)
     return Y
 
 
-def tlp_gcn_backward(g, dY, norm="both", dX=None, F=None, stream=None, n_src=None):
-    """dX = M^T dY for the GCN operator of the given norm (needs the transpose)."""
+def _bwd_args(g, dY, dX, F, info):
+    info = _info(g, info)
     dY, F, lddy = _feat(dY, F)
-    n = tlp_graph_info_get(g)["n_src"] if n_src is None else n_src
-    dX, F, lddx = _out(dX, n, F, dY)
+    _need_rows(dY, info["n_dst"], "dY")
+    if dX is not None:
+        _need_rows(_feat(dX, F)[0], info["n_src"], "dX")
+    dX, F, lddx = _out(dX, info["n_src"], F, dY)
+    return info, dY, F, lddy, dX, lddx
+
+
+def tlp_gcn_backward(g, dY, norm="both", dX=None, F=None, stream=None, n_src=None, info=None):
+    """dX = M^T dY for the GCN operator of the given norm (needs the transpose)."""
+    info, dY, F, lddy, dX, lddx = _bwd_args(g, dY, dX, F, info)
     nm = NORMS[norm] if isinstance(norm, str) else int(norm)
     _check(_lib.tlp_gcn_backward(g, _ptr(dY), F, lddy, nm, _ptr(dX), lddx, _stream(stream, dY.device)),
            "tlp_gcn_backward")
     return dX
 
 
-def tlp_gin_backward(g, dY, eps=0.0, dX=None, F=None, stream=None, n_src=None):
-    dY, F, lddy = _feat(dY, F)
-    n = tlp_graph_info_get(g)["n_src"] if n_src is None else n_src
-    dX, F, lddx = _out(dX, n, F, dY)
+def tlp_gin_backward(g, dY, eps=0.0, dX=None, F=None, stream=None, n_src=None, info=None):
+    info, dY, F, lddy, dX, lddx = _bwd_args(g, dY, dX, F, info)
     _check(_lib.tlp_gin_backward(g, _ptr(dY), F, lddy, float(eps), _ptr(dX), lddx,
                                  _stream(stream, dY.device)), "tlp_gin_backward")
     return dX
 
 
-def tlp_gat_backward(g, X, el, er, slope, Y, dY, dX=None, F=None, stream=None):
+def tlp_gat_backward(g, X, el, er, slope, Y, dY, dX=None, F=None, stream=None, info=None):
     """Single-head GAT backward: returns (dX [n_src, F], del [n_src], der [n_dst]).
     Y is the forward output of tlp_gat_aggregate for the same X, el, er."""
     torch = _torch()
-    X, F, ldx = _feat(X, F)
+    info, dY, F, lddy, dX, lddx = _bwd_args(g, dY, dX, F, info)
+    X, _, ldx = _feat(X, F)
+    _need_rows(X, info["n_src"], "X")
     Y, _, ldy = _feat(Y, F)
-    dY, _, lddy = _feat(dY, F)
-    el = _vec_cuda(el, "el")
-    er = _vec_cuda(er, "er")
-    info = tlp_graph_info_get(g)
-    dX, F, lddx = _out(dX, info["n_src"], F, dY)
+    _need_rows(Y, info["n_dst"], "Y")
+    el, er = _gat_vecs(info, el, er)
     dl = torch.empty(info["n_src"], dtype=torch.float32, device=dY.device)
     dr = torch.empty(info["n_dst"], dtype=torch.float32, device=dY.device)
+    sh = _stream(stream, dY.device)
     _check(_lib.tlp_gat_backward(g, _ptr(X), F, ldx, _ptr(el), _ptr(er), float(slope), _ptr(Y), ldy,
-                                 _ptr(dY), lddy, _ptr(dX), lddx, _ptr(dl), _ptr(dr),
-                                 _stream(stream, dY.device)), "tlp_gat_backward")
+                                 _ptr(dY), lddy, _ptr(dX), lddx, _ptr(dl), _ptr(dr), sh),
+           "tlp_gat_backward")
+    _keep_alive(sh, el, er)
     return dX, dl, dr
 
 
@@ -503,16 +565,27 @@ def tlp_dist_bounds(g, world):
     return b
 
 
+def _dist_args(g, X_full, Y_full, F):
+    """X_full [n x ldx] replicated, Y_full [n x ldy] (n = the global row count)."""
+    info = tlp_graph_info_get(g)
+    n = info["n_src"]
+    X, F, ldx = _feat(X_full, F)
+    _need_rows(X, n, "X_full")
+    Y, _, ldy = _feat(Y_full, F)
+    _need_rows(Y, n, "Y_full")
+    return info, n, X, F, ldx, Y, ldy
+
+
 def tlp_dist_allgather_rows(g, comm, Y_full, stream=None):
     Y, F, ldy = _feat(Y_full, None)
+    _need_rows(Y, tlp_graph_info_get(g)["n_src"], "Y_full")
     _check(_lib.tlp_dist_allgather_rows(g, comm, _ptr(Y), ldy, _stream(stream, Y.device)),
            "tlp_dist_allgather_rows")
     return Y_full
 
 
 def tlp_dist_gcn_aggregate(g, comm, X_full, Y_full, norm="both", F=None, stream=None):
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_full, F)
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_full, F)
     nm = NORMS[norm] if isinstance(norm, str) else int(norm)
     _check(_lib.tlp_dist_gcn_aggregate(g, comm, _ptr(X), F, ldx, nm, _ptr(Y), ldy,
                                        _stream(stream, X.device)), "tlp_dist_gcn_aggregate")
@@ -520,22 +593,38 @@ def tlp_dist_gcn_aggregate(g, comm, X_full, Y_full, norm="both", F=None, stream=
 
 
 def tlp_dist_gin_aggregate(g, comm, X_full, Y_full, eps=0.0, F=None, stream=None):
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_full, F)
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_full, F)
     _check(_lib.tlp_dist_gin_aggregate(g, comm, _ptr(X), F, ldx, float(eps), _ptr(Y), ldy,
                                        _stream(stream, X.device)), "tlp_dist_gin_aggregate")
     return Y_full
 
 
 def tlp_dist_gat_aggregate(g, comm, X_full, Y_full, el, er, slope=0.2, F=None, stream=None):
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_full, F)
-    el = _vec_cuda(el, "el")
-    er = _vec_cuda(er, "er")
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_full, F)
+    el = _vec_cuda(el, "el", n)
+    er = _vec_cuda(er, "er", n)
+    sh = _stream(stream, X.device)
     _check(_lib.tlp_dist_gat_aggregate(g, comm, _ptr(X), F, ldx, _ptr(el), _ptr(er), float(slope),
-                                       _ptr(Y), ldy, _stream(stream, X.device)),
-           "tlp_dist_gat_aggregate")
+                                       _ptr(Y), ldy, sh), "tlp_dist_gat_aggregate")
+    _keep_alive(sh, el, er)
     return Y_full
+
+
+def tlp_comm_async_error(comm):
+    """The communicator's asynchronous NCCL state (0 = ncclSuccess); raises on an error."""
+    r = _I()
+    _check(_lib.tlp_comm_async_error(comm, ctypes.byref(r)), "tlp_comm_async_error")
+    return r.value
+
+
+def tlp_comm_abort(comm):
+    _check(_lib.tlp_comm_abort(comm), "tlp_comm_abort")
+
+
+def tlp_comm_wait(comm, stream=None, timeout_s=0.0):
+    """Drain `stream` while polling NCCL's async error state; abort the
+    communicator on an error or after timeout_s seconds (TlpError)."""
+    _check(_lib.tlp_comm_wait(comm, _stream(stream), float(timeout_s)), "tlp_comm_wait")
 
 
 class _CudaArray:
@@ -564,46 +653,44 @@ def tlp_comm_free_symmetric(comm, ptr):
 def tlp_dist_aggregate_fused(g, comm, op, X_full, Y_sym, F=None, stream=None, **kw):
     """NEXT-2: one kernel computes this rank's rows and stores them into Y_full on
     every rank (Y_sym from tlp_comm_alloc_symmetric)."""
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_sym, F)
-    for k in ("el", "er", "bias"):
-        if kw.get(k) is not None:
-            kw[k] = _vec_cuda(kw[k], k)
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_sym, F)
+    keep = _desc_vectors(info, op, F, kw, n_rows_global=n)
     d = _desc(op, X, Y, F, ldx, ldy, **kw)
-    _check(_lib.tlp_dist_aggregate_fused(g, comm, ctypes.byref(d), _stream(stream, X.device)),
-           "tlp_dist_aggregate_fused")
+    sh = _stream(stream, X.device)
+    _check(_lib.tlp_dist_aggregate_fused(g, comm, ctypes.byref(d), sh), "tlp_dist_aggregate_fused")
+    _keep_alive(sh, *keep)
     return Y_sym
 
 
 def tlp_debug_multi_store(g, op, X, dests, F=None, stream=None, **kw):
     """Test hook: store the aggregation's output rows into every tensor of `dests`."""
+    info = tlp_graph_info_get(g)
     X, F, ldx = _feat(X, F)
+    _need_rows(X, info["n_src"], "X")
     D0, _, ldy = _feat(dests[0], F)
-    for k in ("el", "er", "bias"):
-        if kw.get(k) is not None:
-            kw[k] = _vec_cuda(kw[k], k)
+    for t in dests:
+        _need_rows(_feat(t, F)[0], info["row_offset"] + info["n_dst"], "dest")
+    keep = _desc_vectors(info, op, F, kw)
     d = _desc(op, X, D0, F, ldx, ldy, **kw)
     arr = (ctypes.c_void_p * len(dests))(*[t.data_ptr() for t in dests])
     _check(_lib.tlp_debug_multi_store(g, ctypes.byref(d), arr, len(dests), _stream(stream, X.device)),
            "tlp_debug_multi_store")
+    del keep  # the call is synchronous
     return dests
 
 
 def tlp_dist_aggregate(g, comm, op, X_full, Y_full, F=None, stream=None, **kw):
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_full, F)
-    for k in ("el", "er", "bias"):
-        if kw.get(k) is not None:
-            kw[k] = _vec_cuda(kw[k], k)
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_full, F)
+    keep = _desc_vectors(info, op, F, kw, n_rows_global=n)
     d = _desc(op, X, Y, F, ldx, ldy, **kw)
-    _check(_lib.tlp_dist_aggregate(g, comm, ctypes.byref(d), _stream(stream, X.device)),
-           "tlp_dist_aggregate")
+    sh = _stream(stream, X.device)
+    _check(_lib.tlp_dist_aggregate(g, comm, ctypes.byref(d), sh), "tlp_dist_aggregate")
+    _keep_alive(sh, *keep)
     return Y_full
 
 
 def tlp_dist_sage_aggregate(g, comm, X_full, Y_full, include_self=False, F=None, stream=None):
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_full, F)
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_full, F)
     _check(_lib.tlp_dist_sage_aggregate(g, comm, _ptr(X), F, ldx, int(bool(include_self)), _ptr(Y),
                                         ldy, _stream(stream, X.device)), "tlp_dist_sage_aggregate")
     return Y_full
@@ -611,13 +698,14 @@ def tlp_dist_sage_aggregate(g, comm, X_full, Y_full, include_self=False, F=None,
 
 def tlp_dist_gat_mh_aggregate(g, comm, X_full, Y_full, el, er, heads, slope=0.2, F=None,
                               stream=None):
-    X, F, ldx = _feat(X_full, F)
-    Y, _, ldy = _feat(Y_full, F)
-    el = _vec_cuda(el, "el")
-    er = _vec_cuda(er, "er")
+    info, n, X, F, ldx, Y, ldy = _dist_args(g, X_full, Y_full, F)
+    el = _vec_cuda(el, "el", n * int(heads))
+    er = _vec_cuda(er, "er", n * int(heads))
+    sh = _stream(stream, X.device)
     _check(_lib.tlp_dist_gat_mh_aggregate(g, comm, _ptr(X), int(heads), F, ldx, _ptr(el), _ptr(er),
-                                          float(slope), _ptr(Y), ldy, _stream(stream, X.device)),
+                                          float(slope), _ptr(Y), ldy, sh),
            "tlp_dist_gat_mh_aggregate")
+    _keep_alive(sh, el, er)
     return Y_full
 
 
@@ -643,35 +731,35 @@ class Graph:
         return self.info["n_dst"]
 
     def gcn(self, X, norm="both", Y=None, F=None, stream=None):
-        return tlp_gcn_aggregate(self.handle, X, norm, Y, F, stream, n_dst=self.n_dst)
+        return tlp_gcn_aggregate(self.handle, X, norm, Y, F, stream, info=self.info)
 
     def gin(self, X, eps=0.0, Y=None, F=None, stream=None):
-        return tlp_gin_aggregate(self.handle, X, eps, Y, F, stream, n_dst=self.n_dst)
+        return tlp_gin_aggregate(self.handle, X, eps, Y, F, stream, info=self.info)
 
     def gat(self, X, el, er, slope=0.2, Y=None, F=None, stream=None):
-        return tlp_gat_aggregate(self.handle, X, el, er, slope, Y, F, stream, n_dst=self.n_dst)
+        return tlp_gat_aggregate(self.handle, X, el, er, slope, Y, F, stream, info=self.info)
 
     def sage(self, X, include_self=False, Y=None, F=None, stream=None):
-        return tlp_sage_aggregate(self.handle, X, include_self, Y, F, stream, n_dst=self.n_dst)
+        return tlp_sage_aggregate(self.handle, X, include_self, Y, F, stream, info=self.info)
 
     def gat_mh(self, X, el, er, heads, slope=0.2, Y=None, F=None, stream=None):
         return tlp_gat_mh_aggregate(self.handle, X, el, er, heads, slope, Y, F, stream,
-                                    n_dst=self.n_dst)
+                                    info=self.info)
 
     def aggregate(self, op, X, Y=None, F=None, stream=None, **kw):
-        return tlp_aggregate(self.handle, op, X, Y, F, stream, n_dst=self.n_dst, **kw)
+        return tlp_aggregate(self.handle, op, X, Y, F, stream, info=self.info, **kw)
 
     def build_transpose(self, stream=None):
         tlp_graph_build_transpose(self.handle, stream)
 
     def gcn_backward(self, dY, norm="both", dX=None, F=None, stream=None):
-        return tlp_gcn_backward(self.handle, dY, norm, dX, F, stream, n_src=self.info["n_src"])
+        return tlp_gcn_backward(self.handle, dY, norm, dX, F, stream, info=self.info)
 
     def gin_backward(self, dY, eps=0.0, dX=None, F=None, stream=None):
-        return tlp_gin_backward(self.handle, dY, eps, dX, F, stream, n_src=self.info["n_src"])
+        return tlp_gin_backward(self.handle, dY, eps, dX, F, stream, info=self.info)
 
     def gat_backward(self, X, el, er, slope, Y, dY, dX=None, F=None, stream=None):
-        return tlp_gat_backward(self.handle, X, el, er, slope, Y, dY, dX, F, stream)
+        return tlp_gat_backward(self.handle, X, el, er, slope, Y, dY, dX, F, stream, info=self.info)
 
     def degrees(self):
         return tlp_graph_degrees(self.handle)

@@ -100,6 +100,26 @@ def build(force=False, verbose=False, ptxas_verbose=False, defines=(), out=None)
     return lib
 
 
+PROBE_SRC = os.path.join(ROOT, "bench_probe", "l2_ceiling.cu")
+PROBE_LIB = os.path.join(ROOT, "bench_probe", "libl2c.so")
+
+
+def build_probe(force=False):
+    """bench.py's L2 gather-ceiling probe (a measurement tool, not the product)."""
+    if not os.path.exists(PROBE_SRC):
+        return None
+    if not force and os.path.exists(PROBE_LIB) and os.path.getmtime(PROBE_LIB) >= os.path.getmtime(PROBE_SRC):
+        return PROBE_LIB
+    tmp = PROBE_LIB + ".tmp%d" % os.getpid()
+    cmd = [nvcc()] + ARCH + ["-O3", "-lineinfo", "-shared", "-Xcompiler", "-fPIC", "-o", tmp, PROBE_SRC,
+                             "-cudart", "static"]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"nvcc failed for {PROBE_SRC}:\n{r.stdout}\n{r.stderr}")
+    os.replace(tmp, PROBE_LIB)
+    return PROBE_LIB
+
+
 if __name__ == "__main__":
     defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
     outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]

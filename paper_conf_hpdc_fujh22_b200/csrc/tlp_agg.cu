@@ -699,23 +699,24 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (!panel && !panel_off && n_strips > 1 && g->n_tasks < (int64_t)g->num_sms * 32 * 4) panel = 1;
     if (n_strips < 2) panel = 0;
 
-    // Gather layout.  In panel mode every edge
-    // gathers one strip of a source row from L2; a strip that is not 128-byte
-    // aligned touches one more cache line and one more sector per gather and
-    // inflates the L2 footprint of the panel (measured on Reddit, F = 602:
-    // ld 604 -> 608 cut DRAM reads 50 -> 22 GB per launch, GIN 21.5 -> 17.8
-    // ms).  So when the caller's rows are not 128-byte aligned, the gathers read
-    // a copy of X written by one streaming pass (read + write of n_src x F,
-    // ~1 % of a Reddit launch): padded rows (ld rounded up to 32 floats) or
-    // panel-major blocks of strip_w columns.  The unweighted GCN-BOTH
-    // pre-scale writes its X' in the same layout at no extra cost.  Values are
-    // copied bit for bit (or scaled exactly as before), so no output bit changes.
-    // TLP_LAYOUT=caller|padded|panel overrides.
+    // Gather layout.  In L2-panel mode (X larger
+    // than L2, its strips not) every edge gathers one strip of a source row
+    // from L2.  A strip that is not 128-byte aligned touches one more cache
+    // line and one more sector per gather and inflates the L2 footprint of the
+    // panel; a strip spread over all of X (row stride ld) touches every page of
+    // X per sweep.  So the gathers read a panel-major copy of X -- strip s is a
+    // contiguous [n_src x strip_w] block, 256-byte rows -- written by one
+    // streaming pass (read + write of n_src x F, ~1 % of a Reddit launch); the
+    // unweighted GCN-BOTH pre-scale writes its X' in that layout at no extra
+    // cost.  Measured on Reddit (F = 602): GIN 21.4 ms (caller ld 604) / 17.9
+    // (caller ld 608) / 18.4 (padded copy) / 16.7 (panel-major copy), GCN-BOTH
+    // 22.3 / 18.8 / 18.8 / 17.2, GAT 24.4 / 20.9 / 21.1 / 19.9.  Values are
+    // copied bit for bit (or scaled exactly as before), so no output bit
+    // changes.  TLP_LAYOUT=caller|padded|panel overrides (and applies to any
+    // panel-mode call, so tests can force it on small inputs).
     int layout = 0;  // 0 caller, 1 padded rows, 2 panel-major
-    if (panel && vec == 4 && op != OP_GATH &&
-        4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes) {
-        const bool misaligned = (r.ldx % 32) != 0 || !aligned(r.X, 128);
-        layout = misaligned ? 1 : 0;
+    if (panel && vec == 4 && op != OP_GATH) {
+        if (4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes) layout = 2;
         if (const char *e = getenv("TLP_LAYOUT")) {
             if (!strcmp(e, "caller")) layout = 0;
             else if (!strcmp(e, "padded")) layout = 1;
@@ -784,7 +785,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.tasks = g->tasks;
     a.hub_row = g->hub_row;
     a.hub_off = g->hub_off;
-    a.ctr = reinterpret_cast<unsigned long long *>(g->ctr);
+    a.ctr = g->ctr;
     a.done = g->ctr + 2;
     a.ldx = ldg;
     a.ldy = r.ldy;
@@ -946,6 +947,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     }
     if (blocks < 1) blocks = 1;
     if (blocks > 0x7fffffff) return set_error(TLP_ERR_UNSUPPORTED, "grid too large");
+    // the kernel walks work items with 32-bit indices
+    if (a.n_items + (blocks * wpc + 1) * (int64_t)std::max(step, 1) >= (int64_t(1) << 31))
+        return set_error(TLP_ERR_UNSUPPORTED, "too many work items (tasks x strips >= 2^31)");
     fn<<<(unsigned)blocks, threads, smem, s>>>(a);
     g->launches += 1;
     cudaError_t e = cudaGetLastError();

@@ -89,7 +89,7 @@ struct AggArgs {
     int32_t *hub_ticket;
     float *scratch;  // hub partial vectors [n_chunks x ldp]
     float *md;       // GAT hub (m, den) pairs [n_chunks x 2]
-    unsigned long long *ctr;
+    unsigned int *ctr;   // next work item (32-bit: n_items + W * step < 2^31)
     unsigned int *done;
     int64_t ldx, ldy, ldp, row_offset, n_tasks, n_items, n_hubs, n_chunks, C;
     int F, n_strips, norm, step, sched, panel;
@@ -1131,7 +1131,8 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
             const int64_t e0 = __shfl_sync(FULL, rp, k);
             const int64_t e1 = __shfl_sync(FULL, rp, k + 1);
             const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
-            const int64_t r = rb + k;
+            const int r = rb + k;
+            const int deg = (int)(e1 - e0);
             for (int s = s0; s < s1; ++s) {
                 const int col = strip_col<VEC, G>(a, s, lane);
                 const bool active = in_strip<G>(a, lane, col);
@@ -1166,7 +1167,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                     reduce_edges<VEC, OP, COEF, U, G>(a, e0, e1, s, col, active, er_v, lane, acc, m, den,
                                                          xu, gout);
                 }
-                Vec<VEC> y = epilogue<VEC, OP>(a, r, e1 - e0, col, active, acc, den);
+                Vec<VEC> y = epilogue<VEC, OP>(a, r, deg, col, active, acc, den);
                 if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
                 project_row<VEC, G>(a, r, s, col, active, y, lane);
             }
@@ -1177,8 +1178,11 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
 // One C-edge chunk of hub h (a8), feature strips [s0, s1).  The last chunk of
 // the hub to finish these strips merges all its partials in chunk order and
 // writes the row.  Tickets (and GAT (m, den) pairs) are kept per panel s0.
+#ifndef TLP_HUB_INLINE
+#define TLP_HUB_INLINE __forceinline__
+#endif
 template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int s0, int s1,
+__device__ TLP_HUB_INLINE void do_hub_chunk(const AggArgs &a, int h, int j, int s0, int s1,
                                              int lane) {
     const int r = __ldg(a.hub_row + h);
     const int off = __ldg(a.hub_off + h);
@@ -1308,12 +1312,14 @@ __device__ __forceinline__ void do_hub_chunk(const AggArgs &a, int h, int j, int
 // s = i / n_tasks of task i % n_tasks, so that all warps sweep one L2-resident
 // feature panel of X at a time.
 template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
-__device__ __forceinline__ void do_item(const AggArgs &a, int64_t i, int lane) {
-    int64_t t = i;
+__device__ __forceinline__ void do_item(const AggArgs &a, int i, int lane) {
+    // 32-bit item arithmetic (the host guarantees n_items + W * step < 2^31):
+    // these values stay live across the whole task, so every register counts
+    int t = i;
     int s0 = 0, s1 = a.n_strips;
     if (a.panel) {
-        s0 = (int)(i / a.n_tasks);
-        t = i - (int64_t)s0 * a.n_tasks;
+        s0 = i / (int)a.n_tasks;
+        t = i - s0 * (int)a.n_tasks;
         s1 = s0 + 1;
     }
     const int2 tk = a.tasks[t];
@@ -1338,29 +1344,31 @@ constexpr int min_blocks(int op, int coef, bool async, int G = 1) {
 template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void agg_body(const AggArgs &a) {
     const int lane = threadIdx.x & 31;
-    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int wid = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    const int n_items = (int)a.n_items;
     if (a.sched == S_HARDWARE) {  // one warp per item
-        if (wid < a.n_items) do_item<VEC, OP, COEF, U, ASYNC, G>(a, wid, lane);
+        if (wid < n_items) do_item<VEC, OP, COEF, U, ASYNC, G>(a, wid, lane);
         if (a.n_dests > 0) __threadfence_system();
         return;
     }
-    const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t stride = W * a.step;
-    int64_t t = wid * a.step;  // static first wave
-    while (t < a.n_items) {
-        unsigned long long v = 0;
-        if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned long long)a.step);
-        const int64_t tend = min(t + a.step, a.n_items);
-        for (int64_t tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, G>(a, tt, lane);
-        if (a.sched == S_DYNAMIC) t = stride + (int64_t)__shfl_sync(FULL, v, 0);
-        else t += stride;
+    const int W = (int)((gridDim.x * blockDim.x) >> 5);
+    int t = wid * a.step;  // static first wave
+    while (t < n_items) {
+        // the next batch is claimed before this one is processed (its latency
+        // hides behind the work); 32-bit counter
+        unsigned v = 0;
+        if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned)a.step);
+        const int tend = min(t + a.step, n_items);
+        for (int tt = t; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, G>(a, tt, lane);
+        if (a.sched == S_DYNAMIC) t = W * a.step + (int)__shfl_sync(FULL, v, 0);
+        else t += W * a.step;
     }
     if (a.n_dests > 0) __threadfence_system();  // peer stores visible before the barrier
     if (a.sched == S_DYNAMIC && lane == 0) {
         // last warp out resets the counter: no memset launch between calls
         __threadfence();
         if (atomicAdd(a.done, 1u) == (unsigned)(W - 1)) {
-            *a.ctr = 0ull;
+            *a.ctr = 0u;
             *a.done = 0u;
             __threadfence();
         }

@@ -10,8 +10,10 @@
 // broadcast in place by a grouped ncclBroadcast(root = r).
 #include <nccl.h>
 
+#include <chrono>
 #include <cstring>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "tlp_internal.h"
@@ -31,6 +33,7 @@ struct tlp_comm_s {
     int world = 1, rank = 0;
     std::vector<SymBuf> sym;
     int *barrier = nullptr;     // one device int for the stream barrier
+    cudaStream_t side = nullptr;  // private stream for the communicator's own blocking steps
 };
 
 namespace tlp {
@@ -101,15 +104,74 @@ tlp_status tlp_comm_create(const uint8_t id[128], int world, int rank, tlp_comm 
     }
     c->world = world;
     c->rank = rank;
+    cudaError_t ce = cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking);
+    if (ce != cudaSuccess) {
+        ncclCommDestroy(c->comm);
+        delete c;
+        return cuda_error(ce, "cudaStreamCreate(comm side stream)");
+    }
     *out = c;
     return TLP_OK;
+}
+
+// NCCL failure detection: the asynchronous error state of the
+// communicator (a peer that died, a network / NVLink fault), polled without
+// blocking.
+tlp_status tlp_comm_async_error(tlp_comm c, int *nccl_result) {
+    if (!c || !nccl_result) return set_error(TLP_ERR_INVALID_ARGUMENT, "comm_async_error: bad argument");
+    ncclResult_t a = ncclSuccess;
+    TLP_NCCL_TRY(ncclCommGetAsyncError(c->comm, &a));
+    *nccl_result = (int)a;
+    if (a != ncclSuccess && a != ncclInProgress) return nccl_error(a, "communicator async error");
+    return TLP_OK;
+}
+
+// Abort: tear the communicator down without waiting for peers (after a fault
+// or a timeout); the handle stays valid only for tlp_comm_destroy.
+tlp_status tlp_comm_abort(tlp_comm c) {
+    if (!c) return set_error(TLP_ERR_INVALID_ARGUMENT, "comm_abort: null");
+    if (!c->comm) return TLP_OK;
+    ncclResult_t r = ncclCommAbort(c->comm);
+    c->comm = nullptr;
+    if (r != ncclSuccess) return nccl_error(r, "ncclCommAbort");
+    return TLP_OK;
+}
+
+// Wait for `stream` (whose tail holds this communicator's collectives) while
+// polling the communicator's asynchronous error state; on an error or after
+// timeout_s seconds (<= 0: no limit) the communicator is aborted, so a hung
+// peer cannot hang this rank forever.
+tlp_status tlp_comm_wait(tlp_comm c, void *stream, double timeout_s) {
+    if (!c) return set_error(TLP_ERR_INVALID_ARGUMENT, "comm_wait: null");
+    cudaStream_t s = (cudaStream_t)stream;
+    const auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+        cudaError_t q = cudaStreamQuery(s);
+        if (q == cudaSuccess) return TLP_OK;
+        if (q != cudaErrorNotReady) return cuda_error(q, "cudaStreamQuery");
+        if (c->comm) {
+            ncclResult_t a = ncclSuccess;
+            ncclCommGetAsyncError(c->comm, &a);
+            if (a != ncclSuccess && a != ncclInProgress) {
+                tlp_comm_abort(c);
+                return nccl_error(a, "communicator async error (aborted)");
+            }
+        }
+        const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+        if (timeout_s > 0 && el > timeout_s) {
+            tlp_comm_abort(c);
+            return set_error(TLP_ERR_NCCL, "tlp_comm_wait: timeout, communicator aborted");
+        }
+        std::this_thread::sleep_for(std::chrono::microseconds(200));
+    }
 }
 
 tlp_status tlp_comm_destroy(tlp_comm c) {
     if (!c) return TLP_OK;
     while (!c->sym.empty()) tlp_comm_free_symmetric(c, c->sym.back().local);
     if (c->barrier) cudaFree(c->barrier);
-    ncclResult_t r = ncclCommDestroy(c->comm);
+    if (c->side) cudaStreamDestroy(c->side);
+    ncclResult_t r = c->comm ? ncclCommDestroy(c->comm) : ncclSuccess;
     delete c;
     if (r != ncclSuccess) return nccl_error(r, "ncclCommDestroy");
     return TLP_OK;
@@ -166,6 +228,7 @@ tlp_status tlp_graph_create_rows(int64_t n, int64_t nnz, const int64_t *rowptr,
 
 static tlp_status comm_barrier(tlp_comm c, cudaStream_t s) {
     if (c->world == 1) return TLP_OK;
+    if (!c->comm) return set_error(TLP_ERR_NCCL, "communicator was aborted");
     if (!c->barrier) {
         TLP_CUDA_TRY(cudaMalloc(&c->barrier, sizeof(int)));
         TLP_CUDA_TRY(cudaMemset(c->barrier, 0, sizeof(int)));
@@ -189,12 +252,14 @@ tlp_status tlp_comm_alloc_symmetric(tlp_comm c, size_t bytes, void **local) {
         if (e != cudaSuccess) { cudaFree(b.local); return cuda_error(e, "cudaIpcGetMemHandle"); }
         std::vector<cudaIpcMemHandle_t> all(c->world);
         void *dh = nullptr;
+        // on the communicator's private stream (never the legacy default
+        // stream, which would serialise against every other stream)
         TLP_CUDA_TRY(cudaMalloc(&dh, sizeof(cudaIpcMemHandle_t) * c->world));
-        TLP_CUDA_TRY(cudaMemcpy((char *)dh + sizeof(h) * c->rank, &h, sizeof(h), cudaMemcpyHostToDevice));
-        ncclResult_t r = ncclAllGather((char *)dh + sizeof(h) * c->rank, dh, sizeof(h), ncclUint8, c->comm, 0);
+        TLP_CUDA_TRY(cudaMemcpyAsync((char *)dh + sizeof(h) * c->rank, &h, sizeof(h), cudaMemcpyHostToDevice, c->side));
+        ncclResult_t r = ncclAllGather((char *)dh + sizeof(h) * c->rank, dh, sizeof(h), ncclUint8, c->comm, c->side);
         if (r != ncclSuccess) { cudaFree(dh); cudaFree(b.local); return nccl_error(r, "ncclAllGather(ipc handles)"); }
-        TLP_CUDA_TRY(cudaStreamSynchronize(0));
-        TLP_CUDA_TRY(cudaMemcpy(all.data(), dh, sizeof(h) * c->world, cudaMemcpyDeviceToHost));
+        TLP_CUDA_TRY(cudaMemcpyAsync(all.data(), dh, sizeof(h) * c->world, cudaMemcpyDeviceToHost, c->side));
+        TLP_CUDA_TRY(cudaStreamSynchronize(c->side));
         cudaFree(dh);
         for (int q = 0; q < c->world; ++q) {
             if (q == c->rank) continue;
@@ -222,8 +287,9 @@ tlp_status tlp_comm_free_symmetric(tlp_comm c, void *local) {
         for (int q = 0; q < c->world; ++q)
             if (q != c->rank && b.peers[q]) cudaIpcCloseMemHandle(b.peers[q]);
         // every rank has unmapped before anyone frees
-        tlp_status st = comm_barrier(c, 0);
-        cudaStreamSynchronize(0);
+        cudaDeviceSynchronize();  // no queued kernel still stores through the mappings
+        tlp_status st = comm_barrier(c, c->side);
+        cudaStreamSynchronize(c->side);
         cudaFree(b.dev_ptrs);
         cudaFree(b.local);
         c->sym.erase(c->sym.begin() + i);
@@ -276,6 +342,7 @@ tlp_status tlp_dist_allgather_rows(tlp_graph g, tlp_comm c, float *Y_full, int64
         return set_error(TLP_ERR_INVALID_ARGUMENT, "communicator does not match the graph");
     cudaStream_t s = (cudaStream_t)stream;
     if (c->world == 1) return TLP_OK;
+    if (!c->comm) return set_error(TLP_ERR_NCCL, "communicator was aborted");
     TLP_NCCL_TRY(ncclGroupStart());
     for (int r = 0; r < c->world; ++r) {
         const int64_t rows = g->bounds_host[r + 1] - g->bounds_host[r];
@@ -352,8 +419,15 @@ tlp_status tlp_dist_aggregate_fused(tlp_graph g, tlp_comm c, const tlp_agg_desc 
     r.Y = d->Y + g->row_offset * d->ldy;
     r.dests = b->dev_ptrs;
     r.n_dests = c->world;
-    tlp_status st = aggregate(g, r, (cudaStream_t)stream);
+    // entry barrier: a fast rank must not store into a peer's Y_full while that
+    // peer's stream may still read its previous contents (e.g. the next layer
+    // reads Y_full while this call overwrites it on every rank)
+    tlp_status st = comm_barrier(c, (cudaStream_t)stream);
     if (st != TLP_OK) return st;
+    st = aggregate(g, r, (cudaStream_t)stream);
+    if (st != TLP_OK) return st;
+    // exit barrier: every rank's stores have landed (the kernel ends with
+    // __threadfence_system) before any rank's stream proceeds
     return comm_barrier(c, (cudaStream_t)stream);
 }
 

@@ -332,8 +332,12 @@ tlp_status graph_create_impl(int64_t n_dst, int64_t n_src, int64_t nnz,
         k_rowptr_ingest<<<grid_for(n_dst + 1, nsm), 256, 0, s>>>(rp_dev, n_dst, nnz, g->rowptr,
                                                                   g->in_deg, err.as<int>());
         CTRY(cudaGetLastError());
-        if (nnz) {
-            k_colidx_check<<<grid_for(nnz, nsm), 256, 0, s>>>(g->colidx, nnz, n_src, err.as<int>());
+        // a row slice validates the whole CSR it was cut from: its out-degree
+        // histogram (a2) indexes out_deg with every source of full_colidx
+        const int32_t *chk = full_colidx ? full_colidx : g->colidx;
+        const int64_t chk_n = full_colidx ? full_nnz : nnz;
+        if (chk_n) {
+            k_colidx_check<<<grid_for(chk_n, nsm), 256, 0, s>>>(chk, chk_n, n_src, err.as<int>());
             CTRY(cudaGetLastError());
         }
         int herr = 0;

@@ -446,6 +446,46 @@ def test_panel_modes_bitwise(tlp, monkeypatch):
     g.close()
 
 
+@pytest.mark.parametrize("panel", ["64", "128", "32"])
+@pytest.mark.parametrize("F,ld", [(300, 300), (602, 604), (37, 40)])
+def test_gather_layouts_bitwise(tlp, monkeypatch, panel, F, ld):
+    """The gather copy of X (caller rows, padded
+    128-byte rows, panel-major strip blocks) never changes an output bit, for
+    every op that gathers through it (GCN all norms incl. the pre-scaled BOTH,
+    weighted GCN, GIN, SAGE, GAT in both softmax modes, GAT backward)."""
+    n = 2600
+    rp, ci = synth.chung_lu(n, 70000, 0.5, 23, device="cpu")
+    Xh = synth.features(n, F, ld, seed=7)
+    X = _t(Xh)
+    elh, erh = synth.normal(n, 1), synth.normal(n, 2)
+    el, er = _t(elh), _t(erh)
+    ew = _t(synth.edge_weights(len(ci), 4))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=90, hub_chunk=44))
+    gw = tlp.Graph(_t(rp), _t(ci), edge_weight=ew, opts=dict(hub_threshold=90, hub_chunk=44))
+    monkeypatch.setenv("TLP_PANEL", panel)
+    outs = {}
+    for lay in ("caller", "padded", "panel"):
+        monkeypatch.setenv("TLP_LAYOUT", lay)
+        res = [g.gcn(X, "both", F=F), g.gcn(X, "right", F=F), gw.gcn(X, "both", F=F),
+               g.gin(X, 0.1, F=F), g.sage(X, True, F=F)]
+        for mode in ("alpha", "online"):
+            monkeypatch.setenv("TLP_GAT", mode)
+            res.append(g.gat(X, el, er, 0.2, F=F))
+        monkeypatch.delenv("TLP_GAT")
+        g.build_transpose()
+        dX, dl, dr = g.gat_backward(X, el, er, 0.2, res[-1], X, F=F)
+        res += [dX, dl, dr]
+        torch.cuda.synchronize()
+        outs[lay] = [r.clone() for r in res]
+    for lay in ("padded", "panel"):
+        for i, (a, b) in enumerate(zip(outs[lay], outs["caller"])):
+            assert torch.equal(a, b), (lay, i)
+    _check("layout gcn", outs["panel"][0], oracle.gcn(rp, ci, Xh, "both", F=F))
+    _check("layout gin", outs["panel"][3], oracle.gin(rp, ci, Xh, 0.1, F=F))
+    _check("layout gat", outs["panel"][5], oracle.gat(rp, ci, Xh, elh, erh, 0.2, F=F))
+    g.close(); gw.close()
+
+
 @pytest.mark.parametrize("F,ld", [(100, 100), (300, 300), (37, 40), (5, 6)])
 def test_gather_paths_bitwise(tlp, monkeypatch, F, ld):
     """Register double-buffered and cp.async shared-memory gathers agree bit for bit."""
