@@ -52,11 +52,36 @@ def test_reference_arm_runs_on_host():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["e2e"]["h2d_bytes_per_step"] == 0
 
 
-def test_l2_gather_peak_parses_committed_probe():
-    """bench.py's L2 roofline reads the committed probe: the 256-byte-row,
-    L2-resident (< 80 MB table) entry with the highest bandwidth."""
-    import bench
-    p = bench.l2_gather_peak()
-    assert p is not None
-    assert p["row_bytes"] == 256 and p["table_MB"] < 80
-    assert 5000 < p["GBs"] < 40000
+def test_l2_ceiling_probe_builds_and_exports():
+    """The in-run L2 gather-ceiling probe (bench_probe/l2_ceiling.cu) is built
+    by build() and exports its C entry point (it runs only on a GPU)."""
+    import ctypes
+    p = os.path.join(ROOT, "bench_probe", "libl2c.so")
+    if not os.path.exists(p):
+        sys.path.insert(0, os.path.join(ROOT, "paper_conf_hpdc_fujh22_b200"))
+        import _build
+        _build.build_probe()
+    lib = ctypes.CDLL(p)
+    assert hasattr(lib, "l2c_run")
+
+
+def test_launcher_two_ranks_gloo():
+    """`bench.py --gpus 2` without a launcher starts two ranks itself
+    (torch.distributed.run over 127.0.0.1); the self-test rank body runs on CPU
+    with gloo: libtlp's host partition equals the oracle's rule on every rank,
+    max/sum reductions over ranks, rank 0 prints one JSON line."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--selftest"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.strip().splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["bounds_match_oracle"] and d["edges_total"] == d["nnz"]
+    assert d["edges_max_rank"] <= d["nnz"] // 2 + 200
+
+
+def test_gpus_mismatch_with_world_size_is_an_error():
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--selftest"],
+                       capture_output=True, text=True, timeout=120, cwd=ROOT, env=env)
+    assert r.returncode == 2 and "WORLD_SIZE" in r.stderr
