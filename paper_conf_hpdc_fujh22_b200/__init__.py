@@ -172,11 +172,16 @@ def _as_index(a, dtype):
 
 
 def _stream(stream, device=None):
+    """cudaStream_t of `stream`, or torch's current stream on `device` (the raw
+    handle straight from torch's C layer: this runs once per call, so it
+    avoids building a Stream object)."""
     if stream is not None:
         return getattr(stream, "cuda_stream", stream)
     torch = _torch()
     if torch.cuda.is_available():
-        return torch.cuda.current_stream(device).cuda_stream
+        idx = device.index if device is not None and device.index is not None else torch.cuda.current_device()
+        raw = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+        return raw(idx) if raw is not None else torch.cuda.current_stream(idx).cuda_stream
     return None
 
 
@@ -342,10 +347,8 @@ def _fwd_args(g, X, Y, F, info):
     info = _info(g, info)
     X, F, ldx = _feat(X, F)
     _need_rows(X, info["n_src"], "X")
-    if Y is not None:
-        Y0, _, _ = _feat(Y, F)
-        _need_rows(Y0, info["n_dst"], "Y")
     Y, F, ldy = _out(Y, info["n_dst"], F, X)
+    _need_rows(Y, info["n_dst"], "Y")
     return info, X, F, ldx, Y, ldy
 
 

@@ -6,10 +6,31 @@
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
+#include <unistd.h>
 
 #include "tlp_agg_kernels.cuh"
 
 namespace tlp {
+
+// Tuning / measurement knobs (TLP_* environment variables) are read
+// from a snapshot taken once per aggregate() call: one pass over the
+// environment instead of a getenv scan per knob (host cost of a small call).
+struct KnobSnapshot {
+    int n = 0;
+    const char *kv[32];
+};
+static thread_local KnobSnapshot g_knobs;
+static void snapshot_knobs() {
+    g_knobs.n = 0;
+    for (char **e = environ; e && *e && g_knobs.n < 32; ++e)
+        if ((*e)[0] == 'T' && (*e)[1] == 'L' && (*e)[2] == 'P' && (*e)[3] == '_') g_knobs.kv[g_knobs.n++] = *e;
+}
+static const char *knob(const char *name) {
+    const size_t L = strlen(name);
+    for (int i = 0; i < g_knobs.n; ++i)
+        if (!strncmp(g_knobs.kv[i], name, L) && g_knobs.kv[i][L] == '=') return g_knobs.kv[i] + L + 1;
+    return nullptr;
+}
 
 // ------------------------------------------------------------- dispatch --
 
@@ -437,7 +458,7 @@ constexpr double kHotFrac = 0.5;
 static tlp_status hot_threshold(tlp_graph g, int64_t ldx, bool panel, cudaStream_t s,
                                 unsigned *thr) {
     *thr = 0;
-    const char *e = getenv("TLP_HOT");
+    const char *e = knob("TLP_HOT");
     // by default not in panel mode: there the whole strip of X is meant to stay in L2
     if (!e && panel) return TLP_OK;
     const double frac = e ? atof(e) : kHotFrac;
@@ -483,6 +504,7 @@ static tlp_status hot_threshold(tlp_graph g, int64_t ldx, bool panel, cudaStream
 
 tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    snapshot_knobs();
     if (r.F < 0) return set_error(TLP_ERR_INVALID_ARGUMENT, "F < 0");
     if (r.F == 0 || g->n_dst == 0) return TLP_OK;
     if (r.F >= (int64_t(1) << 30)) return set_error(TLP_ERR_INVALID_ARGUMENT, "F too large");
@@ -563,10 +585,14 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             // (built once per handle).  The choice depends on n_src, ldx and
             // the L2 size only (never on P or the gather path override).
             // TLP_BOTH=prescale|edge overrides.
+            // pre-scale only where the L2-panel gathers need a copy of X anyway
+            // (DESIGN.md "Gather layout"); when X fits in L2 the extra pass is
+            // a launch and a full read + write of X for a latency-bound call
+            // (Cora: 37.6 -> 35.5 us without it)
             const double budget = 0.6 * (double)g->l2_bytes;
-            bool edge = 4.0 * (double)g->n_src * (double)r.ldx > budget &&
-                        256.0 * (double)g->n_src > budget;
-            if (const char *e = getenv("TLP_BOTH")) {
+            bool edge = !(4.0 * (double)g->n_src * (double)r.ldx > budget &&
+                          256.0 * (double)g->n_src <= budget);
+            if (const char *e = knob("TLP_BOTH")) {
                 if (!strcmp(e, "prescale")) edge = false;
                 else if (!strcmp(e, "edge")) edge = true;
             }
@@ -600,7 +626,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         const double budget = 0.6 * (double)g->l2_bytes;
         gat_alpha = vec == 4 && 4.0 * (double)g->n_src * (double)r.ldx > budget &&
                     256.0 * (double)g->n_src <= budget;
-        if (const char *e = getenv("TLP_GAT")) {
+        if (const char *e = knob("TLP_GAT")) {
             if (!strcmp(e, "online")) gat_alpha = false;
             else if (!strcmp(e, "alpha")) gat_alpha = true;
         }
@@ -647,7 +673,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         const double budget = 0.6 * (double)g->l2_bytes;
         const double xbytes = 4.0 * (double)g->n_src * (double)r.ldx;
         int mode = -1;  // auto
-        if (const char *e = getenv("TLP_PANEL")) mode = atoi(e);
+        if (const char *e = knob("TLP_PANEL")) mode = atoi(e);
         if (mode == 0) {
             panel_off = true;
         } else if (mode == 128 && vec == 4) {
@@ -686,7 +712,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         const int64_t nv = (r.F + 3) / 4;
         groups = nv <= 4 ? 8 : nv <= 8 ? 4 : nv <= 16 ? 2 : 1;
     }
-    if (const char *e = getenv("TLP_GROUPS")) {
+    if (const char *e = knob("TLP_GROUPS")) {
         const int gq = atoi(e);
         if ((gq == 1 || gq == 2 || gq == 4 || gq == 8) && vec == 4 && lps == 32 && op != OP_GATH)
             groups = gq;
@@ -696,7 +722,8 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     const int n_strips = (int)((r.F + strip_w - 1) / strip_w);
     // Few tasks for the resident warps (small graphs): split every task into its
     // strips as separate work items too, so all SMs get work.
-    if (!panel && !panel_off && n_strips > 1 && g->n_tasks < (int64_t)g->num_sms * 32 * 4) panel = 1;
+    bool spread = false;  // panel set only to spread a small graph's work (not an L2 panel)
+    if (!panel && !panel_off && n_strips > 1 && g->n_tasks < (int64_t)g->num_sms * 32 * 4) panel = spread = 1;
     if (n_strips < 2) panel = 0;
 
     // Gather layout.  In L2-panel mode (X larger
@@ -717,7 +744,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     int layout = 0;  // 0 caller, 1 padded rows, 2 panel-major
     if (panel && vec == 4 && op != OP_GATH) {
         if (4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes) layout = 2;
-        if (const char *e = getenv("TLP_LAYOUT")) {
+        if (const char *e = knob("TLP_LAYOUT")) {
             if (!strcmp(e, "caller")) layout = 0;
             else if (!strcmp(e, "padded")) layout = 1;
             else if (!strcmp(e, "panel")) layout = 2;
@@ -792,6 +819,11 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.ldp = (r.F + 3) / 4 * 4;
     a.row_offset = g->row_offset;
     a.n_tasks = g->n_tasks;
+    a.tasks_magic = 0;
+    a.skip_hubs = 0;
+    a.hub_H = g->H;
+    if (g->n_tasks > 1)  // ceil(2^64 / n_tasks)
+        a.tasks_magic = (unsigned long long)((((unsigned __int128)1) << 64) / (unsigned __int128)g->n_tasks) + 1ull;
     a.n_hubs = g->n_hubs;
     a.n_chunks = g->n_chunks;
     a.C = g->C;
@@ -909,7 +941,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // gathers that stream from HBM need more bytes in flight than registers can
     // hold -> cp.async shared-memory ring.  TLP_GATHER (reg|async) overrides.
     bool async_path = !panel && (4.0 * (double)g->n_src * (double)r.ldx > 0.6 * (double)g->l2_bytes);
-    if (const char *e = getenv("TLP_GATHER")) {
+    if (const char *e = knob("TLP_GATHER")) {
         if (!strcmp(e, "reg")) async_path = false;
         else if (!strcmp(e, "async")) async_path = true;
     }
@@ -924,7 +956,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             a.colidx = g->colidx_tag;
             a.hot_thr = thr;
             a.cold_first = 1;
-            if (const char *e = getenv("TLP_HOT_COLD")) a.cold_first = atoi(e);
+            if (const char *e = knob("TLP_HOT_COLD")) a.cold_first = atoi(e);
         }
     }
     KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, op, coef, groups);
@@ -933,32 +965,83 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;
     if (r.op == OP_GATH)
         smem = (size_t)wpc * (kMhWarpFloats + (async_path ? TLP_DEPTH * 32 * vec : 0)) * sizeof(float);
-    if (smem > 0 && sched == S_HARDWARE) occupancy_blocks(fn, threads, smem);  // sets attributes
-    int64_t blocks;
-    if (sched == S_HARDWARE) {
-        blocks = (a.n_items + wpc - 1) / wpc;
+    // the general persistent kernel over a.n_items work items
+    auto launch_general = [&](const AggArgs &ag) -> tlp_status {
+        if (smem > 0 && sched == S_HARDWARE) occupancy_blocks(fn, threads, smem);  // sets attributes
+        int64_t blocks;
+        if (sched == S_HARDWARE) {
+            blocks = (ag.n_items + wpc - 1) / wpc;
+        } else {
+            int per_sm = occupancy_blocks(fn, threads, smem);
+            if (const char *e = knob("TLP_CTAS"))  // measurement: cap resident CTAs per SM
+                if (atoi(e) > 0) per_sm = std::min(per_sm, atoi(e));
+            blocks = (int64_t)per_sm * g->num_sms;
+            int64_t need = (ag.n_items + (int64_t)wpc * step - 1) / ((int64_t)wpc * step);
+            if (blocks > need) blocks = need;  // tiny graphs: do not launch idle warps
+        }
+        if (blocks < 1) blocks = 1;
+        if (blocks > 0x7fffffff) return set_error(TLP_ERR_UNSUPPORTED, "grid too large");
+        // the kernel walks work items with 32-bit indices
+        if (ag.n_items + (blocks * wpc + 1) * (int64_t)std::max(step, 1) >= (int64_t(1) << 31))
+            return set_error(TLP_ERR_UNSUPPORTED, "too many work items (tasks x strips >= 2^31)");
+        fn<<<(unsigned)blocks, threads, smem, s>>>(ag);
+        g->launches += 1;
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "k_agg launch");
+        return TLP_OK;
+    };
+    // Short-row kernel (tlp_k_rows.cu): one warp per
+    // (row, 128-column strip) item, static round-robin, small
+    // register footprint, next item's row bounds prefetched.  Used by default
+    // for hub-free graphs whose X is L2-resident (latency-bound calls: Cora,
+    // Pubmed).  With hub rows the general kernel runs their chunks first and
+    // the short-row kernel skips them.  Bitwise the same output as the general
+    // kernel (same coefficients, same canonical order), so the choice never
+    // changes a result.  TLP_ROWS=0|1 overrides.
+    const bool rows_ok = (!panel || spread) && groups == 1 && vec == 4 && lps == 32 &&
+                         (op == OP_GCN || op == OP_GIN || op == OP_SAGE || op == OP_GAT) &&
+                         r.op != OP_GATH && r.op != OP_GATB;
+    bool rows_k = rows_ok && g->n_hubs == 0 && !async_path && !panel_off &&
+                  4.0 * (double)g->n_src * (double)r.ldx <= 0.6 * (double)g->l2_bytes &&
+                  knob("TLP_PANEL") == nullptr && knob("TLP_GATHER") == nullptr;
+    if (const char *e = knob("TLP_ROWS")) rows_k = rows_ok && atoi(e) != 0;
+    KernelFn fr = rows_k ? pick_rows(op, coef, a.hot_thr != 0) : nullptr;
+    if (fr) {
+        const int nstr = (int)((r.F + 127) / 128);
+        if (g->n_hubs > 0) {  // hub chunks in the general kernel (tasks [0, n_chunks))
+            AggArgs ah = a;
+            ah.panel = 0;  // task-major: each hub-chunk item covers all strips
+            ah.n_items = g->n_chunks;
+            tlp_status st = launch_general(ah);
+            if (st != TLP_OK) return st;
+        }
+        AggArgs ar = a;
+        // (keeps the hot-source tags and threshold of the cp.async path, if any)
+        ar.n_strips = nstr;
+        ar.panel = 0;
+        ar.skip_hubs = g->n_hubs > 0 ? 1 : 0;
+        ar.hub_H = g->H;
+        ar.n_items = g->n_dst * (int64_t)nstr;
+        ar.tasks_magic = (nstr > 1)
+                             ? (unsigned long long)((((unsigned __int128)1) << 64) / (unsigned __int128)nstr) + 1ull
+                             : 0ull;
+        if (ar.n_items >= (int64_t(1) << 31)) return set_error(TLP_ERR_UNSUPPORTED, "too many rows x strips");
+        const int per_sm = occupancy_blocks(fr, 256, 0);
+        int64_t nb = std::min<int64_t>((int64_t)per_sm * g->num_sms, (ar.n_items + 7) / 8);
+        if (nb < 1) nb = 1;
+        fr<<<(unsigned)nb, 256, 0, s>>>(ar);
+        g->launches += 1;
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "k_rows launch");
     } else {
-        int per_sm = occupancy_blocks(fn, threads, smem);
-        if (const char *e = getenv("TLP_CTAS"))  // measurement: cap resident CTAs per SM
-            if (atoi(e) > 0) per_sm = std::min(per_sm, atoi(e));
-        blocks = (int64_t)per_sm * g->num_sms;
-        int64_t need = (a.n_items + (int64_t)wpc * step - 1) / ((int64_t)wpc * step);
-        if (blocks > need) blocks = need;  // tiny graphs: do not launch idle warps
+        tlp_status st = launch_general(a);
+        if (st != TLP_OK) return st;
     }
-    if (blocks < 1) blocks = 1;
-    if (blocks > 0x7fffffff) return set_error(TLP_ERR_UNSUPPORTED, "grid too large");
-    // the kernel walks work items with 32-bit indices
-    if (a.n_items + (blocks * wpc + 1) * (int64_t)std::max(step, 1) >= (int64_t(1) << 31))
-        return set_error(TLP_ERR_UNSUPPORTED, "too many work items (tasks x strips >= 2^31)");
-    fn<<<(unsigned)blocks, threads, smem, s>>>(a);
-    g->launches += 1;
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_error(e, "k_agg launch");
     if (want_proj) {
         const int pb = (int)std::min<int64_t>((g->n_dst + 255) / 256, (int64_t)g->num_sms * 8);
         k_proj_sum<<<pb, 256, 0, s>>>(g->proj, n_strips, g->n_dst, r.el_out, r.er_out);
         g->launches += 1;
-        e = cudaGetLastError();
+        cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "k_proj_sum launch");
     }
     g->last_stream = s;

@@ -132,6 +132,14 @@ struct AggArgs {
     int64_t ldown;
     int64_t gps;
     int pw;
+    // panel-mode item decode without a division: s = i / n_tasks =
+    // umul64hi(i, tasks_magic) (tasks_magic = ceil(2^64 / n_tasks), exact for
+    // i < 2^32; n_tasks == 1 is special-cased)
+    unsigned long long tasks_magic;
+    // short-row kernel (tlp_k_rows.cu): rows of in-degree > hub_H are skipped
+    // when skip_hubs (their chunks run in the general kernel)
+    int skip_hubs;
+    int64_t hub_H;
 };
 
 constexpr unsigned kIdxMask = (1u << 27) - 1u;
@@ -1005,7 +1013,7 @@ __device__ __forceinline__ void apply_layer_epilogue(const AggArgs &a, int col, 
 
 // Epilogue (a9) for a full row reduction.
 template <int VEC, int OP>
-__device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_t deg, int col,
+__device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int deg, int col,
                                              bool active, const Vec<VEC> &acc, float den) {
     Vec<VEC> y;
     if constexpr (OP == OP_GATB) {
@@ -1028,7 +1036,7 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int64_
         for (int c = 0; c < VEC; ++c) y.v[c] = fmaf(a.eps1, xs.v[c], acc.v[c]);
     } else if constexpr (OP == OP_SAGE) {
         // mean over N(v) (+ v itself when sage_self): (X[v] + sum) / (deg + 1)
-        const int64_t cnt = deg + a.sage_self;
+        const int cnt = deg + a.sage_self;
         const float inv = 1.0f / (float)(cnt > 1 ? cnt : 1);
         Vec<VEC> xs;
 #pragma unroll
@@ -1300,7 +1308,7 @@ __device__ TLP_HUB_INLINE void do_hub_chunk(const AggArgs &a, int h, int j, int 
             for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] / (c < split ? DA : DB);
             apply_layer_epilogue<VEC>(a, col, y);
         } else {
-            y = epilogue<VEC, OP>(a, r, ee - eb, col, active, acc, D);
+            y = epilogue<VEC, OP>(a, r, (int)(ee - eb), col, active, acc, D);
         }
         if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
         if constexpr (OP != OP_GATH) project_row<VEC, G>(a, r, s, col, active, y, lane);
@@ -1318,7 +1326,7 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int i, int lane) {
     int t = i;
     int s0 = 0, s1 = a.n_strips;
     if (a.panel) {
-        s0 = i / (int)a.n_tasks;
+        s0 = (a.n_tasks == 1) ? i : (int)__umul64hi((unsigned long long)(unsigned)i, a.tasks_magic);
         t = i - s0 * (int)a.n_tasks;
         s1 = s0 + 1;
     }
@@ -1415,5 +1423,6 @@ KernelFn pick_g2(int op, int coef);         // PAIR half-warps (64-column strips
 KernelFn pick_g4(int op, int coef);         // 4 lane groups (narrow rows)
 KernelFn pick_g8(int op, int coef);         // 8 lane groups
 KernelFn pick_mh(int vec, bool async_path); // multi-head GAT
+KernelFn pick_rows(int op, int coef, bool hint);  // short-row kernel (tlp_k_rows.cu), VEC 4
 
 }  // namespace tlp

@@ -36,31 +36,34 @@ def timed(f, reps=200):
     return round(plain, 1), round(statistics.median(ts), 1)
 
 
-for name in ("cora", "pubmed"):
-    cfg = synth.CONFIGS[name]
-    rp, ci = synth.dataset_graph(name, device="cuda")
-    n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
-    X = torch.from_numpy(synth.dataset_features(name, n)).cuda()
-    el = torch.from_numpy(synth.normal(n, 1)).cuda()
-    er = torch.from_numpy(synth.normal(n, 2)).cuda()
-    Y = torch.empty((n, ld), device="cuda")
-    envs = [{}, {"TLP_BOTH": "edge"}, {"TLP_PANEL": "0"}, {"TLP_GAT": "alpha"}]
-    for K in (0, 4, 8, 16, 32):
-        g = tlp.Graph(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(),
-                      opts=dict(unit_edges=K) if K else None)
-        for env in envs:
-            if name == "cora" and "TLP_GAT" in env:
-                continue
-            if name == "pubmed" and "TLP_BOTH" in env:
-                continue
-            old = {k: os.environ.get(k) for k in env}
-            os.environ.update(env)
-            f = (lambda: g.gcn(X, "both", Y=Y, F=F)) if name == "cora" else (lambda: g.gat(X, el, er, 0.2, Y=Y, F=F))
-            p, c = timed(f)
-            print(name, "K", K or "default", env, "units", g.info["n_units"], "us plain", p, "graph", c, flush=True)
-            for k, v in old.items():
-                if v is None:
-                    os.environ.pop(k, None)
-                else:
-                    os.environ[k] = v
-        g.close()
+if __name__ != "__main__":
+    pass
+else:
+  for name in ("cora", "pubmed"):
+      cfg = synth.CONFIGS[name]
+      rp, ci = synth.dataset_graph(name, device="cuda")
+      n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+      X = torch.from_numpy(synth.dataset_features(name, n)).cuda()
+      el = torch.from_numpy(synth.normal(n, 1)).cuda()
+      er = torch.from_numpy(synth.normal(n, 2)).cuda()
+      Y = torch.empty((n, ld), device="cuda")
+      envs = [{}, {"TLP_BOTH": "edge"}, {"TLP_PANEL": "0"}, {"TLP_GAT": "alpha"}]
+      for K in (0, 4, 8, 16, 32):
+          g = tlp.Graph(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(),
+                        opts=dict(unit_edges=K) if K else None)
+          for env in envs:
+              if name == "cora" and "TLP_GAT" in env:
+                  continue
+              if name == "pubmed" and "TLP_BOTH" in env:
+                  continue
+              old = {k: os.environ.get(k) for k in env}
+              os.environ.update(env)
+              f = (lambda: g.gcn(X, "both", Y=Y, F=F)) if name == "cora" else (lambda: g.gat(X, el, er, 0.2, Y=Y, F=F))
+              p, c = timed(f)
+              print(name, "K", K or "default", env, "units", g.info["n_units"], "us plain", p, "graph", c, flush=True)
+              for k, v in old.items():
+                  if v is None:
+                      os.environ.pop(k, None)
+                  else:
+                      os.environ[k] = v
+          g.close()

@@ -486,6 +486,77 @@ def test_gather_layouts_bitwise(tlp, monkeypatch, panel, F, ld):
     g.close(); gw.close()
 
 
+@pytest.mark.parametrize("F,ld", [(1433, 1436), (500, 500), (130, 132), (77, 80)])
+def test_short_row_kernel_bitwise(tlp, monkeypatch, F, ld):
+    """The short-row kernel (tlp_k_rows.cu; hub-free graphs with L2-resident X)
+    gives bitwise the general kernel's output for every op it serves (GCN all
+    norms, weighted and unweighted, GIN, SAGE, online GAT), with the fused
+    layer epilogue and projections, and matches the oracle."""
+    n = 2708
+    rp, ci = synth.chung_lu(n, 10556, 0.58, 31, device="cpu")  # Cora-shaped, no hubs
+    Xh = synth.features(n, F, ld, seed=8)
+    X = _t(Xh)
+    elh, erh = synth.normal(n, 1), synth.normal(n, 2)
+    el, er = _t(elh), _t(erh)
+    ew = _t(synth.edge_weights(len(ci), 5))
+    g = tlp.Graph(_t(rp), _t(ci))
+    gw = tlp.Graph(_t(rp), _t(ci), edge_weight=ew)
+    assert g.info["n_hubs"] == 0
+    bias = _t(synth.normal(F, 3))
+    att = _t(synth.normal(F, 4))
+    outs = {}
+    for mode, major in (("0", "0"), ("1", "0")):
+        monkeypatch.setenv("TLP_ROWS", mode)
+        res = [g.gcn(X, nm, F=F) for nm in ("none", "right", "both")]
+        res += [gw.gcn(X, nm, F=F) for nm in ("right", "both")]
+        res += [g.gin(X, 0.1, F=F), gw.gin(X, 0.1, F=F), g.sage(X, True, F=F), g.sage(X, False, F=F),
+                g.gat(X, el, er, 0.2, F=F)]
+        elo = torch.empty(n, device=DEV)
+        res.append(g.aggregate("gat", X, F=F, el=el, er=er, slope=0.2, bias=bias, act="leaky_relu",
+                               act_param=0.1, att_l=att, el_out=elo))
+        res.append(elo)
+        torch.cuda.synchronize()
+        outs[mode + major] = [r.clone() for r in res]
+    for i, (a, b) in enumerate(zip(outs["10"], outs["00"])):
+        assert torch.equal(a, b), i
+    _check("rows gcn", outs["10"][2], oracle.gcn(rp, ci, Xh, "both", F=F))
+    _check("rows gin", outs["10"][5], oracle.gin(rp, ci, Xh, 0.1, F=F))
+    _check("rows gat", outs["10"][9], oracle.gat(rp, ci, Xh, elh, erh, 0.2, F=F))
+    g.close(); gw.close()
+
+
+@pytest.mark.parametrize("F,ld", [(300, 300), (100, 100)])
+def test_short_row_kernel_with_hub_split_bitwise(tlp, monkeypatch, F, ld):
+    """With hub rows, the general kernel runs the hub chunks and the short-row
+    kernel the other rows (TLP_ROWS=1): bitwise the general kernel's output,
+    for both gather paths of the general kernel and the hot-source hints."""
+    n = 4000
+    deg = np.minimum((3000.0 / (np.arange(n) + 1) ** 0.7).astype(np.int64) + 1, 2500)
+    rp, ci = synth.power_law_rows(n, np.random.default_rng(3).permutation(deg), n, seed=4)
+    Xh = synth.features(n, F, ld, seed=9)
+    X = _t(Xh)
+    elh, erh = synth.normal(n, 1), synth.normal(n, 2)
+    el, er = _t(elh), _t(erh)
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=200, hub_chunk=96))
+    assert g.info["n_hubs"] > 0
+    outs = {}
+    for gather in ("reg", "async"):
+        monkeypatch.setenv("TLP_GATHER", gather)
+        # async: the hot-source tags ride along (TLP_HOT forces them on an L2-sized X)
+        monkeypatch.setenv("TLP_HOT", "0.01" if gather == "async" else "0")
+        for mode, major in (("0", "0"), ("1", "0")):
+            monkeypatch.setenv("TLP_ROWS", mode)
+            outs[gather + mode + major] = [g.gcn(X, "both", F=F).clone(), g.gin(X, 0.1, F=F).clone(),
+                                           g.sage(X, True, F=F).clone(), g.gat(X, el, er, 0.2, F=F).clone()]
+    ref = outs["reg00"]
+    for key, res in outs.items():
+        for i, (a, b) in enumerate(zip(res, ref)):
+            assert torch.equal(a, b), (key, i)
+    _check("split gat", outs["async10"][3], oracle.gat(rp, ci, Xh, elh, erh, 0.2, F=F))
+    _check("split gcn", outs["async10"][0], oracle.gcn(rp, ci, Xh, "both", F=F))
+    g.close()
+
+
 @pytest.mark.parametrize("F,ld", [(100, 100), (300, 300), (37, 40), (5, 6)])
 def test_gather_paths_bitwise(tlp, monkeypatch, F, ld):
     """Register double-buffered and cp.async shared-memory gathers agree bit for bit."""
