@@ -36,7 +36,7 @@ __global__ void __launch_bounds__(256, 4) gather(const float4 *__restrict__ tab,
 #pragma unroll
         for (int k = 0; k < U; ++k) {
             x ^= x << 13; x ^= x >> 17; x ^= x << 5;
-            v[k] = __ldg(tab + (int64_t)(x % nrows) * 16 + col);
+            v[k] = __ldg(tab + (int64_t)__umulhi(x, nrows) * 16 + col);  // fast range reduction
         }
 #pragma unroll
         for (int k = 0; k < U; ++k) { acc.x += v[k].x; acc.y += v[k].y; acc.z += v[k].z; acc.w += v[k].w; }

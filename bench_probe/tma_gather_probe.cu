@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(256, 4) ldg_gather(const float4 *__restrict__ 
 #pragma unroll
         for (int k = 0; k < U; ++k) {
             x ^= x << 13; x ^= x >> 17; x ^= x << 5;
-            v[k] = __ldg(tab + (int64_t)(x % nrows) * 16 + col);
+            v[k] = __ldg(tab + (int64_t)__umulhi(x, nrows) * 16 + col);  // fast range reduction
         }
 #pragma unroll
         for (int k = 0; k < U; ++k) { acc.x += v[k].x; acc.y += v[k].y; acc.z += v[k].z; acc.w += v[k].w; }
@@ -75,7 +75,7 @@ __global__ void __launch_bounds__(256, 1) tma_gather(const __grid_constant__ CUt
         asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&full[s])), "r"(STAGE_BYTES));
         for (int q = 0; q < G4; ++q) {
             int r[4];
-            for (int k = 0; k < 4; ++k) { x ^= x << 13; x ^= x >> 17; x ^= x << 5; r[k] = (int)(x % nrows); }
+            for (int k = 0; k < 4; ++k) { x ^= x << 13; x ^= x >> 17; x ^= x << 5; r[k] = (int)__umulhi(x, nrows); }
             asm volatile(
                 "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
                 " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];"

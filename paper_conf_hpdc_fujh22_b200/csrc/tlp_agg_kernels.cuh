@@ -1045,8 +1045,11 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int de
 #pragma unroll
         for (int c = 0; c < VEC; ++c) y.v[c] = (xs.v[c] + acc.v[c]) * inv;
     } else {
+        // GAT: Y = acc / den, as one reciprocal and VEC products (every
+        // single-head path -- general, short-row, hub merge -- shares this)
+        const float inv = deg > 0 ? 1.0f / den : 0.f;
 #pragma unroll
-        for (int c = 0; c < VEC; ++c) y.v[c] = deg > 0 ? acc.v[c] / den : 0.f;
+        for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] * inv;
     }
     apply_layer_epilogue<VEC>(a, col, y);
     return y;
@@ -1159,10 +1162,11 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                                                 Mh, Dh, h_lo, nh, hl, split);
                     const float dA = Dh[hl], dB = Dh[min(hl + 1, nh - 1)];
                     __syncwarp();  // the head state is reset by the next strip / row
+                    // one reciprocal per head and products, as the single-head epilogue
+                    const float iA = (e1 > e0) ? 1.0f / dA : 0.f, iB = (e1 > e0) ? 1.0f / dB : 0.f;
                     Vec<VEC> y;
 #pragma unroll
-                    for (int c = 0; c < VEC; ++c)
-                        y.v[c] = (e1 > e0) ? acc.v[c] / (c < split ? dA : dB) : 0.f;
+                    for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] * (c < split ? iA : iB);
                     apply_layer_epilogue<VEC>(a, col, y);
                     if (active) store_out<VEC>(a, r, col, y);
                     continue;
@@ -1304,8 +1308,9 @@ __device__ TLP_HUB_INLINE void do_hub_chunk(const AggArgs &a, int h, int j, int 
         }
         Vec<VEC> y;
         if constexpr (OP == OP_GATH) {
+            const float iA = 1.0f / DA, iB = 1.0f / DB;
 #pragma unroll
-            for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] / (c < split ? DA : DB);
+            for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] * (c < split ? iA : iB);
             apply_layer_epilogue<VEC>(a, col, y);
         } else {
             y = epilogue<VEC, OP>(a, r, (int)(ee - eb), col, active, acc, D);

@@ -10,7 +10,7 @@ name, op = sys.argv[1], sys.argv[2]
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 4
 cfg = synth.CONFIGS[name]
 rp, ci = synth.dataset_graph(name, device="cuda")
-n, F, ld = cfg["n"], cfg["F"], cfg["ld"]
+n, F, ld = cfg.get("n", 1 << cfg.get("scale", 0)), cfg["F"], cfg["ld"]
 X = torch.from_numpy(synth.dataset_features(name, n)).cuda()
 el = torch.from_numpy(synth.normal(n, 1)).cuda()
 er = torch.from_numpy(synth.normal(n, 2)).cuda()
