@@ -67,9 +67,19 @@ __global__ void k_colidx_check(const int32_t *__restrict__ colidx, int64_t nnz,
 
 __global__ void k_out_degree(const int32_t *__restrict__ colidx, int64_t nnz,
                              int32_t *__restrict__ out_deg) {
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz;
-         e += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(&out_deg[colidx[e]], 1);  // integer: exact in any order
+    // 8 independent index loads in flight per thread before their fire-and-
+    // forget reductions (the loads cannot be hoisted across the atomics by the
+    // compiler on its own)
+    constexpr int UN = 8;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nnz; b += stride * UN) {
+        int32_t u[UN];
+#pragma unroll
+        for (int k = 0; k < UN; ++k) u[k] = (b + k * stride < nnz) ? __ldg(colidx + b + k * stride) : -1;
+#pragma unroll
+        for (int k = 0; k < UN; ++k)
+            if (u[k] >= 0) atomicAdd(&out_deg[u[k]], 1);  // integer: exact in any order
+    }
 }
 
 // c_out[u] = 1/sqrt(max(out_deg,1)) (BOTH norm, Kipf [26]; R1) and

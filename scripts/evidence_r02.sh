@@ -33,5 +33,13 @@ if [ "$P" = "ncu" ] || [ "$P" = "all" ]; then
   prof rmat24_gcn k_agg 3 python scripts/one_call.py rmat24 gcn 4
   prof cora_gcn k_rows 3 python scripts/one_call.py cora gcn 4
   prof pubmed_gat k_rows 3 python scripts/one_call.py pubmed gat 4
+  prof reddit_outdeg k_out_degree 1 python scripts/create_probe.py reddit
+  TLP_TRACE_CREATE=1 python scripts/create_probe.py reddit > $O/create_probe.txt 2>&1
 fi
 ls -la $O
+if [ "$P" = "probes" ] || [ "$P" = "all" ]; then
+  nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/tma_probe bench_probe/tma_gather_probe.cu -lcuda > $O/tma_build.log 2>&1
+  timeout 300 /tmp/tma_probe > $O/tma_probe.txt 2>&1
+  python scripts/host_probe.py > $O/host_probe.txt 2>&1
+  (cd scripts && python small_probe2.py > ../$O/small_probe.txt 2>&1)
+fi
