@@ -304,17 +304,21 @@ __device__ __forceinline__ void issue_group(const char *base, unsigned row_bytes
 }
 
 // PHASE: parity of the group's first step (the caller's j is a multiple of 2U).
-template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE, bool SMC = false>
+template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE, bool SMC = false, bool SHC = false>
 __device__ __forceinline__ void consume_group(int j, int n, int grp, const Vec<VEC> (&xv)[U],
                                               const float (&ck)[U], Vec<VEC> (&ac)[2],
-                                              const float *cw = nullptr) {
+                                              const float *cw = nullptr, float c_l = 0.f) {
 #pragma unroll
     for (int k = 0; k < U; ++k) {
         const int p = G * (j + k) + grp;
         const int ch = (G > 1) ? 0 : ((PHASE + k) & 1);
+        // (the shuffle runs on every lane: lane groups past the chunk end take
+        // a clamped index; their value is not used)
+        float cvs = 0.f;
+        if constexpr (HASC && SHC) cvs = __shfl_sync(FULL, c_l, GUARD ? min(p, n - 1) : p);
         if (!GUARD || p < n) {
             float cv = 0.f;
-            if constexpr (HASC) cv = SMC ? cw[p] : ck[k];
+            if constexpr (HASC) cv = SHC ? cvs : (SMC ? cw[p] : ck[k]);
 #pragma unroll
             for (int c = 0; c < VEC; ++c) {
                 if constexpr (HASC) ac[ch].v[c] = fmaf(cv, xv[k].v[c], ac[ch].v[c]);
@@ -453,7 +457,11 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     static_assert(STEPS % (2 * U) == 0, "U must divide the gather steps of a chunk in two groups");
     static_assert(!GB || G <= 2, "GAT backward edge dots: full warp or PAIR only");
     constexpr bool PAIR = (G == 2);
-    constexpr bool SMC = TLP_SMEMC && HASC && (G > 1);
+    // lane-group coefficients: TLP_SMEMC 1 = chunk row in shared memory, read
+    // at consume time; 2 = shuffled from the owning lane at consume time
+    constexpr bool SHC = (TLP_SMEMC == 2) && HASC && (G > 1);
+    constexpr bool SMC = (TLP_SMEMC == 1) && HASC && (G > 1);
+    constexpr bool NOCK = SMC || SHC;  // no coefficient register per row in flight
     float *cw = SMC ? chunk_coef_smem() : nullptr;
     // lanes past F read column 0 of the strip (a valid address); their results
     // are never stored.  Panel-major gather layout: strip s is a block of pw
@@ -536,29 +544,29 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             DotTree dt_;      // OP_GATB (full chunk): pending butterfly levels
             if (n0 == 32) {
                 // full chunk: fully unrolled, compile-time shuffle lanes, no guards
-                issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, 0, 32, grp, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, G, false, NOCK>(base, row_bytes, 0, 32, grp, u0, c_l, xa, ca);
 #pragma unroll
                 for (int j = 0; j < STEPS; j += 2 * U) {
-                    issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, j + U, 32, grp, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, G, false, 0, SMC>(j, 32, grp, xa, ca, ac, cw);
+                    issue_group<VEC, U, HASC, G, false, NOCK>(base, row_bytes, j + U, 32, grp, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, G, false, 0, SMC, SHC>(j, 32, grp, xa, ca, ac, cw, c_l);
                     if constexpr (GB) dot_tree<VEC, U, PAIR>(j, lane, xa, xu, dt_, gout + off);
                     if (j + 2 * U < STEPS)
-                        issue_group<VEC, U, HASC, G, false, SMC>(base, row_bytes, j + 2 * U, 32, grp, u0, c_l, xa, ca);
-                    consume_group<VEC, U, HASC, G, false, U, SMC>(j + U, 32, grp, xb, cb, ac, cw);
+                        issue_group<VEC, U, HASC, G, false, NOCK>(base, row_bytes, j + 2 * U, 32, grp, u0, c_l, xa, ca);
+                    consume_group<VEC, U, HASC, G, false, U, SMC, SHC>(j + U, 32, grp, xb, cb, ac, cw, c_l);
                     if constexpr (GB) dot_tree<VEC, U, PAIR>(j + U, lane, xb, xu, dt_, gout + off);
                 }
             } else {
                 // partial chunk (n0 is warp-uniform: the guards never diverge)
                 const int steps = (n0 + G - 1) / G;
-                issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, 0, n0, grp, u0, c_l, xa, ca);
+                issue_group<VEC, U, HASC, G, true, NOCK>(base, row_bytes, 0, n0, grp, u0, c_l, xa, ca);
                 for (int j = 0; j < steps; j += 2 * U) {
                     const bool more = j + U < steps;
-                    if (more) issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, j + U, n0, grp, u0, c_l, xb, cb);
-                    consume_group<VEC, U, HASC, G, true, 0, SMC>(j, n0, grp, xa, ca, ac, cw);
+                    if (more) issue_group<VEC, U, HASC, G, true, NOCK>(base, row_bytes, j + U, n0, grp, u0, c_l, xb, cb);
+                    consume_group<VEC, U, HASC, G, true, 0, SMC, SHC>(j, n0, grp, xa, ca, ac, cw, c_l);
                     if constexpr (GB) dot_group<VEC, U, PAIR, true>(j, n0, lane, xa, xu, g_l);
                     if (j + 2 * U < steps)
-                        issue_group<VEC, U, HASC, G, true, SMC>(base, row_bytes, j + 2 * U, n0, grp, u0, c_l, xa, ca);
-                    if (more) consume_group<VEC, U, HASC, G, true, U, SMC>(j + U, n0, grp, xb, cb, ac, cw);
+                        issue_group<VEC, U, HASC, G, true, NOCK>(base, row_bytes, j + 2 * U, n0, grp, u0, c_l, xa, ca);
+                    if (more) consume_group<VEC, U, HASC, G, true, U, SMC, SHC>(j + U, n0, grp, xb, cb, ac, cw, c_l);
                     if constexpr (GB)
                         if (more) dot_group<VEC, U, PAIR, true>(j + U, n0, lane, xb, xu, g_l);
                 }
@@ -687,6 +695,48 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
         }
         if constexpr (DEP)
             if (lane < n0) d0 = __ldg(dep + (u0 & kIdxMask));
+        if (len < D) {
+            // short row (R-MAT / products have many): its rows go into ring
+            // slots 0 .. len-1 under ONE commit group and one wait, instead of
+            // the D-1 prologue groups and a wait per edge of the pipeline below
+            // (same values, same order: bitwise the pipelined result)
+            for (int k = 0; k < len; ++k) {
+                const int uk = __shfl_sync(FULL, u0, k);
+                cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active);
+            }
+            cp_async_commit();
+            float c_l = 1.f;
+            if constexpr (OP == OP_GAT) {
+                float s = -INFINITY;
+                if (lane < n0) {
+                    const float t = d0 + er_v;
+                    s = t >= 0.f ? t : a.slope * t;
+                }
+                const float m_new = fmaxf(m, warp_max(s));
+                const float scale = __expf(m - m_new);
+                c_l = (lane < n0) ? __expf(s - m_new) : 0.f;
+                den = fmaf(den, scale, warp_sum(c_l));
+#pragma unroll
+                for (int c = 0; c < VEC; ++c) {
+                    ae.v[c] *= scale;
+                    ao.v[c] *= scale;
+                }
+                m = m_new;
+            } else {
+                if constexpr (COEF & COEF_COUT) c_l = d0;
+                if constexpr (COEF & COEF_W) c_l *= w0;
+            }
+            cp_async_wait<0>();
+            for (int j = 0; j < len; ++j) {
+                const float cj = __shfl_sync(FULL, c_l, j);
+                if (j & 1) acc_from_smem<VEC, HASC>(ring + j * 32 * VEC, cj, ao);
+                else acc_from_smem<VEC, HASC>(ring + j * 32 * VEC, cj, ae);
+            }
+            __syncwarp();  // the ring is rewritten by the next row
+#pragma unroll
+            for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
+            return;
+        }
         // prologue: edges 0 .. D-2 in flight
 #pragma unroll
         for (int k = 0; k < D - 1; ++k) {
