@@ -822,6 +822,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.tasks_magic = 0;
     a.skip_hubs = 0;
     a.hub_H = g->H;
+    a.stream_hint = 0;
     if (g->n_tasks > 1)  // ceil(2^64 / n_tasks)
         a.tasks_magic = (unsigned long long)((((unsigned __int128)1) << 64) / (unsigned __int128)g->n_tasks) + 1ull;
     a.n_hubs = g->n_hubs;
@@ -959,6 +960,10 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
             if (const char *e = knob("TLP_HOT_COLD")) a.cold_first = atoi(e);
         }
     }
+    // L2 stream hints in L2-panel mode only;
+    // TLP_HINTS=0|1 overrides
+    a.stream_hint = (panel && !spread && !async_path) ? 1 : 0;
+    if (const char *e = knob("TLP_HINTS")) a.stream_hint = atoi(e) != 0;
     KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, op, coef, groups);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;

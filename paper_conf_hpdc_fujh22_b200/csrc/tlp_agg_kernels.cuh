@@ -64,9 +64,7 @@ constexpr unsigned FULL = 0xffffffffu;
 #ifndef TLP_MHB
 #define TLP_MHB 4      // multi-head GAT: heads scored together per pass
 #endif
-#ifndef TLP_HINTS
-#define TLP_HINTS 0    // 1: L2 evict_first policy on per-edge streams and Y stores (measured: no gain)
-#endif
+
 #ifndef TLP_MINB_LIGHT
 #define TLP_MINB_LIGHT 4  // register path, no edge coefficient (GIN, SAGE): <= 64 registers, 32 warps/SM
 #endif
@@ -140,6 +138,7 @@ struct AggArgs {
     // when skip_hubs (their chunks run in the general kernel)
     int skip_hubs;
     int64_t hub_H;
+    int stream_hint;  // L2 evict_first on the per-edge streams and Y stores (L2-panel mode)
 };
 
 constexpr unsigned kIdxMask = (1u << 27) - 1u;
@@ -197,17 +196,16 @@ __device__ __forceinline__ Vec<VEC> ld_vec_cg(const float *p) {
     return r;
 }
 
+// pol != 0: the store carries that L2 cache policy (evict_first for Y in
+// L2-panel mode)
 template <int VEC>
-__device__ __forceinline__ void st_vec(float *p, const Vec<VEC> &x) {
+__device__ __forceinline__ void st_vec(float *p, const Vec<VEC> &x, unsigned long long pol = 0ull) {
     if constexpr (VEC == 4) {
-#if TLP_HINTS
-        unsigned long long pol;
-        asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
-                     ::"l"(p), "f"(x.v[0]), "f"(x.v[1]), "f"(x.v[2]), "f"(x.v[3]), "l"(pol) : "memory");
-#else
-        *reinterpret_cast<float4 *>(p) = make_float4(x.v[0], x.v[1], x.v[2], x.v[3]);
-#endif
+        if (pol)
+            asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
+                         ::"l"(p), "f"(x.v[0]), "f"(x.v[1]), "f"(x.v[2]), "f"(x.v[3]), "l"(pol) : "memory");
+        else
+            *reinterpret_cast<float4 *>(p) = make_float4(x.v[0], x.v[1], x.v[2], x.v[3]);
     } else if constexpr (VEC == 2) {
         *reinterpret_cast<float2 *>(p) = make_float2(x.v[0], x.v[1]);
     } else {
@@ -217,9 +215,10 @@ __device__ __forceinline__ void st_vec(float *p, const Vec<VEC> &x) {
 
 // Store only columns < F (the tail vector of a row may straddle F).
 template <int VEC>
-__device__ __forceinline__ void st_row(float *row, int col, int F, const Vec<VEC> &x) {
+__device__ __forceinline__ void st_row(float *row, int col, int F, const Vec<VEC> &x,
+                                       unsigned long long pol = 0ull) {
     if (col + VEC <= F) {
-        st_vec<VEC>(row + col, x);
+        st_vec<VEC>(row + col, x, pol);
     } else {
 #pragma unroll
         for (int c = 0; c < VEC; ++c)
@@ -401,34 +400,31 @@ __device__ __forceinline__ void dot_tree(int j, int lane, const Vec<VEC> (&xv)[U
     }
 }
 
-// ---- L2 residency hints -------------------------------------------------------
-// Per-edge streams (colidx, edge coefficients) and Y are touched once per strip:
-// with TLP_HINTS they are loaded / stored with an L2 evict_first policy so they
-// do not evict the L2-resident panel of X that every edge gathers from.
+// ---- L2 stream hints --------------------------------
+// In L2-panel mode the per-edge streams (colidx, edge coefficients such as
+// GAT's alpha) and the Y stores are touched once per strip: loaded / stored
+// with an L2 evict_first policy they do not evict the L2-resident panel of X
+// that every edge gathers from (a.stream_hint; measured: Reddit GAT 19.4 ->
+// 18.4 ms, GCN 16.7 -> 16.3; on HBM-streaming inputs it costs 2-3 %, so it is
+// off there).  A cache policy only: no value changes.
 __device__ __forceinline__ unsigned long long policy_evict_first() {
     unsigned long long p;
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
-__device__ __forceinline__ int ld_stream(const int32_t *ptr) {
-#if TLP_HINTS
+__device__ __forceinline__ int ld_stream(const int32_t *ptr, unsigned long long pol = 0ull) {
+    if (!pol) return __ldg(ptr);
     int v;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
-                 : "=r"(v) : "l"(ptr), "l"(policy_evict_first()));
+                 : "=r"(v) : "l"(ptr), "l"(pol));
     return v;
-#else
-    return __ldg(ptr);
-#endif
 }
-__device__ __forceinline__ float ld_stream(const float *ptr) {
-#if TLP_HINTS
+__device__ __forceinline__ float ld_stream(const float *ptr, unsigned long long pol = 0ull) {
+    if (!pol) return __ldg(ptr);
     float v;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
-                 : "=f"(v) : "l"(ptr), "l"(policy_evict_first()));
+                 : "=f"(v) : "l"(ptr), "l"(pol));
     return v;
-#else
-    return __ldg(ptr);
-#endif
 }
 
 // Reduce the edges [e0, e1) of one destination row for the feature vector at
@@ -481,6 +477,7 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
     const float *__restrict__ wp = (COEF & COEF_W) ? a.ew + e0 : nullptr;
     const int len = (int)(e1 - e0);
     const int grp = lane / (32 / G);  // lane group (G > 1)
+    const unsigned long long spol = a.stream_hint ? policy_evict_first() : 0ull;
     Vec<VEC> ac[2];
 #pragma unroll
     for (int c = 0; c < VEC; ++c) ac[0].v[c] = ac[1].v[c] = 0.f;
@@ -491,12 +488,12 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
         int u0 = 0, u1 = 0;
         float w0 = 1.f, w1 = 1.f, d0 = 0.f, d1 = 0.f;
         if (lane < n0) {
-            u0 = ld_stream(ci + lane);
-            if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane);
+            u0 = ld_stream(ci + lane, spol);
+            if constexpr (COEF & COEF_W) w0 = ld_stream(wp + lane, spol);
         }
         if (lane < n1) {
-            u1 = ld_stream(ci + 32 + lane);
-            if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
+            u1 = ld_stream(ci + 32 + lane, spol);
+            if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane, spol);
         }
         if constexpr (DEP)
             if (lane < n0) d0 = __ldg(dep + u0);
@@ -506,8 +503,8 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             int u2 = 0;
             float w2 = 1.f;
             if (lane < n2) {
-                u2 = ld_stream(ci + off + 64 + lane);
-                if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
+                u2 = ld_stream(ci + off + 64 + lane, spol);
+                if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane, spol);
             }
             if constexpr (DEP)
                 if (lane < n1) d1 = __ldg(dep + u1);
@@ -602,6 +599,9 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
 // in flight then cost no registers, so occupancy and depth are decoupled.
 #ifndef TLP_DEPTH
 #define TLP_DEPTH 16   // edges in flight per warp on the async path
+#endif
+#ifndef TLP_ASYNC_PAIR
+#define TLP_ASYNC_PAIR 1  // two edges per cp.async commit group (fewer waits per edge)
 #endif
 
 template <int VEC>
@@ -737,6 +737,18 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
             for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
             return;
         }
+#if TLP_ASYNC_PAIR
+        // prologue: edges 0 .. D-3 in flight, two edges per commit group
+        static_assert(D % 2 == 0, "paired async pipeline needs an even ring depth");
+#pragma unroll
+        for (int k = 0; k < D - 2; k += 2) {
+            const int ua = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
+            const int ub = __shfl_sync(FULL, k + 1 < 32 ? u0 : u1, (k + 1) & 31);
+            cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && k < len);
+            cp_async_x<VEC>(ring + (k + 1) * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && k + 1 < len);
+            cp_async_commit();
+        }
+#else
         // prologue: edges 0 .. D-2 in flight
 #pragma unroll
         for (int k = 0; k < D - 1; ++k) {
@@ -744,6 +756,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
             cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active && k < len);
             cp_async_commit();
         }
+#endif
         int slot = 0;  // ring slot of edge `off + j`
         while (true) {
             const int n2 = min(32, len - off - 64);
@@ -776,6 +789,29 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
                 if constexpr (COEF & COEF_COUT) c_l = d0;
                 if constexpr (COEF & COEF_W) c_l *= w0;
             }
+#if TLP_ASYNC_PAIR
+            // edges in pairs: one commit group and one wait per two edges; the
+            // pair's first edge is at an even position (chunks start at even
+            // offsets), so it feeds the even chain and the second the odd one
+            for (int j = 0; j < n0; j += 2) {
+                const int ja = j + D - 2, jb = j + D - 1;  // in this chunk or the next one
+                const int ua = __shfl_sync(FULL, ja < 32 ? u0 : u1, ja & 31);
+                const int ub = __shfl_sync(FULL, jb < 32 ? u0 : u1, jb & 31);
+                int wa = slot + D - 2;
+                if (wa >= D) wa -= D;
+                const int wb = wa + 1;  // slot and D are even
+                cp_async_x<VEC>(ring + wa * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && (off + ja) < len);
+                cp_async_x<VEC>(ring + wb * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && (off + jb) < len);
+                cp_async_commit();
+                cp_async_wait<(D - 2) / 2>();
+                const float ca = __shfl_sync(FULL, c_l, j);
+                const float cb = __shfl_sync(FULL, c_l, min(j + 1, 31));
+                acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, ca, ae);
+                if (j + 1 < n0) acc_from_smem<VEC, HASC>(ring + (slot + 1) * 32 * VEC, cb, ao);
+                slot += 2;
+                if (slot == D) slot = 0;
+            }
+#else
             for (int j = 0; j < n0; ++j) {
                 // issue edge j + D - 1 (in this chunk or the next one)
                 const int jj = j + D - 1;
@@ -792,6 +828,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
                 else acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, cj, ae);
                 if (++slot == D) slot = 0;
             }
+#endif
             if (n1 <= 0) break;
             off += 32;
             n0 = n1; n1 = n2;
@@ -1110,7 +1147,7 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int de
 template <int VEC>
 __device__ __forceinline__ void store_out(const AggArgs &a, int64_t r, int col, const Vec<VEC> &y) {
     if (a.n_dests == 0) {
-        st_row<VEC>(a.Y + r * a.ldy, col, a.F, y);
+        st_row<VEC>(a.Y + r * a.ldy, col, a.F, y, a.stream_hint ? policy_evict_first() : 0ull);
     } else {
         const int64_t off = (a.row_offset + r) * a.ldy;
         for (int i = 0; i < a.n_dests; ++i) st_row<VEC>(a.dests[i] + off, col, a.F, y);
