@@ -218,6 +218,15 @@ tlp_status tlp_graph_plan(tlp_graph g, int32_t *tasks, int32_t *hub_rows,
 
 /* Selects the scheduler (tlp_sched), warps per CTA (0 = default 8) and the
  * tasks fetched per atomic (Alg. 1's `step`; 0 = derived from F). */
+/* Debug visit counter (Alg. 1's exactly-once semantics,
+ * P:883-906): while `counter` (device int32 [n_dst], zeroed by the caller) is
+ * set, every aggregation on this handle adds 1 to counter[r] each time it
+ * finishes one feature strip of local row r -- after a call every row holds
+ * exactly the number of strips that call used (hub rows included: their
+ * chunk partials are merged, and the row stored, once per strip).  Borrowed
+ * until reset with NULL.  Costs one atomic per row strip; off by default. */
+tlp_status tlp_graph_set_visit_counter(tlp_graph g, int32_t *counter);
+
 tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta,
                                   int step);
 

@@ -81,6 +81,7 @@ _sig = {
     "tlp_graph_degrees": ([_P, _P, _P, _P], _I),
     "tlp_graph_plan": ([_P, _P, _P, _P, _P], _I),
     "tlp_graph_set_schedule": ([_P, _I, _I, _I], _I),
+    "tlp_graph_set_visit_counter": ([_P, _P], _I),
     "tlp_graph_build_transpose": ([_P, _P], _I),
     "tlp_gcn_backward": ([_P, _P, _I64, _I64, _I, _P, _I64, _P], _I),
     "tlp_gin_backward": ([_P, _P, _I64, _I64, _F, _P, _I64, _P], _I),
@@ -325,6 +326,16 @@ def tlp_graph_set_schedule(g, sched="dynamic", warps_per_cta=0, step=0):
     s = SCHEDS[sched] if isinstance(sched, str) else int(sched)
     _check(_lib.tlp_graph_set_schedule(g, s, int(warps_per_cta), int(step)),
            "tlp_graph_set_schedule")
+
+
+def tlp_graph_set_visit_counter(g, counter=None):
+    """Debug: count finished (row, strip) stores into `counter` (int32 CUDA
+    tensor [n_dst], zeroed by the caller); None switches it off."""
+    torch = _torch()
+    if counter is not None and (not isinstance(counter, torch.Tensor) or not counter.is_cuda
+                                or counter.dtype != torch.int32 or not counter.is_contiguous()):
+        raise TypeError("counter must be a contiguous int32 CUDA tensor")
+    _check(_lib.tlp_graph_set_visit_counter(g, _ptr(counter)), "tlp_graph_set_visit_counter")
 
 
 def tlp_graph_build_transpose(g, stream=None):

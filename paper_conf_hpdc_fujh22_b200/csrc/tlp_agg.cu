@@ -823,6 +823,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.skip_hubs = 0;
     a.hub_H = g->H;
     a.stream_hint = 0;
+    a.visits = g->visits;
     if (g->n_tasks > 1)  // ceil(2^64 / n_tasks)
         a.tasks_magic = (unsigned long long)((((unsigned __int128)1) << 64) / (unsigned __int128)g->n_tasks) + 1ull;
     a.n_hubs = g->n_hubs;

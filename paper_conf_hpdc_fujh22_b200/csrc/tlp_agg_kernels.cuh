@@ -139,7 +139,15 @@ struct AggArgs {
     int skip_hubs;
     int64_t hub_H;
     int stream_hint;  // L2 evict_first on the per-edge streams and Y stores (L2-panel mode)
+    // debug visit counter (Alg. 1's exactly-once semantics):
+    // visits[r] += 1 per finished (row, strip) store; NULL = off
+    int32_t *visits;
 };
+
+// One finished (row, strip) of local row r (warp-uniform call).
+__device__ __forceinline__ void count_visit(const AggArgs &a, int64_t r, int lane) {
+    if (a.visits && lane == 0) atomicAdd(a.visits + r, 1);
+}
 
 constexpr unsigned kIdxMask = (1u << 27) - 1u;
 
@@ -1030,11 +1038,22 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
         int u0 = (lane < n0) ? __ldg(ci + lane) : 0;
         int u1 = (lane < n1) ? __ldg(ci + 32 + lane) : 0;
 #pragma unroll
+#if TLP_ASYNC_PAIR
+        for (int k = 0; k < DD - 2; k += 2) {  // two edges per commit group
+            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
+            const int ub = __shfl_sync(FULL, k + 1 < 32 ? u0 : u1, (k + 1) & 31);
+            cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
+            cp_async_vec<VEC>(ring + (k + 1) * 32 * VEC, row_ptr(base, (unsigned)ub, row_bytes),
+                              active && k + 1 < len);
+            cp_async_commit();
+        }
+#else
         for (int k = 0; k < DD - 1; ++k) {
             const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
             cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
             cp_async_commit();
         }
+#endif
         int slot = 0, off = 0;
         while (true) {
             const int n2 = min(32, len - off - 64);
@@ -1049,6 +1068,35 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
             }
             const float *pa = P + hl * 32;
             const float *pb = P + hl2 * 32;
+#if TLP_ASYNC_PAIR
+            for (int j = 0; j < n0; j += 2) {  // as the single-head pipeline
+                const int ja = j + DD - 2, jb = j + DD - 1;
+                const int ua = __shfl_sync(FULL, ja < 32 ? u0 : u1, ja & 31);
+                const int ub = __shfl_sync(FULL, jb < 32 ? u0 : u1, jb & 31);
+                int wa = slot + DD - 2;
+                if (wa >= DD) wa -= DD;
+                cp_async_vec<VEC>(ring + wa * 32 * VEC, row_ptr(base, (unsigned)ua, row_bytes),
+                                  active && (off + ja) < len);
+                cp_async_vec<VEC>(ring + (wa + 1) * 32 * VEC, row_ptr(base, (unsigned)ub, row_bytes),
+                                  active && (off + jb) < len);
+                cp_async_commit();
+                cp_async_wait<(DD - 2) / 2>();
+                {
+                    const float ca = pa[j], cb = pb[j];
+                    const float *src = ring + slot * 32 * VEC;
+#pragma unroll
+                    for (int c = 0; c < VEC; ++c) ae.v[c] = fmaf(c < split ? ca : cb, src[c], ae.v[c]);
+                }
+                if (j + 1 < n0) {
+                    const float ca = pa[j + 1], cb = pb[j + 1];
+                    const float *src = ring + (slot + 1) * 32 * VEC;
+#pragma unroll
+                    for (int c = 0; c < VEC; ++c) ao.v[c] = fmaf(c < split ? ca : cb, src[c], ao.v[c]);
+                }
+                slot += 2;
+                if (slot == DD) slot = 0;
+            }
+#else
             for (int j = 0; j < n0; ++j) {
                 const int jj = j + DD - 1;
                 const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
@@ -1065,6 +1113,7 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
                 for (int c = 0; c < VEC; ++c) ac.v[c] = fmaf(c < split ? ca : cb, src[c], ac.v[c]);
                 if (++slot == DD) slot = 0;
             }
+#endif
             __syncwarp();  // P, S are rewritten by the next chunk
             if (n1 <= 0) break;
             off += 32;
@@ -1256,6 +1305,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                     for (int c = 0; c < VEC; ++c) y.v[c] = acc.v[c] * (c < split ? iA : iB);
                     apply_layer_epilogue<VEC>(a, col, y);
                     if (active) store_out<VEC>(a, r, col, y);
+                    count_visit(a, r, lane);
                     continue;
                 } else if constexpr (ASYNC) {
                     reduce_edges_async<VEC, OP, COEF, U>(a, e0, e1, col, active, er_v, lane, acc, m, den);
@@ -1268,6 +1318,7 @@ __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0
                 }
                 Vec<VEC> y = epilogue<VEC, OP>(a, r, deg, col, active, acc, den);
                 if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
+                count_visit(a, r, lane);
                 project_row<VEC, G>(a, r, s, col, active, y, lane);
             }
         }
@@ -1403,6 +1454,7 @@ __device__ TLP_HUB_INLINE void do_hub_chunk(const AggArgs &a, int h, int j, int 
             y = epilogue<VEC, OP>(a, r, (int)(ee - eb), col, active, acc, D);
         }
         if (active && stores<G>(lane)) store_out<VEC>(a, r, col, y);
+        count_visit(a, r, lane);
         if constexpr (OP != OP_GATH) project_row<VEC, G>(a, r, s, col, active, y, lane);
     }
     if (lane == 0) *ticket = 0;  // self-reset for the next launch

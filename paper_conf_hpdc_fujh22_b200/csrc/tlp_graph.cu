@@ -731,6 +731,12 @@ tlp_status tlp_graph_build_transpose(tlp_graph g, void *stream) {
     return build_transpose(g, (cudaStream_t)stream);
 }
 
+tlp_status tlp_graph_set_visit_counter(tlp_graph g, int32_t *counter) {
+    if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
+    g->visits = counter;
+    return TLP_OK;
+}
+
 tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta, int step) {
     if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
     if (sched < TLP_SCHED_DYNAMIC || sched > TLP_SCHED_PAPER)

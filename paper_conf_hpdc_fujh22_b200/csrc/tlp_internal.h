@@ -76,6 +76,7 @@ struct tlp_graph_s {
     double create_ms = 0.0;
     int64_t launches = 0;        // kernels enqueued by calls on this handle (after create)
 
+    int32_t *visits = nullptr;   // debug visit counter (tlp_graph_set_visit_counter), borrowed
     int sched = TLP_SCHED_DYNAMIC;
     int warps_per_cta = 8;
     int step = 0;

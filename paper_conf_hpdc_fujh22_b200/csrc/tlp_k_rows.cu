@@ -180,6 +180,7 @@ __global__ void __launch_bounds__(256, TLP_ROWS_MINB) k_rows(const AggArgs a) {
         for (int c = 0; c < VEC; ++c) acc.v[c] = ac[0].v[c] + ac[1].v[c];
         Vec<VEC> y = epilogue<VEC, OP>(a, r, len, col, active, acc, den);
         if (active) store_out<VEC>(a, r, col, y);
+        count_visit(a, r, lane);
         project_row<VEC, 1>(a, r, s, col, active, y, lane);
     }
     if (a.n_dests > 0) __threadfence_system();  // peer stores visible before the barrier

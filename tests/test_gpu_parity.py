@@ -1309,3 +1309,38 @@ def test_launch_counter(tlp, monkeypatch):
     monkeypatch.setenv("TLP_GAT", "alpha")
     assert count(lambda: g.gat(X, el, er, 0.2)) == 2
     g.close()
+
+
+@pytest.mark.parametrize("mode", ["default", "panel64", "async", "rows_split", "gat_alpha", "narrow"])
+def test_visit_counter_exactly_once(tlp, monkeypatch, mode):
+    """SURVEY 4 T7 (Alg. 1's exactly-once semantics): with the debug
+    visit counter on, every row -- hub rows split into chunks included -- is
+    finished exactly once per feature strip, whatever the scheduler, gather
+    path, strip width or kernel (general, short-row with hub split)."""
+    n = 3000
+    deg = np.minimum((2500.0 / (np.arange(n) + 1) ** 0.65).astype(np.int64) + 1, 2000)
+    rp, ci = synth.power_law_rows(n, np.random.default_rng(5).permutation(deg), n, seed=6)
+    F = 32 if mode == "narrow" else 300
+    X = _t(synth.features(n, F, F, seed=3))
+    el, er = _t(synth.normal(n, 1)), _t(synth.normal(n, 2))
+    g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=90, hub_chunk=44))
+    assert g.info["n_hubs"] > 0
+    strips = {"default": 3, "panel64": 5, "async": 3, "rows_split": 3, "gat_alpha": 5, "narrow": 1}[mode]
+    env = {"panel64": {"TLP_PANEL": "64"}, "async": {"TLP_PANEL": "0", "TLP_GATHER": "async"},
+           "rows_split": {"TLP_ROWS": "1"}, "gat_alpha": {"TLP_GAT": "alpha", "TLP_PANEL": "64"}}.get(mode, {})
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    cnt = torch.zeros(n, dtype=torch.int32, device=DEV)
+    tlp.tlp_graph_set_visit_counter(g.handle, cnt)
+    ops = [lambda: g.gat(X, el, er, 0.2)] if mode == "gat_alpha" else \
+          [lambda: g.gcn(X, "both"), lambda: g.gin(X, 0.1), lambda: g.gat(X, el, er, 0.2)]
+    for sched in ("dynamic", "static", "hardware"):
+        g.set_schedule(sched)
+        for f in ops:
+            cnt.zero_()
+            f()
+            torch.cuda.synchronize()
+            c = cnt.cpu().numpy()
+            assert c.min() == strips and c.max() == strips, (mode, sched, int(c.min()), int(c.max()))
+    tlp.tlp_graph_set_visit_counter(g.handle, None)
+    g.close()
