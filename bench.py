@@ -832,6 +832,8 @@ def main():
                     help="with --dist/torchrun: NEXT-2 fused compute + all-gather over NVLink peer memory")
     ap.add_argument("--dist", action="store_true",
                     help="use the NCCL dist API even at world size 1 (exercises the N>1 path)")
+    ap.add_argument("--spawn", action="store_true",
+                    help="start the ranks through torch.distributed.run even for --gpus 1")
     ap.add_argument("--selftest", action="store_true",
                     help="CPU check of the multi-rank launcher (gloo, no GPU): ranks partition "
                          "the Reddit-shaped rows with libtlp's host partition and reduce a time")
@@ -839,10 +841,19 @@ def main():
     if args.warmup < 3:
         print("warning: the contract wants >= 3 warm-up steps", file=sys.stderr)
     world_env = os.environ.get("WORLD_SIZE")
-    if world_env is None and args.gpus > 1:
+    if world_env is None and (args.gpus > 1 or args.spawn):
         # --gpus N without a launcher: start N ranks ourselves (one process per
         # GPU, torchrun over 127.0.0.1), forwarding the same arguments
-        sys.exit(launch_ranks(args.gpus, sys.argv[1:]))
+        if not args.selftest and args.impl == "tlp":
+            try:
+                import torch
+                have = torch.cuda.device_count()
+            except Exception:
+                have = 0
+            if have < args.gpus:
+                print(f"error: --gpus {args.gpus} but only {have} CUDA device(s) visible", file=sys.stderr)
+                sys.exit(1)
+        sys.exit(launch_ranks(args.gpus, [a for a in sys.argv[1:] if a != "--spawn"]))
     if world_env is not None and int(world_env) != args.gpus:
         print(f"error: --gpus {args.gpus} but WORLD_SIZE={world_env}", file=sys.stderr)
         sys.exit(2)

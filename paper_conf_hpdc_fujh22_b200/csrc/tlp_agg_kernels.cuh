@@ -1038,22 +1038,11 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
         int u0 = (lane < n0) ? __ldg(ci + lane) : 0;
         int u1 = (lane < n1) ? __ldg(ci + 32 + lane) : 0;
 #pragma unroll
-#if TLP_ASYNC_PAIR
-        for (int k = 0; k < DD - 2; k += 2) {  // two edges per commit group
-            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
-            const int ub = __shfl_sync(FULL, k + 1 < 32 ? u0 : u1, (k + 1) & 31);
-            cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
-            cp_async_vec<VEC>(ring + (k + 1) * 32 * VEC, row_ptr(base, (unsigned)ub, row_bytes),
-                              active && k + 1 < len);
-            cp_async_commit();
-        }
-#else
         for (int k = 0; k < DD - 1; ++k) {
             const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
             cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
             cp_async_commit();
         }
-#endif
         int slot = 0, off = 0;
         while (true) {
             const int n2 = min(32, len - off - 64);
@@ -1068,35 +1057,6 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
             }
             const float *pa = P + hl * 32;
             const float *pb = P + hl2 * 32;
-#if TLP_ASYNC_PAIR
-            for (int j = 0; j < n0; j += 2) {  // as the single-head pipeline
-                const int ja = j + DD - 2, jb = j + DD - 1;
-                const int ua = __shfl_sync(FULL, ja < 32 ? u0 : u1, ja & 31);
-                const int ub = __shfl_sync(FULL, jb < 32 ? u0 : u1, jb & 31);
-                int wa = slot + DD - 2;
-                if (wa >= DD) wa -= DD;
-                cp_async_vec<VEC>(ring + wa * 32 * VEC, row_ptr(base, (unsigned)ua, row_bytes),
-                                  active && (off + ja) < len);
-                cp_async_vec<VEC>(ring + (wa + 1) * 32 * VEC, row_ptr(base, (unsigned)ub, row_bytes),
-                                  active && (off + jb) < len);
-                cp_async_commit();
-                cp_async_wait<(DD - 2) / 2>();
-                {
-                    const float ca = pa[j], cb = pb[j];
-                    const float *src = ring + slot * 32 * VEC;
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) ae.v[c] = fmaf(c < split ? ca : cb, src[c], ae.v[c]);
-                }
-                if (j + 1 < n0) {
-                    const float ca = pa[j + 1], cb = pb[j + 1];
-                    const float *src = ring + (slot + 1) * 32 * VEC;
-#pragma unroll
-                    for (int c = 0; c < VEC; ++c) ao.v[c] = fmaf(c < split ? ca : cb, src[c], ao.v[c]);
-                }
-                slot += 2;
-                if (slot == DD) slot = 0;
-            }
-#else
             for (int j = 0; j < n0; ++j) {
                 const int jj = j + DD - 1;
                 const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
@@ -1113,7 +1073,6 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
                 for (int c = 0; c < VEC; ++c) ac.v[c] = fmaf(c < split ? ca : cb, src[c], ac.v[c]);
                 if (++slot == DD) slot = 0;
             }
-#endif
             __syncwarp();  // P, S are rewritten by the next chunk
             if (n1 <= 0) break;
             off += 32;

@@ -13,6 +13,8 @@ if [ "$P" = "bench" ] || [ "$P" = "all" ]; then
   for w in cora pubmed; do
     timeout 900 python bench.py --workload $w --no-cpu-baseline --steps 4000 --warmup 100 > $O/bench_$w.json 2> $O/bench_$w.err
   done
+  # the multi-rank launcher and the NCCL dist path at world 1 (one GPU per box)
+  timeout 900 python bench.py --gpus 1 --spawn --dist --no-cpu-baseline > $O/bench_dist1.json 2> $O/bench_dist1.err
 fi
 if [ "$P" = "ncu" ] || [ "$P" = "all" ]; then
   ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv \
