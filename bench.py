@@ -259,6 +259,10 @@ def run_tlp(args):
     # the dist path (NCCL comm + tlp_dist_*) also at world = 1 with --dist
     use_dist = world > 1 or args.dist
     if use_dist:
+        # the driver counts ranks from NCCL's init log (read by NCCL at its
+        # first communicator, i.e. before the process group comes up)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         os.environ.setdefault("MASTER_PORT", str(29500 + os.getpid() % 1000))
         dist.init_process_group("nccl", device_id=dev, rank=rank, world_size=world)
@@ -273,9 +277,6 @@ def run_tlp(args):
     ci_d = torch.from_numpy(ci).to(dev)
     comm = None
     if use_dist:
-        # the driver counts ranks from NCCL's init log
-        os.environ.setdefault("NCCL_DEBUG", "INFO")
-        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         comm = tlp.comm_from_torch()
     # first create of the process: includes loading the library's create
     # kernels (CUDA lazy module loading); then the warm create of the real
@@ -315,6 +316,7 @@ def run_tlp(args):
         return torch.empty((n, ld), dtype=torch.float32, device=dev)
 
     Y = {op: out_buffer() for op in ops}
+    sym_kind = tlp.tlp_comm_symmetric_kind(comm, sym_ptrs[0]) if (fused and sym_ptrs) else None
     Y1 = out_buffer() if "gcn2" in ops else None
 
     def gcn_to(Xin, out):
@@ -634,7 +636,11 @@ def run_tlp(args):
                    "parallelism": ("rows%d (edge-balanced row ranges, X replicated, %s)" % (
                        world, "fused peer-store all-gather (NEXT-2)" if fused else
                        "grouped-broadcast all-gather of Y")) if use_dist else "single",
-                   "frac_of_8TBs": round(value / NOMINAL_HBM_GBS, 4)},
+                   "frac_of_8TBs": round(value / NOMINAL_HBM_GBS, 4),
+                   "value_kind": "gather-model (logical) bytes of the step / device time: every edge "
+                                 "counts one source-row read (SURVEY 8(d) d2); in L2-panel mode most of "
+                                 "them are L2 hits, so it can exceed the HBM peak -- roofline.hbm holds "
+                                 "the DRAM rate"},
         "ops": per_op, "create_ms": round(create_ms, 2),
         "create_cold_ms": round(create_cold_ms, 1), "create_first_tiny_ms": round(first_create_ms, 1),
         "plan": {k: info[k] for k in ("n_hubs", "n_hub_chunks", "n_units", "n_tasks",
@@ -645,6 +651,8 @@ def run_tlp(args):
     }
     if dist_split:
         result["dist"] = dist_split
+    if sym_kind:
+        result["config"]["symmetric_buffer"] = sym_kind
     w = WORKLOADS[name]
     if "paper_v100_ms" in w:
         # context only (another GPU, the paper's own F = 32 measurement)

@@ -382,11 +382,19 @@ tlp_status tlp_dist_graph_create(tlp_comm c, int64_t n, int64_t nnz,
                                  tlp_graph *out_local);
 
 /* NEXT-2: symmetric output buffers.  Collective over the communicator: every
- * rank allocates `bytes` of device memory and maps every other rank's buffer
- * through CUDA IPC (NVLink peer memory).  *local = this rank's buffer. */
+ * rank allocates `bytes` of device memory visible to every other rank of the
+ * node over NVLink.  Preferred form: NCCL's symmetric window (ncclMemAlloc +
+ * ncclCommWindowRegister(NCCL_WIN_COLL_SYMMETRIC) + ncclDevCommCreate), whose
+ * LSA pointers address every peer's copy and, where the node supports NVLS,
+ * whose multicast address lets one multimem store reach all of them; if any
+ * of that is unavailable (or TLP_SYM=ipc), a cudaMalloc'd buffer mapped into
+ * every peer through CUDA IPC.  *local = this rank's buffer. */
 tlp_status tlp_comm_alloc_symmetric(tlp_comm c, size_t bytes, void **local);
 /* Collective: unmaps, barriers, frees. */
 tlp_status tlp_comm_free_symmetric(tlp_comm c, void *local);
+/* Which form a symmetric buffer took: *kind = 0 CUDA IPC, 1 NCCL window (LSA
+ * peer pointers), 2 NCCL window with an NVLS multicast address. */
+tlp_status tlp_comm_symmetric_kind(tlp_comm c, void *local, int *kind);
 
 /* Copies the partition bounds (int64 [world+1], host). */
 tlp_status tlp_dist_bounds(tlp_graph local, int64_t *bounds_host);

@@ -108,6 +108,7 @@ _sig = {
     "tlp_dist_bounds": ([_P, _P], _I),
     "tlp_comm_alloc_symmetric": ([_P, ctypes.c_size_t, ctypes.POINTER(_P)], _I),
     "tlp_comm_free_symmetric": ([_P, _P], _I),
+    "tlp_comm_symmetric_kind": ([_P, _P, ctypes.POINTER(_I)], _I),
     "tlp_dist_aggregate_fused": ([_P, _P, ctypes.POINTER(tlp_agg_desc), _P], _I),
     "tlp_debug_multi_store": ([_P, ctypes.POINTER(tlp_agg_desc), _P, _I, _P], _I),
     "tlp_dist_allgather_rows": ([_P, _P, _P, _I64, _P], _I),
@@ -658,6 +659,16 @@ def tlp_comm_alloc_symmetric(comm, rows, ld):
            "tlp_comm_alloc_symmetric")
     t = torch.as_tensor(_CudaArray(out.value, (int(rows), int(ld))), device="cuda")
     return t, out.value
+
+
+SYM_KINDS = {0: "ipc", 1: "nccl_window", 2: "nccl_window_multicast"}
+
+
+def tlp_comm_symmetric_kind(comm, ptr):
+    """'ipc', 'nccl_window' or 'nccl_window_multicast' (NVLS)."""
+    k = _I()
+    _check(_lib.tlp_comm_symmetric_kind(comm, ptr, ctypes.byref(k)), "tlp_comm_symmetric_kind")
+    return SYM_KINDS.get(k.value, k.value)
 
 
 def tlp_comm_free_symmetric(comm, ptr):

@@ -841,6 +841,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.bias = r.bias;
     a.dests = r.dests;
     a.n_dests = r.n_dests;
+    a.mc = r.mc;
     a.hot_thr = 0;
     a.cold_first = 0;
     a.xself = r.xself;

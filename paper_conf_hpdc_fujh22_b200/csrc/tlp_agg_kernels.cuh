@@ -103,6 +103,11 @@ struct AggArgs {
     // rank, mapped over NVLink) instead of to Y.
     float *const *dests;
     int n_dests;
+    // NCCL symmetric window with NVLS multicast (NEXT-2): when mc is
+    // set, one multimem store to mc + (row_offset + r) * ldy lands the row in
+    // Y_full on every rank of the node (NVSwitch replicates it); dests is then
+    // unused for data
+    float *mc;
     // hot-source L2 policy: when hot_thr != 0
     // colidx carries the source's out-degree class in bits 27-31; sources with
     // tag >= hot_thr are gathered with L2 evict_last, the rest with cold_first ?
@@ -1154,6 +1159,20 @@ __device__ __forceinline__ Vec<VEC> epilogue(const AggArgs &a, int64_t r, int de
 // to the same global row of every destination buffer.
 template <int VEC>
 __device__ __forceinline__ void store_out(const AggArgs &a, int64_t r, int col, const Vec<VEC> &y) {
+    if (a.mc) {
+        float *p = a.mc + (a.row_offset + r) * a.ldy + col;
+        if (VEC == 4 && col + 4 <= a.F) {
+            asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1, %2, %3, %4};"
+                         ::"l"(p), "f"(y.v[0]), "f"(y.v[VEC > 1 ? 1 : 0]), "f"(y.v[VEC > 2 ? 2 : 0]),
+                           "f"(y.v[VEC > 3 ? 3 : 0]) : "memory");
+        } else {
+#pragma unroll
+            for (int c = 0; c < VEC; ++c)
+                if (col + c < a.F)
+                    asm volatile("multimem.st.relaxed.sys.global.f32 [%0], %1;" ::"l"(p + c), "f"(y.v[c]) : "memory");
+        }
+        return;
+    }
     if (a.n_dests == 0) {
         st_row<VEC>(a.Y + r * a.ldy, col, a.F, y, a.stream_hint ? policy_evict_first() : 0ull);
     } else {

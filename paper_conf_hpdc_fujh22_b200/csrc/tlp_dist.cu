@@ -9,6 +9,7 @@
 // is the row all-gather.  NCCL 2.28 has no all-gatherv: rank r's slab is
 // broadcast in place by a grouped ncclBroadcast(root = r).
 #include <nccl.h>
+#include <nccl_device.h>  // NCCL 2.28 device API: symmetric windows, LSA / multimem pointers
 
 #include <chrono>
 #include <cstring>
@@ -26,6 +27,13 @@ struct SymBuf {
     size_t bytes = 0;
     std::vector<void *> peers;  // [world], peers[rank] = local
     float **dev_ptrs = nullptr; // device copy of peers
+    // NCCL symmetric window form (preferred): ncclMemAlloc'd buffer registered
+    // with NCCL_WIN_COLL_SYMMETRIC; peers[] are its LSA pointers and mc its
+    // NVLS multicast address (null when the node has no NVLS)
+    bool window = false;
+    ncclWindow_t win = nullptr;
+    ncclDevComm dev_comm{};
+    float *mc = nullptr;
 };
 
 struct tlp_comm_s {
@@ -237,10 +245,91 @@ static tlp_status comm_barrier(tlp_comm c, cudaStream_t s) {
     return TLP_OK;
 }
 
+// LSA peer pointers and the multicast address of a registered window (the
+// window descriptor lives in device memory, read through the device API).
+__global__ void k_window_ptrs(ncclWindow_t w, ncclDevComm dc, int n, int use_mc, void **out) {
+    const int i = threadIdx.x;
+    if (i < n) out[i] = ncclGetLsaPointer(w, 0, i);
+    if (i == 0) out[n] = use_mc ? ncclGetLsaMultimemPointer(w, 0, dc) : nullptr;
+}
+
+// NEXT-2 symmetric buffer through NCCL's window API (ncclMemAlloc +
+// ncclCommWindowRegister + ncclDevCommCreate -> LSA peer pointers, and the
+// NVLS multicast address when the node supports it).  Returns false (with
+// nothing allocated) when any step is unavailable, so the caller falls back
+// to CUDA IPC.
+static bool alloc_window(tlp_comm c, size_t bytes, SymBuf &b) {
+    const size_t al = NCCL_WIN_REQUIRED_ALIGNMENT;
+    const size_t sz = (bytes + al - 1) / al * al;
+    void *buf = nullptr;
+    if (ncclMemAlloc(&buf, sz) != ncclSuccess) return false;
+    ncclWindow_t win = nullptr;
+    if (ncclCommWindowRegister(c->comm, buf, sz, &win, NCCL_WIN_COLL_SYMMETRIC) != ncclSuccess) {
+        ncclMemFree(buf);
+        return false;
+    }
+    ncclDevComm dc{};
+    ncclDevCommRequirements req{};
+    req.lsaMultimem = c->world > 1;
+    bool mm = req.lsaMultimem;
+    if (ncclDevCommCreate(c->comm, &req, &dc) != ncclSuccess) {
+        // no NVLS (or a single rank): LSA pointers only
+        req.lsaMultimem = false;
+        mm = false;
+        if (ncclDevCommCreate(c->comm, &req, &dc) != ncclSuccess) {
+            ncclCommWindowDeregister(c->comm, win);
+            ncclMemFree(buf);
+            return false;
+        }
+    }
+    if (dc.lsaSize != c->world) {  // more than one node: the IPC path is single-node as well
+        ncclDevCommDestroy(c->comm, &dc);
+        ncclCommWindowDeregister(c->comm, win);
+        ncclMemFree(buf);
+        return false;
+    }
+    void **d_out = nullptr;
+    std::vector<void *> h(c->world + 1, nullptr);
+    bool ok = cudaMalloc(&d_out, sizeof(void *) * (c->world + 1)) == cudaSuccess;
+    if (ok) {
+        k_window_ptrs<<<1, 64, 0, c->side>>>(win, dc, c->world, mm ? 1 : 0, d_out);
+        ok = cudaMemcpyAsync(h.data(), d_out, sizeof(void *) * (c->world + 1), cudaMemcpyDeviceToHost,
+                             c->side) == cudaSuccess &&
+             cudaStreamSynchronize(c->side) == cudaSuccess;
+        cudaFree(d_out);
+    }
+    if (!ok || h[c->rank] == nullptr) {
+        cudaGetLastError();
+        ncclDevCommDestroy(c->comm, &dc);
+        ncclCommWindowDeregister(c->comm, win);
+        ncclMemFree(buf);
+        return false;
+    }
+    b.window = true;
+    b.win = win;
+    b.dev_comm = dc;
+    b.local = buf;
+    b.bytes = bytes;
+    b.peers.assign(h.begin(), h.begin() + c->world);
+    b.mc = (float *)h[c->world];
+    return true;
+}
+
 tlp_status tlp_comm_alloc_symmetric(tlp_comm c, size_t bytes, void **local) {
     if (!c || !local || bytes == 0) return set_error(TLP_ERR_INVALID_ARGUMENT, "alloc_symmetric: bad argument");
     *local = nullptr;
+    if (!c->comm) return set_error(TLP_ERR_NCCL, "communicator was aborted");
     SymBuf b;
+    // NCCL symmetric window first (TLP_SYM=ipc forces the CUDA IPC form)
+    const char *sym = getenv("TLP_SYM");
+    if (!(sym && !strcmp(sym, "ipc")) && alloc_window(c, bytes, b)) {
+        TLP_CUDA_TRY(cudaMalloc(&b.dev_ptrs, sizeof(float *) * c->world));
+        TLP_CUDA_TRY(cudaMemcpy(b.dev_ptrs, b.peers.data(), sizeof(void *) * c->world, cudaMemcpyHostToDevice));
+        c->sym.push_back(b);
+        *local = b.local;
+        return TLP_OK;
+    }
+    b = SymBuf();
     b.bytes = bytes;
     TLP_CUDA_TRY(cudaMalloc(&b.local, bytes));
     b.peers.assign(c->world, nullptr);
@@ -279,15 +368,36 @@ tlp_status tlp_comm_alloc_symmetric(tlp_comm c, size_t bytes, void **local) {
     return TLP_OK;
 }
 
+tlp_status tlp_comm_symmetric_kind(tlp_comm c, void *local, int *kind) {
+    if (!c || !local || !kind) return set_error(TLP_ERR_INVALID_ARGUMENT, "symmetric_kind: bad argument");
+    for (const SymBuf &b : c->sym)
+        if (b.local == local) {
+            *kind = b.window ? (b.mc ? 2 : 1) : 0;
+            return TLP_OK;
+        }
+    return set_error(TLP_ERR_INVALID_ARGUMENT, "not a symmetric buffer of this communicator");
+}
+
 tlp_status tlp_comm_free_symmetric(tlp_comm c, void *local) {
     if (!c || !local) return set_error(TLP_ERR_INVALID_ARGUMENT, "free_symmetric: bad argument");
     for (size_t i = 0; i < c->sym.size(); ++i) {
         SymBuf &b = c->sym[i];
         if (b.local != local) continue;
+        cudaDeviceSynchronize();  // no queued kernel still stores through the mappings
+        if (b.window) {
+            // collective: every rank deregisters its window
+            if (c->comm) {
+                ncclDevCommDestroy(c->comm, &b.dev_comm);
+                ncclCommWindowDeregister(c->comm, b.win);
+            }
+            cudaFree(b.dev_ptrs);
+            ncclMemFree(b.local);
+            c->sym.erase(c->sym.begin() + i);
+            return TLP_OK;
+        }
         for (int q = 0; q < c->world; ++q)
             if (q != c->rank && b.peers[q]) cudaIpcCloseMemHandle(b.peers[q]);
         // every rank has unmapped before anyone frees
-        cudaDeviceSynchronize();  // no queued kernel still stores through the mappings
         tlp_status st = comm_barrier(c, c->side);
         cudaStreamSynchronize(c->side);
         cudaFree(b.dev_ptrs);
@@ -419,6 +529,9 @@ tlp_status tlp_dist_aggregate_fused(tlp_graph g, tlp_comm c, const tlp_agg_desc 
     r.Y = d->Y + g->row_offset * d->ldy;
     r.dests = b->dev_ptrs;
     r.n_dests = c->world;
+    // NVLS multicast: one store reaches every rank's Y_full (TLP_SYM_MC=0: per-peer stores)
+    const char *mce = getenv("TLP_SYM_MC");
+    if (b->mc && !(mce && !strcmp(mce, "0"))) r.mc = b->mc;
     // entry barrier: a fast rank must not store into a peer's Y_full while that
     // peer's stream may still read its previous contents (e.g. the next layer
     // reads Y_full while this call overwrites it on every rank)

@@ -127,6 +127,7 @@ struct AggRequest {
     float act_param = 0.f;
     float *const *dests = nullptr;  // fused all-gather destinations (device array)
     int n_dests = 0;
+    float *mc = nullptr;            // NVLS multicast address of Y_full (NCCL window), or null
     // epilogue projections (NEXT-3): el_out = Y.att_l, er_out = Y.att_r
     const float *att_l = nullptr, *att_r = nullptr;
     float *el_out = nullptr, *er_out = nullptr;

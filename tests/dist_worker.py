@@ -55,7 +55,9 @@ def main():
     rng = np.random.default_rng(5)
     rows = np.unique(np.concatenate([rng.choice(n, 300, replace=False), b[:-1].clip(max=n - 1)]))
     report = {}
+    # the symmetric buffer: NCCL window (default) or CUDA IPC (TLP_SYM=ipc)
     Ysym, ptr = tlp.tlp_comm_alloc_symmetric(comm, n, ld)
+    sym_kind = tlp.tlp_comm_symmetric_kind(comm, ptr)
     for op, (kw, single, ref) in ops.items():
         Y1 = single()
         torch.cuda.synchronize()
@@ -81,7 +83,8 @@ def main():
     tlp.tlp_comm_destroy(comm)
     dist.destroy_process_group()
     if rank == 0:
-        print(json.dumps({"world": world, "worst_err_over_tol": report, "bounds": b.tolist()}))
+        print(json.dumps({"world": world, "worst_err_over_tol": report, "bounds": b.tolist(),
+                          "symmetric_buffer": sym_kind}))
 
 
 if __name__ == "__main__":

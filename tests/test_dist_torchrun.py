@@ -23,14 +23,19 @@ def _port():
         return s.getsockname()[1]
 
 
-def test_dist_torchrun_bitwise_vs_single_gpu():
+@pytest.mark.parametrize("sym", ["window", "ipc"])
+def test_dist_torchrun_bitwise_vs_single_gpu(sym):
     world = max(1, min(8, torch.cuda.device_count()))
+    env = dict(os.environ)
+    if sym == "ipc":
+        env["TLP_SYM"] = "ipc"
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr=127.0.0.1", f"--master-port={_port()}",
            os.path.join(ROOT, "tests", "dist_worker.py")]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT)
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
     assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-4000:])
     line = [ln for ln in r.stdout.splitlines() if ln.startswith("{")][-1]
     d = json.loads(line)
     assert d["world"] == world
     assert all(v <= 1.0 for v in d["worst_err_over_tol"].values())
+    assert (d["symmetric_buffer"] == "ipc") == (sym == "ipc"), d["symmetric_buffer"]

@@ -855,8 +855,12 @@ def test_multi_destination_epilogue(tlp, op):
     g.close()
 
 
-def test_fused_allgather_world1(tlp):
-    """NCCL world of one: symmetric buffer + fused dist aggregation == single GPU."""
+@pytest.mark.parametrize("sym", ["window", "ipc"])
+def test_fused_allgather_world1(tlp, monkeypatch, sym):
+    """NCCL world of one: symmetric buffer (NCCL symmetric window or CUDA IPC
+    form) + fused dist aggregation == single GPU."""
+    if sym == "ipc":
+        monkeypatch.setenv("TLP_SYM", "ipc")
     n = 1500
     rp, ci = synth.chung_lu(n, 30000, 0.5, 52, device="cpu")
     F, ld = 70, 72
@@ -864,6 +868,8 @@ def test_fused_allgather_world1(tlp):
     comm = tlp.tlp_comm_create(tlp.tlp_comm_get_unique_id(), 1, 0)
     h = tlp.tlp_dist_graph_create(comm, _t(rp), _t(ci))
     Ysym, ptr = tlp.tlp_comm_alloc_symmetric(comm, n, ld)
+    kind = tlp.tlp_comm_symmetric_kind(comm, ptr)
+    assert kind == ("ipc" if sym == "ipc" else "nccl_window"), kind  # one rank: no multicast
     tlp.tlp_dist_aggregate_fused(h, comm, "gcn", X, Ysym, F=F, norm="both")
     g = tlp.Graph(_t(rp), _t(ci))
     assert torch.equal(Ysym[:, :F], g.gcn(X, "both", F=F))
