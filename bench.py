@@ -602,9 +602,17 @@ def run_tlp(args):
                                   "dram__bytes_write.sum per launch, ncu --set full of this round's kernels)"}
     probe = None
     if panel and rank == 0:
+        # ~30 probe runs (~0.1 s) so the clock sampler sees them; the best run is the ceiling
+        runs = []
         with ClockSampler(local) as pclk:
-            probe = l2_gather_ceiling(n * 256)
-        if probe:
+            for _ in range(30):
+                r_ = l2_gather_ceiling(n * 256)
+                if r_:
+                    runs.append(r_)
+        if runs:
+            probe = max(runs, key=lambda r_: r_["GBs"])
+            probe["median_GBs"] = round(statistics.median(r_["GBs"] for r_ in runs), 1)
+            probe["runs"] = len(runs)
             probe["clocks"] = pclk.summary()
     if probe:
         roofline.update({"bound": "l2", "peak": probe["GBs"], "frac": round(achieved / probe["GBs"], 4),
