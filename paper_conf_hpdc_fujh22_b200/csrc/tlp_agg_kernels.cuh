@@ -1239,23 +1239,38 @@ __device__ __forceinline__ void gatb_self(const AggArgs &a, int64_t r, int s, in
     }
 }
 
+// Per-warp shared-memory copy of the row offsets (and GAT's er) of the rows a
+// unit walks: they stay out of the registers while the edge loop runs (the
+// edge loop is what the 64-register budget is for; round 2: row-level spills
+// -> shared memory).
+__device__ __forceinline__ int64_t *warp_rowptr_smem() {
+    __shared__ int64_t tlp_rp[TLP_MAXT / 32][32];
+    return tlp_rp[threadIdx.x >> 5];
+}
+__device__ __forceinline__ float *warp_er_smem() {
+    __shared__ float tlp_er[TLP_MAXT / 32][32];
+    return tlp_er[threadIdx.x >> 5];
+}
+
 // A regular work unit: whole rows [r0, r1), feature strips [s0, s1).
 template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void do_unit(const AggArgs &a, int r0, int r1, int s0, int s1,
                                         int lane) {
+    int64_t *rps = warp_rowptr_smem();
+    float *ers = warp_er_smem();
     for (int rb = r0; rb < r1; rb += 31) {
         const int nr = min(31, r1 - rb);
         // lanes fetch the row offsets of up to 31 rows at once (register caching
-        // of the index boundary, Fig. 7a)
-        int64_t rp = 0;
-        if (lane <= nr) rp = __ldg(a.rowptr + rb + lane);
-        float erl = 0.f;
+        // of the index boundary, Fig. 7a), parked in shared memory
+        __syncwarp();  // the previous block's offsets are consumed
+        if (lane <= nr) rps[lane] = __ldg(a.rowptr + rb + lane);
         if constexpr (OP == OP_GAT)
-            if (lane < nr) erl = __ldg(a.er + a.row_offset + rb + lane);
+            if (lane < nr) ers[lane] = __ldg(a.er + a.row_offset + rb + lane);
+        __syncwarp();
         for (int k = 0; k < nr; ++k) {
-            const int64_t e0 = __shfl_sync(FULL, rp, k);
-            const int64_t e1 = __shfl_sync(FULL, rp, k + 1);
-            const float er_v = (OP == OP_GAT) ? __shfl_sync(FULL, erl, k) : 0.f;
+            const int64_t e0 = rps[k];
+            const int64_t e1 = rps[k + 1];
+            const float er_v = (OP == OP_GAT) ? ers[k] : 0.f;
             const int r = rb + k;
             const int deg = (int)(e1 - e0);
             for (int s = s0; s < s1; ++s) {
