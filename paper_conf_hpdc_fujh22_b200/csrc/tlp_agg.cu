@@ -55,12 +55,16 @@ static int occupancy_blocks(KernelFn fn, int threads, size_t smem) {
         if (cache[i].fn == fn && cache[i].threads == threads && cache[i].smem == smem)
             return cache[i].blocks;
     if (smem > 0) {
-        // opt in to the device maximum once per kernel (never lowered afterwards)
+        // opt in to the device maximum once per kernel (never lowered afterwards):
+        // the opt-in limit covers static + dynamic shared memory
         int dev = 0, mx = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&mx, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, mx);
-        cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+        cudaFuncAttributes fa;
+        if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) mx -= (int)fa.sharedSizeBytes;
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, mx) != cudaSuccess ||
+            cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, 100) != cudaSuccess)
+            cudaGetLastError();  // the launch reports it if the request does not fit
     }
     int nb = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, smem) != cudaSuccess || nb < 1)
@@ -1013,6 +1017,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
                   knob("TLP_PANEL") == nullptr && knob("TLP_GATHER") == nullptr;
     if (const char *e = knob("TLP_ROWS")) rows_k = rows_ok && atoi(e) != 0;
     KernelFn fr = rows_k ? pick_rows(op, coef, a.hot_thr != 0) : nullptr;
+
     if (fr) {
         const int nstr = (int)((r.F + 127) / 128);
         if (g->n_hubs > 0) {  // hub chunks in the general kernel (tasks [0, n_chunks))
