@@ -955,7 +955,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     if (groups > 1 || r.op == OP_GATB) async_path = false;  // OP_GATB: register path only
     const int path = groups > 1 ? 2 : (async_path ? 1 : 0);
     // hot-source L2 policy: cp.async path only (rows streamed from HBM)
-    if (async_path && r.op != OP_GATH && r.op != OP_GATB) {
+    if (async_path && r.op != OP_GATB) {
         unsigned thr = 0;
         tlp_status st = hot_threshold(g, panel ? (int64_t)strip_w : r.ldx, panel != 0, s, &thr);
         if (st != TLP_OK) return st;
@@ -974,8 +974,13 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;
     size_t smem = async_path ? (size_t)wpc * TLP_DEPTH * 32 * vec * sizeof(float) : 0;
-    if (r.op == OP_GATH)
-        smem = (size_t)wpc * (kMhWarpFloats + (async_path ? TLP_DEPTH * 32 * vec : 0)) * sizeof(float);
+    if (r.op == OP_GATH) {
+        // heads a 32*vec-column strip can touch: ceil((W - 1) / fh) + 1, at most H
+        const int W = 32 * vec;
+        a.mh_nh = std::min((int)r.heads, (W - 1 + fh - 1) / fh + 1);
+        a.mh_words = (a.mh_nh * 32 + 3 * a.mh_nh + 1 + 3) & ~3;
+        smem = (size_t)wpc * (a.mh_words + (async_path ? TLP_DEPTH * 32 * vec : 0)) * sizeof(float);
+    }
     // the general persistent kernel over a.n_items work items
     auto launch_general = [&](const AggArgs &ag) -> tlp_status {
         if (smem > 0 && sched == S_HARDWARE) occupancy_blocks(fn, threads, smem);  // sets attributes

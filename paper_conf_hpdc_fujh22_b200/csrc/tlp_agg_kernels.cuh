@@ -68,6 +68,9 @@ constexpr unsigned FULL = 0xffffffffu;
 #ifndef TLP_MINB_LIGHT
 #define TLP_MINB_LIGHT 4  // register path, no edge coefficient (GIN, SAGE): <= 64 registers, 32 warps/SM
 #endif
+#ifndef TLP_MINB_MH_ASYNC
+#define TLP_MINB_MH_ASYNC 2  // multi-head async path: per-head softmax state needs ~100 registers
+#endif
 #ifndef TLP_MINB_ASYNC
 #define TLP_MINB_ASYNC 3  // async path: 3 CTAs/SM (ring = 3 x 64 KB of shared memory)
 #endif
@@ -98,6 +101,7 @@ struct AggArgs {
     int act;
     float act_param;
     int heads, fh;  // OP_GATH: H heads of fh columns each (F = heads * fh)
+    int mh_nh, mh_words;  // OP_GATH: heads one strip can touch; per-warp head-block floats
     // NEXT-2 fused all-gather: when n_dests > 0 every output row is stored to
     // dests[i] + (row_offset + r) * ldy for each destination (the Y_full of every
     // rank, mapped over NVLink) instead of to Y.
@@ -157,18 +161,25 @@ __device__ __forceinline__ void count_visit(const AggArgs &a, int64_t r, int lan
 constexpr unsigned kIdxMask = (1u << 27) - 1u;
 
 // Per-thread L2 policies for tagged gathers (createpolicy once per task).
+// mask: the index bits of a colidx entry (kIdxMask when the entries carry tags,
+// else all 32 bits: untagged graphs may have 2^27 or more source vertices).
 struct GPol {
-    unsigned thr;
+    unsigned thr, mask;
     unsigned long long hot, cold;
 };
 __device__ __forceinline__ GPol make_gpol(const AggArgs &a) {
     GPol g;
     g.thr = a.hot_thr;
-    g.hot = g.cold = 0;
+    g.mask = g.thr ? kIdxMask : 0xffffffffu;
     if (g.thr) {
         asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(g.hot));
         if (a.cold_first) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(g.cold));
         else asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(g.cold));
+    } else {
+        // untagged: every gather takes the default (evict_normal) policy, so the
+        // copy is one instruction form whether or not the graph is tagged
+        asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(g.hot));
+        g.cold = g.hot;
     }
     return g;
 }
@@ -628,21 +639,39 @@ __device__ __forceinline__ void cp_async_vec(float *dst_smem, const float *src, 
     else
         asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(d), "l"(src), "r"(bytes));
 }
-// cp.async of source row u (possibly tagged) with the hot/cold L2 policy.
+// cp.async of source row u (possibly tagged) with the hot/cold L2 policy into
+// the shared-space address dst (a 32-bit offset: no generic-to-shared
+// conversion per copy).
 template <int VEC>
-__device__ __forceinline__ void cp_async_x(float *dst_smem, const char *base, unsigned u,
+__device__ __forceinline__ void cp_async_x(unsigned dst, const char *base, unsigned u,
                                            unsigned row_bytes, const GPol &gp, bool pred) {
     const float *src = reinterpret_cast<const float *>(
-        base + (unsigned long long)(u & kIdxMask) * row_bytes);
-    if (gp.thr == 0 || VEC != 4) {
-        cp_async_vec<VEC>(dst_smem, src, pred);
-        return;
+        base + (unsigned long long)(u & gp.mask) * row_bytes);
+    if constexpr (VEC == 4) {
+        // two predicated forms with loop-invariant policies (no per-copy policy
+        // select into a uniform register); ignore-src (!pred) zero-fills
+        asm volatile("{\n\t.reg .pred pi, ph;\n\t"
+                     "setp.eq.u32 pi, %2, 0;\n\t"
+                     "setp.ge.u32 ph, %3, %4;\n\t"
+                     "@ph cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, pi, %5;\n\t"
+                     "@!ph cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, pi, %6;\n\t}\n"
+                     ::"r"(dst), "l"(src), "r"((unsigned)pred), "r"(u), "r"(gp.thr), "l"(gp.hot), "l"(gp.cold));
+    } else {
+        const int bytes = pred ? 4 * VEC : 0;  // src-size 0 => zero fill, no global read
+        if constexpr (VEC == 2)
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(dst), "l"(src), "r"(bytes));
+        else
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(dst), "l"(src), "r"(bytes));
     }
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
-    const int bytes = pred ? 16 : 0;
-    const unsigned long long pol = u >= gp.thr ? gp.hot : gp.cold;
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;\n"
-                 ::"r"(d), "l"(src), "r"(bytes), "l"(pol));
+}
+// Lane l gets the index of edge l + K of the 64 held in (u0, u1): u0[l + K]
+// while l + K < 32, else u1[l + K - 32] (two shuffles and a select per chunk
+// instead of a select per issued edge).
+template <int K>
+__device__ __forceinline__ int ahead_index(int u0, int u1, int lane) {
+    const int a0 = __shfl_sync(FULL, u0, (lane + K) & 31);
+    const int a1 = __shfl_sync(FULL, u1, (lane + K) & 31);
+    return lane + K < 32 ? a0 : a1;
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 template <int N>
@@ -693,6 +722,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
     for (int c = 0; c < VEC; ++c) ae.v[c] = ao.v[c] = 0.f;
     if (len > 0) {
         float *ring = warp_ring<VEC>() + lane * VEC;
+        const unsigned ring_s = (unsigned)__cvta_generic_to_shared(ring);
         int off = 0;
         int n0 = min(32, len);
         int n1 = min(32, len - 32);
@@ -707,7 +737,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
             if constexpr (COEF & COEF_W) w1 = ld_stream(wp + 32 + lane);
         }
         if constexpr (DEP)
-            if (lane < n0) d0 = __ldg(dep + (u0 & kIdxMask));
+            if (lane < n0) d0 = __ldg(dep + (u0 & gp.mask));
         if (len < D) {
             // short row (R-MAT / products have many): its rows go into ring
             // slots 0 .. len-1 under ONE commit group and one wait, instead of
@@ -715,7 +745,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
             // (same values, same order: bitwise the pipelined result)
             for (int k = 0; k < len; ++k) {
                 const int uk = __shfl_sync(FULL, u0, k);
-                cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active);
+                cp_async_x<VEC>(ring_s + 4u * k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active);
             }
             cp_async_commit();
             float c_l = 1.f;
@@ -757,8 +787,8 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
         for (int k = 0; k < D - 2; k += 2) {
             const int ua = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
             const int ub = __shfl_sync(FULL, k + 1 < 32 ? u0 : u1, (k + 1) & 31);
-            cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && k < len);
-            cp_async_x<VEC>(ring + (k + 1) * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && k + 1 < len);
+            cp_async_x<VEC>(ring_s + 4u * k * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && k < len);
+            cp_async_x<VEC>(ring_s + 4u * (k + 1) * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && k + 1 < len);
             cp_async_commit();
         }
 #else
@@ -766,7 +796,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
 #pragma unroll
         for (int k = 0; k < D - 1; ++k) {
             const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
-            cp_async_x<VEC>(ring + k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active && k < len);
+            cp_async_x<VEC>(ring_s + 4u * k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active && k < len);
             cp_async_commit();
         }
 #endif
@@ -780,7 +810,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
                 if constexpr (COEF & COEF_W) w2 = ld_stream(wp + off + 64 + lane);
             }
             if constexpr (DEP)
-                if (lane < n1) d1 = __ldg(dep + (u1 & kIdxMask));
+                if (lane < n1) d1 = __ldg(dep + (u1 & gp.mask));
             float c_l = 1.f;
             if constexpr (OP == OP_GAT) {
                 float s = -INFINITY;
@@ -806,19 +836,22 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
             // edges in pairs: one commit group and one wait per two edges; the
             // pair's first edge is at an even position (chunks start at even
             // offsets), so it feeds the even chain and the second the odd one
+            // uq: lane l holds the index of edge l + D - 2 of this chunk (or of
+            // the next chunk past its end), so the loop's two shuffles need no select
+            const int uq = ahead_index<D - 2>(u0, u1, lane);
             for (int j = 0; j < n0; j += 2) {
                 const int ja = j + D - 2, jb = j + D - 1;  // in this chunk or the next one
-                const int ua = __shfl_sync(FULL, ja < 32 ? u0 : u1, ja & 31);
-                const int ub = __shfl_sync(FULL, jb < 32 ? u0 : u1, jb & 31);
+                const int ua = __shfl_sync(FULL, uq, j);
+                const int ub = __shfl_sync(FULL, uq, j + 1);
                 int wa = slot + D - 2;
                 if (wa >= D) wa -= D;
                 const int wb = wa + 1;  // slot and D are even
-                cp_async_x<VEC>(ring + wa * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && (off + ja) < len);
-                cp_async_x<VEC>(ring + wb * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && (off + jb) < len);
+                cp_async_x<VEC>(ring_s + 4u * wa * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && (off + ja) < len);
+                cp_async_x<VEC>(ring_s + 4u * wb * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && (off + jb) < len);
                 cp_async_commit();
                 cp_async_wait<(D - 2) / 2>();
                 const float ca = __shfl_sync(FULL, c_l, j);
-                const float cb = __shfl_sync(FULL, c_l, min(j + 1, 31));
+                const float cb = __shfl_sync(FULL, c_l, j + 1);  // lane j+1 mod 32: unused past n0
                 acc_from_smem<VEC, HASC>(ring + slot * 32 * VEC, ca, ae);
                 if (j + 1 < n0) acc_from_smem<VEC, HASC>(ring + (slot + 1) * 32 * VEC, cb, ao);
                 slot += 2;
@@ -832,7 +865,7 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
                 const bool valid = (off + jj) < len;
                 int ws = slot + D - 1;
                 if (ws >= D) ws -= D;
-                cp_async_x<VEC>(ring + ws * 32 * VEC, base, (unsigned)ui, row_bytes, gp, active && valid);
+                cp_async_x<VEC>(ring_s + 4u * ws * 32 * VEC, base, (unsigned)ui, row_bytes, gp, active && valid);
                 cp_async_commit();
                 cp_async_wait<D - 1>();
                 const float cj = __shfl_sync(FULL, c_l, j);
@@ -863,29 +896,41 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
 // rescale S) and the weights p[j], kept in a per-warp shared-memory block;
 // each lane then gathers with the weights of its own head.  Scores never
 // leave the SM.  Reduction order: the canonical two chains per head.
-constexpr int kMhMaxHeads = 33;  // heads one strip can touch (fh >= VEC)
-constexpr int kMhWarpFloats = kMhMaxHeads * 32 + 3 * kMhMaxHeads + 1;  // P, M, D, S (+pad)
-
-__device__ __forceinline__ float *mh_warp_smem() {
+// The per-warp head block (P, M, D, S) is sized at launch for the heads a
+// strip can actually touch (a.mh_nh <= 33 for fh >= VEC; a.mh_words floats,
+// a multiple of 4), so few heads leave room for more resident CTAs.
+__device__ __forceinline__ float *mh_warp_smem(const AggArgs &a) {
     extern __shared__ __align__(16) float tlp_smem[];
-    return tlp_smem + (size_t)(threadIdx.x >> 5) * kMhWarpFloats;
+    return tlp_smem + (size_t)(threadIdx.x >> 5) * a.mh_words;
+}
+
+// The el values of one chunk's sources for the first TLP_MHB heads of a strip
+// (lane j: source u_l of edge j), loaded ahead of the chunk's scoring so the
+// dependent gather overlaps the previous chunk's row gathers.
+__device__ __forceinline__ void mh_load_el(const AggArgs &a, unsigned u_l, int n0, int h_lo, int nh,
+                                           int lane, float (&v)[TLP_MHB]) {
+    const float *__restrict__ elu = a.el + (size_t)u_l * a.heads + h_lo;
+#pragma unroll
+    for (int k = 0; k < TLP_MHB; ++k) v[k] = (k < nh && lane < n0) ? __ldg(elu + k) : 0.f;
 }
 
 // Scores, online-softmax update and weights of one 32-edge chunk for the heads
 // [h_lo, h_lo+nh) of a strip (lane j holds edge j with source u_l).  Heads are
-// processed TLP_MHB at a time so their el loads and warp reductions overlap.
-__device__ __forceinline__ void mh_chunk_scores(const AggArgs &a, int u_l, int n0, int H, int h_lo,
-                                                int nh, const float *__restrict__ erv, int lane,
-                                                float *P, float *M, float *D, float *S) {
+// processed TLP_MHB at a time so their el loads and warp reductions overlap;
+// the first block's el / er values come in el0 / er0.
+__device__ __forceinline__ void mh_chunk_scores(const AggArgs &a, unsigned u_l, int n0, int H, int h_lo,
+                                                int nh, const float *__restrict__ erv,
+                                                const float (&el0)[TLP_MHB], const float (&er0)[TLP_MHB],
+                                                int lane, float *P, float *M, float *D, float *S) {
     constexpr int B = TLP_MHB;
-    const float *__restrict__ elu = a.el + (size_t)((unsigned)u_l) * H + h_lo;
+    const float *__restrict__ elu = a.el + (size_t)u_l * H + h_lo;
     for (int hb = 0; hb < nh; hb += B) {
         float sv[B], mo[B], mn[B], sm[B];
 #pragma unroll
         for (int k = 0; k < B; ++k) {
             sv[k] = -INFINITY;
             if (hb + k < nh && lane < n0) {
-                const float t = __ldg(elu + hb + k) + __ldg(erv + hb + k);
+                const float t = hb == 0 ? el0[k] + er0[k] : __ldg(elu + hb + k) + __ldg(erv + hb + k);
                 sv[k] = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
             }
         }
@@ -921,10 +966,10 @@ __device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, in
                                                 int col, bool active, int64_t rglob, int lane,
                                                 Vec<VEC> &acc, float *&Mh, float *&Dh, int &h_lo,
                                                 int &nh, int &hl, int &split) {
-    float *P = mh_warp_smem();
-    float *M = P + kMhMaxHeads * 32;
-    float *D = M + kMhMaxHeads;
-    float *S = D + kMhMaxHeads;
+    float *P = mh_warp_smem(a);
+    float *M = P + a.mh_nh * 32;
+    float *D = M + a.mh_nh;
+    float *S = D + a.mh_nh;
     Mh = M;
     Dh = D;
     const int H = a.heads, fh = a.fh;
@@ -945,6 +990,9 @@ __device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, in
     const unsigned row_bytes = (unsigned)a.ldx * 4u;
     const int32_t *__restrict__ ci = a.colidx + e0;
     const float *__restrict__ erv = a.er + rglob * H + h_lo;
+    float er0[TLP_MHB];
+#pragma unroll
+    for (int k = 0; k < TLP_MHB; ++k) er0[k] = k < nh ? __ldg(erv + k) : 0.f;
     const int len = (int)(e1 - e0);
     Vec<VEC> ac[2];
 #pragma unroll
@@ -952,7 +1000,9 @@ __device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, in
     for (int off = 0; off < len; off += 32) {
         const int n0 = min(32, len - off);
         const int u_l = (lane < n0) ? __ldg(ci + off + lane) : 0;
-        mh_chunk_scores(a, u_l, n0, H, h_lo, nh, erv, lane, P, M, D, S);
+        float el0[TLP_MHB];
+        mh_load_el(a, (unsigned)u_l, n0, h_lo, nh, lane, el0);
+        mh_chunk_scores(a, (unsigned)u_l, n0, H, h_lo, nh, erv, el0, er0, lane, P, M, D, S);
         const float sA = S[hl], sB = S[hl2];
 #pragma unroll
         for (int c = 0; c < VEC; ++c) {
@@ -990,16 +1040,29 @@ __device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, in
 // Multi-head GAT with the cp.async ring (gathers that stream from HBM): the
 // per-warp shared memory holds the head block followed by a D-deep ring.
 template <int VEC>
-__device__ __forceinline__ float *mh_warp_ring() {
+__device__ __forceinline__ float *mh_warp_smem_async(const AggArgs &a) {
     extern __shared__ __align__(16) float tlp_smem[];
-    constexpr int stride = kMhWarpFloats + TLP_DEPTH * 32 * VEC;
-    return tlp_smem + (size_t)(threadIdx.x >> 5) * stride + kMhWarpFloats;
-}
-template <int VEC>
-__device__ __forceinline__ float *mh_warp_smem_async() {
-    extern __shared__ __align__(16) float tlp_smem[];
-    constexpr int stride = kMhWarpFloats + TLP_DEPTH * 32 * VEC;
+    const int stride = a.mh_words + TLP_DEPTH * 32 * VEC;
     return tlp_smem + (size_t)(threadIdx.x >> 5) * stride;
+}
+
+// The cp.async path mirrors reduce_edges_async: rows shorter than the ring go
+// in under one commit group (their scores computed while the rows land), longer
+// rows run the paired pipeline, two edges per commit group; the next chunk's
+// indices and el values are loaded one chunk ahead; hot-source L2 policy on the
+// gathers (tagged colidx).  Same values in the same order as the register path.
+template <int VEC>
+__device__ __forceinline__ void mh_consume(const float *src, float ca, float cb, int split, Vec<VEC> &ac) {
+    if constexpr (VEC == 4) {
+        const float4 x = *reinterpret_cast<const float4 *>(src);
+        ac.v[0] = fmaf(0 < split ? ca : cb, x.x, ac.v[0]);
+        ac.v[1] = fmaf(1 < split ? ca : cb, x.y, ac.v[1]);
+        ac.v[2] = fmaf(2 < split ? ca : cb, x.z, ac.v[2]);
+        ac.v[3] = fmaf(3 < split ? ca : cb, x.w, ac.v[3]);
+    } else {
+#pragma unroll
+        for (int c = 0; c < VEC; ++c) ac.v[c] = fmaf(c < split ? ca : cb, src[c], ac.v[c]);
+    }
 }
 
 template <int VEC>
@@ -1009,10 +1072,11 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
                                                       float *&Dh, int &h_lo, int &nh, int &hl,
                                                       int &split) {
     constexpr int DD = TLP_DEPTH;
-    float *P = mh_warp_smem_async<VEC>();
-    float *M = P + kMhMaxHeads * 32;
-    float *Dn = M + kMhMaxHeads;
-    float *S = Dn + kMhMaxHeads;
+    static_assert(DD % 2 == 0, "paired async pipeline needs an even ring depth");
+    float *P = mh_warp_smem_async<VEC>(a);
+    float *M = P + a.mh_nh * 32;
+    float *Dn = M + a.mh_nh;
+    float *S = Dn + a.mh_nh;
     Mh = M;
     Dh = Dn;
     const int H = a.heads, fh = a.fh;
@@ -1031,28 +1095,56 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
     __syncwarp();
     const char *base = reinterpret_cast<const char *>(a.X + (active ? col : 0));
     const unsigned row_bytes = (unsigned)a.ldx * 4u;
+    const GPol gp = make_gpol(a);
     const int32_t *__restrict__ ci = a.colidx + e0;
     const float *__restrict__ erv = a.er + rglob * H + h_lo;
+    float er0[TLP_MHB];
+#pragma unroll
+    for (int k = 0; k < TLP_MHB; ++k) er0[k] = k < nh ? __ldg(erv + k) : 0.f;
     const int len = (int)(e1 - e0);
+    const float *pa = P + hl * 32;
+    const float *pb = P + hl2 * 32;
     Vec<VEC> ae, ao;
 #pragma unroll
     for (int c = 0; c < VEC; ++c) ae.v[c] = ao.v[c] = 0.f;
     if (len > 0) {
-        float *ring = mh_warp_ring<VEC>() + lane * VEC;
+        float *ring = P + a.mh_words + lane * VEC;
+        const unsigned ring_s = (unsigned)__cvta_generic_to_shared(ring);
         int n0 = min(32, len), n1 = min(32, len - 32);
-        int u0 = (lane < n0) ? __ldg(ci + lane) : 0;
-        int u1 = (lane < n1) ? __ldg(ci + 32 + lane) : 0;
+        int u0 = (lane < n0) ? ld_stream(ci + lane) : 0;
+        int u1 = (lane < n1) ? ld_stream(ci + 32 + lane) : 0;
+        float el0[TLP_MHB], el1[TLP_MHB];
+        mh_load_el(a, (unsigned)u0 & gp.mask, n0, h_lo, nh, lane, el0);
+        if (len < DD) {
+            for (int k = 0; k < len; ++k) {
+                const int uk = __shfl_sync(FULL, u0, k);
+                cp_async_x<VEC>(ring_s + 4u * k * 32 * VEC, base, (unsigned)uk, row_bytes, gp, active);
+            }
+            cp_async_commit();
+            // one chunk: the rescale of the (zero) chains is the identity
+            mh_chunk_scores(a, (unsigned)u0 & gp.mask, n0, H, h_lo, nh, erv, el0, er0, lane, P, M, Dn, S);
+            cp_async_wait<0>();
+            for (int j = 0; j < len; ++j) mh_consume<VEC>(ring + j * 32 * VEC, pa[j], pb[j], split, (j & 1) ? ao : ae);
+            __syncwarp();  // P and the ring are rewritten by the next row
 #pragma unroll
-        for (int k = 0; k < DD - 1; ++k) {
-            const int uk = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
-            cp_async_vec<VEC>(ring + k * 32 * VEC, row_ptr(base, (unsigned)uk, row_bytes), active && k < len);
+            for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
+            return;
+        }
+        // prologue: edges 0 .. DD-3 in flight, two edges per commit group
+#pragma unroll
+        for (int k = 0; k < DD - 2; k += 2) {
+            const int ua = __shfl_sync(FULL, k < 32 ? u0 : u1, k & 31);
+            const int ub = __shfl_sync(FULL, k + 1 < 32 ? u0 : u1, (k + 1) & 31);
+            cp_async_x<VEC>(ring_s + 4u * k * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && k < len);
+            cp_async_x<VEC>(ring_s + 4u * (k + 1) * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && k + 1 < len);
             cp_async_commit();
         }
         int slot = 0, off = 0;
         while (true) {
             const int n2 = min(32, len - off - 64);
-            const int u2 = (lane < n2) ? __ldg(ci + off + 64 + lane) : 0;
-            mh_chunk_scores(a, u0, n0, H, h_lo, nh, erv, lane, P, M, Dn, S);
+            const int u2 = (lane < n2) ? ld_stream(ci + off + 64 + lane) : 0;
+            if (n1 > 0) mh_load_el(a, (unsigned)u1 & gp.mask, n1, h_lo, nh, lane, el1);
+            mh_chunk_scores(a, (unsigned)u0 & gp.mask, n0, H, h_lo, nh, erv, el0, er0, lane, P, M, Dn, S);
             const float sA = S[hl], sB = S[hl2];
 #pragma unroll
             for (int c = 0; c < VEC; ++c) {
@@ -1060,29 +1152,30 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
                 ae.v[c] *= sc;
                 ao.v[c] *= sc;
             }
-            const float *pa = P + hl * 32;
-            const float *pb = P + hl2 * 32;
-            for (int j = 0; j < n0; ++j) {
-                const int jj = j + DD - 1;
-                const int ui = __shfl_sync(FULL, jj < 32 ? u0 : u1, jj & 31);
-                int ws = slot + DD - 1;
-                if (ws >= DD) ws -= DD;
-                cp_async_vec<VEC>(ring + ws * 32 * VEC, row_ptr(base, (unsigned)ui, row_bytes),
-                                  active && (off + jj) < len);
+            const int uq = ahead_index<DD - 2>(u0, u1, lane);
+            for (int j = 0; j < n0; j += 2) {
+                const int ja = j + DD - 2, jb = j + DD - 1;  // in this chunk or the next one
+                const int ua = __shfl_sync(FULL, uq, j);
+                const int ub = __shfl_sync(FULL, uq, j + 1);
+                int wa = slot + DD - 2;
+                if (wa >= DD) wa -= DD;
+                const int wb = wa + 1;  // slot and DD are even
+                cp_async_x<VEC>(ring_s + 4u * wa * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && (off + ja) < len);
+                cp_async_x<VEC>(ring_s + 4u * wb * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && (off + jb) < len);
                 cp_async_commit();
-                cp_async_wait<DD - 1>();
-                const float ca = pa[j], cb = pb[j];
-                const float *src = ring + slot * 32 * VEC;
-                Vec<VEC> &ac = (j & 1) ? ao : ae;
-#pragma unroll
-                for (int c = 0; c < VEC; ++c) ac.v[c] = fmaf(c < split ? ca : cb, src[c], ac.v[c]);
-                if (++slot == DD) slot = 0;
+                cp_async_wait<(DD - 2) / 2>();
+                mh_consume<VEC>(ring + slot * 32 * VEC, pa[j], pb[j], split, ae);
+                if (j + 1 < n0) mh_consume<VEC>(ring + (slot + 1) * 32 * VEC, pa[j + 1], pb[j + 1], split, ao);
+                slot += 2;
+                if (slot == DD) slot = 0;
             }
             __syncwarp();  // P, S are rewritten by the next chunk
             if (n1 <= 0) break;
             off += 32;
             n0 = n1; n1 = n2;
             u0 = u1; u1 = u2;
+#pragma unroll
+            for (int k = 0; k < TLP_MHB; ++k) el0[k] = el1[k];
         }
         cp_async_wait<0>();
     }
@@ -1479,7 +1572,7 @@ __device__ __forceinline__ void do_item(const AggArgs &a, int i, int lane) {
 // warps), where fewer registers spill into the edge loop (measured slower;
 // the alpha-mode GAT gather at 4 CTAs/SM: 26.9 -> 31.0 ms on Reddit).
 constexpr int min_blocks(int op, int coef, bool async, int G = 1) {
-    return async ? TLP_MINB_ASYNC
+    return async ? (op == OP_GATH ? TLP_MINB_MH_ASYNC : TLP_MINB_ASYNC)
          : (TLP_SMEMC && G > 1 && coef != COEF_NONE && (op == OP_GCN || op == OP_GIN || op == OP_GATB))
                ? TLP_MINB_SMC
                  : ((op == OP_GIN || op == OP_SAGE || op == OP_GCN) && coef == COEF_NONE)

@@ -32,6 +32,7 @@ if [ "$P" = "ncu" ] || [ "$P" = "all" ]; then
   prof reddit_repack k_repack 3 python scripts/traffic_probe.py gin 604 1
   prof reddit_gat_online k_agg 3 env TLP_GAT=online python scripts/traffic_probe.py gat 604 1
   prof products_gat k_agg 3 python scripts/one_call.py products gat 4
+  prof products_gat4 k_agg 3 python scripts/one_call.py products gat4 4
   prof rmat24_gcn k_agg 3 python scripts/one_call.py rmat24 gcn 4
   prof cora_gcn k_rows 3 python scripts/one_call.py cora gcn 4
   prof pubmed_gat k_rows 3 python scripts/one_call.py pubmed gat 4

@@ -38,7 +38,7 @@ METRICS = [
 TRAFFIC_KEYS = {
     "reddit_gcn": ("reddit", "gcn"), "reddit_gin": ("reddit", "gin"), "reddit_gat": ("reddit", "gat"),
     "reddit_gat_alpha": ("reddit", "gat_alpha"), "reddit_repack": ("reddit", "repack"),
-    "reddit_gat_online": ("reddit", "gat_online"), "products_gat": ("products", "gat"),
+    "reddit_gat_online": ("reddit", "gat_online"), "products_gat": ("products", "gat"), "products_gat4": ("products", "gat4"),
     "rmat24_gcn": ("rmat24", "gcn"), "cora_gcn": ("cora", "gcn"), "pubmed_gat": ("pubmed", "gat"),
 }
 
