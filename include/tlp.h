@@ -75,12 +75,17 @@ typedef enum tlp_norm {
  *   STATIC  : persistent grid, task t handled by warp t mod W (no atomics)
  *   HARDWARE: one warp per task, grid sized to the task count
  *   PAPER   : the paper's heuristic switch: DYNAMIC if
- *             n_dst > 1,000,000 or nnz/n_dst > 50, else HARDWARE. */
+ *             n_dst > 1,000,000 or nnz/n_dst > 50, else HARDWARE.
+ *   CLC     : Blackwell Cluster Launch Control work stealing:
+ *             one CTA per warps_per_cta x step tasks; a running CTA cancels a
+ *             not-yet-started CTA (clusterlaunchcontrol.try_cancel) and takes
+ *             over its tasks -- Alg. 1's balancing without a global counter. */
 typedef enum tlp_sched {
     TLP_SCHED_DYNAMIC = 0,
     TLP_SCHED_STATIC = 1,
     TLP_SCHED_HARDWARE = 2,
-    TLP_SCHED_PAPER = 3
+    TLP_SCHED_PAPER = 3,
+    TLP_SCHED_CLC = 4
 } tlp_sched;
 
 /* Aggregation kinds of the descriptor API (tlp_aggregate). */
@@ -216,8 +221,6 @@ tlp_status tlp_graph_degrees(tlp_graph g, int32_t *in_deg, int32_t *out_deg,
 tlp_status tlp_graph_plan(tlp_graph g, int32_t *tasks, int32_t *hub_rows,
                           int32_t *hub_chunk_off, void *stream);
 
-/* Selects the scheduler (tlp_sched), warps per CTA (0 = default 8) and the
- * tasks fetched per atomic (Alg. 1's `step`; 0 = derived from F). */
 /* Debug visit counter (Alg. 1's exactly-once semantics,
  * P:883-906): while `counter` (device int32 [n_dst], zeroed by the caller) is
  * set, every aggregation on this handle adds 1 to counter[r] each time it
@@ -227,6 +230,9 @@ tlp_status tlp_graph_plan(tlp_graph g, int32_t *tasks, int32_t *hub_rows,
  * until reset with NULL.  Costs one atomic per row strip; off by default. */
 tlp_status tlp_graph_set_visit_counter(tlp_graph g, int32_t *counter);
 
+/* Selects the scheduler (tlp_sched), warps per CTA (0 = default 8) and the
+ * tasks fetched per atomic (Alg. 1's `step`; 0 = derived from F; CLC: tasks
+ * per warp of one CTA's block).  Unknown sched -> TLP_ERR_INVALID_ARGUMENT. */
 tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta,
                                   int step);
 

@@ -36,7 +36,7 @@ STATUS = {0: "TLP_OK", 1: "TLP_ERR_INVALID_ARGUMENT", 2: "TLP_ERR_INVALID_GRAPH"
           3: "TLP_ERR_OUT_OF_MEMORY", 4: "TLP_ERR_CUDA", 5: "TLP_ERR_NCCL",
           6: "TLP_ERR_UNSUPPORTED"}
 NORMS = {"none": 0, "right": 1, "both": 2}
-SCHEDS = {"dynamic": 0, "static": 1, "hardware": 2, "paper": 3}
+SCHEDS = {"dynamic": 0, "static": 1, "hardware": 2, "paper": 3, "clc": 4}
 
 
 class tlp_create_opts(ctypes.Structure):

@@ -954,6 +954,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     }
     if (groups > 1 || r.op == OP_GATB) async_path = false;  // OP_GATB: register path only
     const int path = groups > 1 ? 2 : (async_path ? 1 : 0);
+    // CLC scheduling is compiled into the register-path kernels only (see
+    // agg_clc): the cp.async kernels run it with the atomic counter
+    if (sched == S_CLC && async_path) a.sched = sched = S_DYNAMIC;
     // hot-source L2 policy: cp.async path only (rows streamed from HBM)
     if (async_path && r.op != OP_GATB) {
         unsigned thr = 0;
@@ -983,10 +986,12 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     }
     // the general persistent kernel over a.n_items work items
     auto launch_general = [&](const AggArgs &ag) -> tlp_status {
-        if (smem > 0 && sched == S_HARDWARE) occupancy_blocks(fn, threads, smem);  // sets attributes
+        if (smem > 0 && (sched == S_HARDWARE || sched == S_CLC)) occupancy_blocks(fn, threads, smem);  // sets attributes
         int64_t blocks;
         if (sched == S_HARDWARE) {
             blocks = (ag.n_items + wpc - 1) / wpc;
+        } else if (sched == S_CLC) {  // one CTA per wpc * step items; running CTAs steal the rest
+            blocks = (ag.n_items + (int64_t)wpc * step - 1) / ((int64_t)wpc * step);
         } else {
             int per_sm = occupancy_blocks(fn, threads, smem);
             if (const char *e = knob("TLP_CTAS"))  // measurement: cap resident CTAs per SM

@@ -46,7 +46,7 @@ namespace tlp {
 // OP_GATB: GAT backward on the transposed graph (NEXT-4, tlp_gat_backward).
 enum Op : int { OP_GCN = 0, OP_GIN = 1, OP_GAT = 2, OP_SAGE = 3, OP_GATH = 4, OP_GATB = 5 };
 enum Coef : int { COEF_NONE = 0, COEF_COUT = 1, COEF_W = 2, COEF_W_COUT = 3 };
-enum Sched : int { S_DYNAMIC = 0, S_STATIC = 1, S_HARDWARE = 2 };
+enum Sched : int { S_DYNAMIC = 0, S_STATIC = 1, S_HARDWARE = 2, S_CLC = 4 };
 
 constexpr unsigned FULL = 0xffffffffu;
 
@@ -1579,6 +1579,72 @@ constexpr int min_blocks(int op, int coef, bool async, int G = 1) {
                        ? TLP_MINB_LIGHT : TLP_MINB;
 }
 
+// Cluster Launch Control work stealing (S_CLC, SURVEY 8(a) a4's Blackwell
+// option): the grid has one CTA per block of wpc * step work items.  Each warp
+// first does its own step items of its CTA's block; then, warp by warp (no CTA
+// barrier), it asks the hardware to cancel a CTA that has not started yet
+// (clusterlaunchcontrol.try_cancel, answered through the warp's own mbarrier)
+// and does that CTA's whole block alone, until no launch is left to cancel.
+// The request for the next block is issued before the current one is
+// processed, so its latency hides behind the work.  No global atomics, no
+// counter reset.  Register-path kernels only: with the cp.async kernels'
+// cache-policy copies in the same kernel, ptxas 12.9 emits LDGSTS with an
+// odd uniform-register descriptor (desc[UR1]: illegal instruction at run
+// time), so the dispatcher runs those kernels with the atomic counter.
+__device__ __forceinline__ void clc_request(unsigned res, unsigned bar) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], 16;\n" ::"r"(bar) : "memory");
+    asm volatile("clusterlaunchcontrol.try_cancel.async.shared::cta.mbarrier::complete_tx::bytes.b128 [%0], [%1];\n"
+                 ::"r"(res), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void clc_wait(unsigned bar, unsigned phase) {
+    asm volatile("{\n\t.reg .pred p;\n"
+                 "CLC_WAIT:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+                 "@!p bra CLC_WAIT;\n\t}\n" ::"r"(bar), "r"(phase) : "memory");
+}
+// the canceled CTA's x coordinate, or -1 when nothing was left to cancel
+__device__ __forceinline__ int clc_result(unsigned res) {
+    int bx, ok;
+    asm volatile("{\n\t.reg .pred p;\n\t.reg .b128 r;\n\t"
+                 "ld.shared.b128 r, [%2];\n\t"
+                 "clusterlaunchcontrol.query_cancel.is_canceled.pred.b128 p, r;\n\t"
+                 "selp.u32 %1, 1, 0, p;\n\t"
+                 "@p clusterlaunchcontrol.query_cancel.get_first_ctaid::x.b32.b128 %0, r;\n\t}\n"
+                 : "=r"(bx), "=r"(ok) : "r"(res) : "memory");
+    return ok ? bx : -1;
+}
+
+template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
+__device__ __forceinline__ void agg_clc(const AggArgs &a, int lane) {
+    __shared__ __align__(16) uint4 clc_res[TLP_MAXT / 32];
+    __shared__ __align__(8) unsigned long long clc_bar[TLP_MAXT / 32];
+    const int wpc = (int)(blockDim.x >> 5), warp = (int)(threadIdx.x >> 5);
+    const unsigned res = (unsigned)__cvta_generic_to_shared(&clc_res[warp]);
+    const unsigned bar = (unsigned)__cvta_generic_to_shared(&clc_bar[warp]);
+    if (lane == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(bar) : "memory");
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncwarp();
+    const int n_items = (int)a.n_items;
+    const int blk = wpc * a.step;  // work items of one CTA
+    // own share of this CTA's block
+    int t0 = (int)blockIdx.x * blk + warp * a.step, tend = min(t0 + a.step, n_items);
+    unsigned phase = 0;
+    while (true) {
+        if (lane == 0) clc_request(res, bar);
+        for (int tt = t0; tt < tend; ++tt) do_item<VEC, OP, COEF, U, ASYNC, G>(a, tt, lane);
+        clc_wait(bar, phase);
+        const int b = clc_result(res);
+        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");  // read before the next async write
+        __syncwarp();
+        if (b < 0) break;
+        phase ^= 1u;
+        t0 = b * blk;  // a canceled CTA's whole block
+        tend = min(t0 + blk, n_items);
+    }
+}
+
 template <int VEC, int OP, int COEF, int U, bool ASYNC, int G>
 __device__ __forceinline__ void agg_body(const AggArgs &a) {
     const int lane = threadIdx.x & 31;
@@ -1588,6 +1654,13 @@ __device__ __forceinline__ void agg_body(const AggArgs &a) {
         if (wid < n_items) do_item<VEC, OP, COEF, U, ASYNC, G>(a, wid, lane);
         if (a.n_dests > 0) __threadfence_system();
         return;
+    }
+    if constexpr (!ASYNC) {
+        if (a.sched == S_CLC) {
+            agg_clc<VEC, OP, COEF, U, ASYNC, G>(a, lane);
+            if (a.n_dests > 0) __threadfence_system();
+            return;
+        }
     }
     const int W = (int)((gridDim.x * blockDim.x) >> 5);
     int t = wid * a.step;  // static first wave

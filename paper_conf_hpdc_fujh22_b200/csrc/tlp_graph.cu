@@ -739,7 +739,7 @@ tlp_status tlp_graph_set_visit_counter(tlp_graph g, int32_t *counter) {
 
 tlp_status tlp_graph_set_schedule(tlp_graph g, int sched, int warps_per_cta, int step) {
     if (!g) return set_error(TLP_ERR_INVALID_ARGUMENT, "null graph");
-    if (sched < TLP_SCHED_DYNAMIC || sched > TLP_SCHED_PAPER)
+    if (sched < TLP_SCHED_DYNAMIC || sched > TLP_SCHED_CLC)
         return set_error(TLP_ERR_INVALID_ARGUMENT, "unknown scheduler");
     if (warps_per_cta < 0 || warps_per_cta > 32 || step < 0)
         return set_error(TLP_ERR_INVALID_ARGUMENT, "warps_per_cta in [0,32], step >= 0");

@@ -56,6 +56,26 @@ def test_library_is_sm100a_only():
     assert archs == {"100a"}, archs
 
 
+def test_sass_cache_policy_descriptors_are_register_pairs():
+    """Every memory instruction that carries an L2 cache-policy descriptor
+    (desc[URx], a 64-bit uniform-register pair) names an even register.
+    ptxas 12.9 emitted LDGSTS with desc[UR1] in the cp.async kernels once they
+    also held the Cluster Launch Control scheduler (an illegal instruction at
+    run time); this guards the built library against that miscompile."""
+    import shutil
+    import subprocess
+    import paper_conf_hpdc_fujh22_b200 as tlp
+    cuobjdump = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(cuobjdump):
+        pytest.skip("cuobjdump not available")
+    sass = subprocess.run([cuobjdump, "-sass", tlp.LIB_PATH], capture_output=True, text=True).stdout
+    regs = [int(r) for r in re.findall(r"desc\[UR(\d+)\]", sass)]
+    assert regs, "no cache-policy descriptors found (disassembly failed?)"
+    odd = sorted({r for r in regs if r % 2})
+    assert not odd, f"odd uniform registers used as descriptors: {odd}"
+    assert "UGETNEXTWORKID" in sass  # the CLC scheduler is compiled in
+
+
 @pytest.mark.parametrize("parts", [1, 2, 3, 4, 7, 8])
 def test_partition_rows_bit_exact(parts):
     import paper_conf_hpdc_fujh22_b200 as tlp

@@ -259,7 +259,7 @@ def test_deterministic_across_runs_and_schedules(tlp):
     g = tlp.Graph(_t(rp), _t(ci), opts=dict(hub_threshold=100, hub_chunk=40))
     base = {"gcn": g.gcn(X, "both", F=130).clone(), "gin": g.gin(X, 0.1, F=130).clone(),
             "gat": g.gat(X, el, er, 0.2, F=130).clone()}
-    for sched in ("dynamic", "static", "hardware", "paper"):
+    for sched in ("dynamic", "static", "hardware", "paper", "clc"):
         for wpc, step in ((8, 0), (4, 1), (2, 3), (16, 7)):
             g.set_schedule(sched, wpc, step)
             for _ in range(2):
@@ -821,7 +821,7 @@ def test_backward_deterministic_and_transpose_once(tlp):
     g.build_transpose()  # idempotent
     G = _t(synth.features(3000, 130, 132, seed=3))
     a = g.gcn_backward(G, "both", F=130).clone()
-    for sched in ("static", "hardware", "dynamic"):
+    for sched in ("static", "hardware", "dynamic", "clc"):
         g.set_schedule(sched)
         assert torch.equal(g.gcn_backward(G, "both", F=130), a)
     g.close()
@@ -1147,7 +1147,7 @@ def test_gat_alpha_mode_bitwise_across_paths(tlp, monkeypatch):
         assert torch.equal(g.gat(X, el, er, 0.2), base), path
     monkeypatch.delenv("TLP_GATHER")
     monkeypatch.setenv("TLP_PANEL", "64")
-    for sched in ("static", "hardware", "dynamic"):
+    for sched in ("static", "hardware", "dynamic", "clc"):
         for wpc, step in ((4, 1), (8, 3)):
             g.set_schedule(sched, wpc, step)
             assert torch.equal(g.gat(X, el, er, 0.2), base), (sched, wpc, step)
@@ -1225,7 +1225,7 @@ def test_lane_groups_bitwise_across_schedules_and_partitions(tlp, monkeypatch, F
     base = {"gcn": g.gcn(X, "both").clone(), "gin": g.gin(X, 0.1).clone(), "gat": g.gat(X, el, er, 0.2).clone()}
     _check("groups gcn", base["gcn"], oracle.gcn(rp, ci, Xh, "both"))
     _check("groups gat", base["gat"], oracle.gat(rp, ci, Xh, elh, erh, 0.2))
-    for sched in ("static", "hardware", "dynamic", "paper"):
+    for sched in ("static", "hardware", "dynamic", "paper", "clc"):
         for wpc, step in ((4, 1), (8, 3), (2, 7)):
             g.set_schedule(sched, wpc, step)
             assert torch.equal(g.gcn(X, "both"), base["gcn"]), (sched, wpc, step)
@@ -1340,7 +1340,7 @@ def test_visit_counter_exactly_once(tlp, monkeypatch, mode):
     tlp.tlp_graph_set_visit_counter(g.handle, cnt)
     ops = [lambda: g.gat(X, el, er, 0.2)] if mode == "gat_alpha" else \
           [lambda: g.gcn(X, "both"), lambda: g.gin(X, 0.1), lambda: g.gat(X, el, er, 0.2)]
-    for sched in ("dynamic", "static", "hardware"):
+    for sched in ("dynamic", "static", "hardware", "clc"):
         g.set_schedule(sched)
         for f in ops:
             cnt.zero_()
