@@ -914,18 +914,42 @@ __device__ __forceinline__ void mh_load_el(const AggArgs &a, unsigned u_l, int n
     for (int k = 0; k < TLP_MHB; ++k) v[k] = (k < nh && lane < n0) ? __ldg(elu + k) : 0.f;
 }
 
+// Butterfly reduction of four values per lane at once (heads k = 0..3 of a
+// block): after the first two exchange steps every lane carries one head,
+// q = (lane >> 3) & 3, so the four reductions take 6 shuffles instead of 20.
+// Each head's value is formed with the association of warp_sum / warp_max
+// (own + partner at distances 16, 8, 4, 2, 1), so it is bitwise the
+// one-value-at-a-time result; every lane of octet q holds head q's total.
+template <bool MAX>
+__device__ __forceinline__ float reduce4_transposed(const float (&v)[4], int lane) {
+    auto op = [](float x, float y) { return MAX ? fmaxf(x, y) : x + y; };
+    const bool hi = lane & 16;
+    const float s0 = hi ? v[0] : v[2], s1 = hi ? v[1] : v[3];
+    const float k0 = hi ? v[2] : v[0], k1 = hi ? v[3] : v[1];
+    const float a0 = op(k0, __shfl_xor_sync(FULL, s0, 16));  // head 0 (2 on the upper half)
+    const float a1 = op(k1, __shfl_xor_sync(FULL, s1, 16));  // head 1 (3)
+    const bool b3 = lane & 8;
+    float c = op(b3 ? a1 : a0, __shfl_xor_sync(FULL, b3 ? a0 : a1, 8));
+#pragma unroll
+    for (int o = 4; o > 0; o >>= 1) c = op(c, __shfl_xor_sync(FULL, c, o));
+    return c;
+}
+
 // Scores, online-softmax update and weights of one 32-edge chunk for the heads
-// [h_lo, h_lo+nh) of a strip (lane j holds edge j with source u_l).  Heads are
-// processed TLP_MHB at a time so their el loads and warp reductions overlap;
-// the first block's el / er values come in el0 / er0.
+// [h_lo, h_lo+nh) of a strip (lane j holds edge j with source u_l), four heads
+// per block: transposed max / sum reductions, and the running max, denominator
+// and rescale of head q updated by lane 8q (all four in parallel); the first
+// block's el / er values come in el0 / er0.
 __device__ __forceinline__ void mh_chunk_scores(const AggArgs &a, unsigned u_l, int n0, int H, int h_lo,
                                                 int nh, const float *__restrict__ erv,
                                                 const float (&el0)[TLP_MHB], const float (&er0)[TLP_MHB],
                                                 int lane, float *P, float *M, float *D, float *S) {
+    static_assert(TLP_MHB == 4, "the transposed head reductions take four heads per block");
     constexpr int B = TLP_MHB;
     const float *__restrict__ elu = a.el + (size_t)u_l * H + h_lo;
+    const int q = (lane >> 3) & 3;
     for (int hb = 0; hb < nh; hb += B) {
-        float sv[B], mo[B], mn[B], sm[B];
+        float sv[B];
 #pragma unroll
         for (int k = 0; k < B; ++k) {
             sv[k] = -INFINITY;
@@ -934,26 +958,22 @@ __device__ __forceinline__ void mh_chunk_scores(const AggArgs &a, unsigned u_l, 
                 sv[k] = t >= 0.f ? t : a.slope * t;  // LeakyReLU (R6)
             }
         }
+        const bool mine = hb + q < nh;  // head q of this block exists
+        const float mo = mine ? M[hb + q] : -INFINITY;
+        const float mn = fmaxf(mo, reduce4_transposed<true>(sv, lane));
+        float p[B];
 #pragma unroll
         for (int k = 0; k < B; ++k) {
-            if (hb + k < nh) {  // warp-uniform
-                mo[k] = M[hb + k];
-                mn[k] = fmaxf(mo[k], warp_max(sv[k]));
-                const float p = (lane < n0) ? __expf(sv[k] - mn[k]) : 0.f;
-                sm[k] = warp_sum(p);
-                P[(hb + k) * 32 + lane] = p;
-            }
+            const float mk = __shfl_sync(FULL, mn, 8 * k);
+            p[k] = (lane < n0 && hb + k < nh) ? __expf(sv[k] - mk) : 0.f;
+            if (hb + k < nh) P[(hb + k) * 32 + lane] = p[k];
         }
-        __syncwarp();
-        if (lane == 0) {
-#pragma unroll
-            for (int k = 0; k < B; ++k)
-                if (hb + k < nh) {
-                    const float scale = __expf(mo[k] - mn[k]);
-                    M[hb + k] = mn[k];
-                    D[hb + k] = fmaf(D[hb + k], scale, sm[k]);
-                    S[hb + k] = scale;
-                }
+        const float sm = reduce4_transposed<false>(p, lane);
+        if ((lane & 7) == 0 && mine) {
+            const float scale = __expf(mo - mn);
+            M[hb + q] = mn;
+            D[hb + q] = fmaf(D[hb + q], scale, sm);
+            S[hb + q] = scale;
         }
         __syncwarp();
     }
