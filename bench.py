@@ -137,6 +137,8 @@ class ClockSampler:
         self.period = int(period_ms or os.environ.get("TLP_CLOCK_MS", "50"))
         self.proc = None
         self.lines = []
+        self.stamps = []
+        self.t0 = 0.0
 
     def __enter__(self):
         if self.period <= 0:
@@ -148,12 +150,19 @@ class ClockSampler:
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            # nvidia-smi takes a few hundred ms to emit its first sample: wait
+            # for it, so the region that follows is sampled from its start
+            t_wait = time.time() + 3.0
+            while not self.lines and time.time() < t_wait:
+                time.sleep(0.005)
+            self.t0 = time.time()
         except Exception:
             self.proc = None
         return self
 
     def _read(self):
         for line in self.proc.stdout:
+            self.stamps.append(time.time())
             self.lines.append(line.strip())
 
     def __exit__(self, *a):
@@ -168,7 +177,10 @@ class ClockSampler:
     def summary(self):
         sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        stamps = self.stamps + [float("inf")] * (len(self.lines) - len(self.stamps))
+        for ts, ln in zip(stamps, self.lines):
+            if ts < self.t0:  # the warm-up sample taken before the region
+                continue
             parts = [p.strip() for p in ln.split(",")]
             if len(parts) < 9:
                 continue

@@ -7,9 +7,14 @@ P=${1:-all}
 export TLP_SYNTH_CACHE=/tmp/tlp_synth
 if [ "$P" = "bench" ] || [ "$P" = "all" ]; then
   TLP_TRACE_CREATE=1 python bench.py > $O/bench.json 2> $O/bench.err
-  for w in products rmat24 reddit_f32 products_f32 reddit_sage products_gat4 reddit_bwd reddit_gat_bwd; do
+  # short steps get more of them, so the clock sampler sees >= ~10 samples
+  for w in rmat24 reddit_sage reddit_bwd reddit_gat_bwd; do
     timeout 900 python bench.py --workload $w --no-cpu-baseline > $O/bench_$w.json 2> $O/bench_$w.err
   done
+  for w in products products_gat4 products_f32; do
+    timeout 900 python bench.py --workload $w --no-cpu-baseline --steps 60 > $O/bench_$w.json 2> $O/bench_$w.err
+  done
+  timeout 900 python bench.py --workload reddit_f32 --no-cpu-baseline --steps 200 > $O/bench_reddit_f32.json 2> $O/bench_reddit_f32.err
   for w in cora pubmed; do
     timeout 900 python bench.py --workload $w --no-cpu-baseline --steps 4000 --warmup 100 > $O/bench_$w.json 2> $O/bench_$w.err
   done
