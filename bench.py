@@ -618,13 +618,15 @@ def run_tlp(args):
                                   "dram__bytes_write.sum per launch, ncu --set full of this round's kernels)"}
     probe = None
     if panel and rank == 0:
-        # ~30 probe runs (~0.1 s) so the clock sampler sees them; the best run is the ceiling
+        # probe runs for ~0.4 s so the clock sampler sees them; the best run is the ceiling
         runs = []
         with ClockSampler(local) as pclk:
-            for _ in range(30):
+            t_end = time.time() + 0.4  # >= ~8 clock samples
+            while (time.time() < t_end or len(runs) < 30) and len(runs) < 2000:
                 r_ = l2_gather_ceiling(n * 256)
-                if r_:
-                    runs.append(r_)
+                if not r_:
+                    break
+                runs.append(r_)
         if runs:
             probe = max(runs, key=lambda r_: r_["GBs"])
             probe["median_GBs"] = round(statistics.median(r_["GBs"] for r_ in runs), 1)
