@@ -982,7 +982,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         const int W = 32 * vec;
         a.mh_nh = std::min((int)r.heads, (W - 1 + fh - 1) / fh + 1);
         a.mh_words = (a.mh_nh * 32 + 3 * a.mh_nh + 1 + 3) & ~3;
-        smem = (size_t)wpc * (a.mh_words + (async_path ? TLP_DEPTH * 32 * vec : 0)) * sizeof(float);
+        smem = (size_t)wpc * (a.mh_words + (async_path ? TLP_DEPTH_MH * 32 * vec : 0)) * sizeof(float);
     }
     // the general persistent kernel over a.n_items work items
     auto launch_general = [&](const AggArgs &ag) -> tlp_status {

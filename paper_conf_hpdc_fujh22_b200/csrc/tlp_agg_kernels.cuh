@@ -624,6 +624,9 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
 #ifndef TLP_DEPTH
 #define TLP_DEPTH 16   // edges in flight per warp on the async path
 #endif
+#ifndef TLP_DEPTH_MH
+#define TLP_DEPTH_MH 16  // multi-head GAT async ring depth (its scoring pauses the issue)
+#endif
 #ifndef TLP_ASYNC_PAIR
 #define TLP_ASYNC_PAIR 1  // two edges per cp.async commit group (fewer waits per edge)
 #endif
@@ -1062,7 +1065,7 @@ __device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, in
 template <int VEC>
 __device__ __forceinline__ float *mh_warp_smem_async(const AggArgs &a) {
     extern __shared__ __align__(16) float tlp_smem[];
-    const int stride = a.mh_words + TLP_DEPTH * 32 * VEC;
+    const int stride = a.mh_words + TLP_DEPTH_MH * 32 * VEC;
     return tlp_smem + (size_t)(threadIdx.x >> 5) * stride;
 }
 
@@ -1091,7 +1094,7 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
                                                       int lane, Vec<VEC> &acc, float *&Mh,
                                                       float *&Dh, int &h_lo, int &nh, int &hl,
                                                       int &split) {
-    constexpr int DD = TLP_DEPTH;
+    constexpr int DD = TLP_DEPTH_MH;
     static_assert(DD % 2 == 0, "paired async pipeline needs an even ring depth");
     float *P = mh_warp_smem_async<VEC>(a);
     float *M = P + a.mh_nh * 32;
