@@ -45,6 +45,14 @@ OPS = ("gcn", "gin", "gat")
 
 # ------------------------------------------------------------------ bytes --
 
+
+def _sig(x, digits=5):
+    """x rounded to `digits` significant digits (small-graph steps are ~0.02 ms)."""
+    if not x:
+        return x
+    import math
+    return round(x, max(0, digits - 1 - int(math.floor(math.log10(abs(x))))))
+
 def gather_bytes(op, n_rows, n_edges, F):
     """Algorithmic (gather-model) bytes of one aggregation."""
     if op == "gcn":
@@ -414,18 +422,24 @@ def run_tlp(args):
     torch.cuda.synchronize()
     l_before = tlp.tlp_graph_info_get(g.handle)["launches"]
     with ClockSampler(local) as clk:
+        # a one-op step is timed by the start / stop pair alone: per-launch
+        # events would add host work between back-to-back launches of a
+        # microsecond-scale kernel (Cora, Pubmed) and leave the GPU idle
+        per_op_events = len(ops) > 1
         start.record(stream)
         for _ in range(args.steps):
             for op in ops:
-                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                a.record(stream)
+                if per_op_events:
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
                 if graphs is not None:
                     for _r in range(args.graph_reps):
                         graphs[op].replay()
                 else:
                     launch(op)
-                b.record(stream)
-                ev[op].append((a, b))
+                if per_op_events:
+                    b.record(stream)
+                    ev[op].append((a, b))
         stop.record(stream)
         torch.cuda.synchronize()
     if use_dist:
@@ -437,7 +451,10 @@ def run_tlp(args):
         n_launches = tlp.tlp_graph_info_get(g.handle)["launches"] - l_before
     reps = args.graph_reps if graphs is not None else 1
     total_ms = start.elapsed_time(stop) / reps
-    op_ms = {op: [a.elapsed_time(b) / reps for a, b in ev[op]] for op in ops}
+    if per_op_events:
+        op_ms = {op: [a.elapsed_time(b) / reps for a, b in ev[op]] for op in ops}
+    else:  # one op: its time per launch is the step time
+        op_ms = {op: [total_ms / args.steps] for op in ops}
     t = torch.tensor([total_ms], device=dev)
     if use_dist:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -454,10 +471,13 @@ def run_tlp(args):
     # overhead, not synchronised) and, with --cold, each op with L2 flushed
     host_us = {}
     for op in ops:
-        torch.cuda.synchronize()
-        t_h = time.perf_counter()
-        launch(op)
-        host_us[op] = (time.perf_counter() - t_h) * 1e6
+        hs = []
+        for _ in range(21):
+            torch.cuda.synchronize()
+            t_h = time.perf_counter()
+            launch(op)
+            hs.append((time.perf_counter() - t_h) * 1e6)
+        host_us[op] = statistics.median(hs)
         torch.cuda.synchronize()
     cold_ms = {}
     if args.cold:
@@ -537,7 +557,7 @@ def run_tlp(args):
         h2d = Xp.numel() * 4 + elp.numel() * 4 + erp.numel() * 4
         d2h = sum(Yp[op].numel() * 4 for op in ops) if read_back else 0
         e2e = {"value": round(step_bytes / (e2e_ms * 1e-3) / 1e9, 2), "unit": "GB/s",
-               "ms_per_step": round(e2e_ms, 3), "h2d_bytes_per_step": int(h2d),
+               "ms_per_step": _sig(e2e_ms), "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h),
                "note": "per step: pinned host X/el/er -> device (every rank), the step's "
                        "aggregations, every Y -> pinned host (rank 0); copies pipelined on two "
@@ -592,9 +612,9 @@ def run_tlp(args):
         ms = statistics.mean(op_ms[op])
         by = gather_bytes(op, n, E, F)
         srt = sorted(op_ms[op])
-        per_op[op] = {"ms_mean": round(ms, 4), "ms_median": round(statistics.median(op_ms[op]), 4),
-                      "ms_min": round(srt[0], 4),
-                      "ms_p90": round(srt[min(len(srt) - 1, int(0.9 * len(srt)))], 4),
+        per_op[op] = {"ms_mean": _sig(ms), "ms_median": _sig(statistics.median(op_ms[op])),
+                      "ms_min": _sig(srt[0]),
+                      "ms_p90": _sig(srt[min(len(srt) - 1, int(0.9 * len(srt)))]),
                       "host_call_us": round(host_us[op], 1),
                       "gather_bytes": int(by), "gather_GBs": round(by / (ms * 1e-3) / 1e9, 1),
                       "frac_of_8TBs": round(by / (ms * 1e-3) / 1e9 / NOMINAL_HBM_GBS, 4),
@@ -608,11 +628,14 @@ def run_tlp(args):
     # gathered rows are L2 hits, so the bound is the L2 random-row gather rate,
     # measured in this run by the probe (same clocks, same box)
     panel = n * ld * 4 > 0.6 * 126e6 and n * 256 <= 0.6 * 126e6 and F > 64
-    roofline = {"kernel": f"k_agg ({dom})", "achieved": achieved, "unit": "GB/s",
+    # hub-free graphs whose X fits in L2 run the short-row kernel (tlp_k_rows.cu)
+    kname = "k_rows" if (info["n_hubs"] == 0 and n * ld * 4 <= 0.6 * 126e6) else "k_agg"
+    roofline = {"kernel": f"{kname} ({dom})", "achieved": achieved, "unit": "GB/s",
                 "bytes_per_launch": per_op[dom]["gather_bytes"],
                 "bytes_model": "gather model (SURVEY 8(d) d2): per edge 4F + 4 colidx + 4 coef/el; "
                                "per row Y, rowptr (+self/er); time = the op's mean CUDA-event "
-                               "duration over the timed region (all of its launches)",
+                               "duration over the timed region (all of its launches; a one-op "
+                               "step: the step time)",
                 "traffic": traffic,
                 "traffic_source": "profiles/ncu_traffic.json (dram__bytes_read.sum + "
                                   "dram__bytes_write.sum per launch, ncu --set full of this round's kernels)"}
@@ -654,7 +677,7 @@ def run_tlp(args):
 
     result = {
         "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3),
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": _sig(ms_per_step),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic",
         "config": {"workload": workload_desc(name, cfg, E),

@@ -1026,10 +1026,17 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
                   4.0 * (double)g->n_src * (double)r.ldx <= 0.6 * (double)g->l2_bytes &&
                   knob("TLP_PANEL") == nullptr && knob("TLP_GATHER") == nullptr;
     if (const char *e = knob("TLP_ROWS")) rows_k = rows_ok && atoi(e) != 0;
-    KernelFn fr = rows_k ? pick_rows(op, coef, a.hot_thr != 0) : nullptr;
+    const int nstr = (int)((r.F + 127) / 128);
+    // strips per short-row work item (TLP_ROWS_NSI=1|2 overrides)
+    int nsi = nstr >= 2 ? 2 : 1;
+    if (const char *e = knob("TLP_ROWS_NSI")) nsi = (atoi(e) == 2) ? 2 : 1;
+    // nothing but the aggregation itself: the short-row kernel's lean store path
+    const bool plain = a.bias == nullptr && a.act == TLP_ACT_NONE && a.n_dests == 0 && a.mc == nullptr &&
+                       a.proj == nullptr && !a.stream_hint && a.visits == nullptr;
+    KernelFn fr = rows_k ? pick_rows(op, coef, a.hot_thr != 0, nsi, plain) : nullptr;
 
     if (fr) {
-        const int nstr = (int)((r.F + 127) / 128);
+        const int ipr = (nstr + nsi - 1) / nsi;  // work items per row
         if (g->n_hubs > 0) {  // hub chunks in the general kernel (tasks [0, n_chunks))
             AggArgs ah = a;
             ah.panel = 0;  // task-major: each hub-chunk item covers all strips
@@ -1043,9 +1050,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
         ar.panel = 0;
         ar.skip_hubs = g->n_hubs > 0 ? 1 : 0;
         ar.hub_H = g->H;
-        ar.n_items = g->n_dst * (int64_t)nstr;
-        ar.tasks_magic = (nstr > 1)
-                             ? (unsigned long long)((((unsigned __int128)1) << 64) / (unsigned __int128)nstr) + 1ull
+        ar.n_items = g->n_dst * (int64_t)ipr;
+        ar.tasks_magic = (ipr > 1)
+                             ? (unsigned long long)((((unsigned __int128)1) << 64) / (unsigned __int128)ipr) + 1ull
                              : 0ull;
         if (ar.n_items >= (int64_t(1) << 31)) return set_error(TLP_ERR_UNSUPPORTED, "too many rows x strips");
         const int per_sm = occupancy_blocks(fr, 256, 0);

@@ -1749,6 +1749,6 @@ KernelFn pick_g2(int op, int coef);         // PAIR half-warps (64-column strips
 KernelFn pick_g4(int op, int coef);         // 4 lane groups (narrow rows)
 KernelFn pick_g8(int op, int coef);         // 8 lane groups
 KernelFn pick_mh(int vec, bool async_path); // multi-head GAT
-KernelFn pick_rows(int op, int coef, bool hint);  // short-row kernel (tlp_k_rows.cu), VEC 4
+KernelFn pick_rows(int op, int coef, bool hint, int nsi, bool plain);  // short-row kernel (tlp_k_rows.cu), VEC 4
 
 }  // namespace tlp
