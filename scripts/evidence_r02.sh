@@ -50,4 +50,5 @@ if [ "$P" = "probes" ] || [ "$P" = "all" ]; then
   timeout 300 /tmp/tma_probe > $O/tma_probe.txt 2>&1
   python scripts/host_probe.py > $O/host_probe.txt 2>&1
   (cd scripts && python small_probe2.py > ../$O/small_probe.txt 2>&1)
+  (cd scripts && python rows_probe.py > ../$O/rows_probe.txt 2>&1)
 fi
