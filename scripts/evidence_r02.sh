@@ -16,7 +16,7 @@ if [ "$P" = "bench" ] || [ "$P" = "all" ]; then
   done
   timeout 900 python bench.py --workload reddit_f32 --no-cpu-baseline --steps 200 > $O/bench_reddit_f32.json 2> $O/bench_reddit_f32.err
   for w in cora pubmed; do
-    timeout 900 python bench.py --workload $w --no-cpu-baseline --steps 4000 --warmup 100 > $O/bench_$w.json 2> $O/bench_$w.err
+    timeout 900 python bench.py --workload $w --no-cpu-baseline --steps 40000 --warmup 100 > $O/bench_$w.json 2> $O/bench_$w.err
   done
   # the multi-rank launcher and the NCCL dist path at world 1 (one GPU per box)
   timeout 900 python bench.py --gpus 1 --spawn --dist --no-cpu-baseline > $O/bench_dist1.json 2> $O/bench_dist1.err
