@@ -308,8 +308,17 @@ __device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, un
 #define TLP_MINB_SMC 4   // resident CTAs for the shared-memory-coefficient kernels
 #endif
 __device__ __forceinline__ float *chunk_coef_smem() {
-    __shared__ float tlp_cw[TLP_MAXT / 32][32];
+    __shared__ __align__(16) float tlp_cw[TLP_MAXT / 32][32];
     return tlp_cw[threadIdx.x >> 5];
+}
+#ifndef TLP_PAIR_C2
+#define TLP_PAIR_C2 1
+#endif
+// Slot of lane (edge) l's coefficient in the chunk row: half-warp-major for
+// PAIR strips with two-step groups (consume_group reads a float2 per group).
+template <int G, int U>
+__device__ __forceinline__ int pair_coef_slot(int lane) {
+    return (G == 2 && U == 2 && TLP_PAIR_C2) ? (lane & 1) * 16 + (lane >> 1) : lane;
 }
 
 template <int VEC, int U, bool HASC, int G, bool CLAMP, bool SMC = false>
@@ -331,6 +340,13 @@ template <int VEC, int U, bool HASC, int G, bool GUARD, int PHASE, bool SMC = fa
 __device__ __forceinline__ void consume_group(int j, int n, int grp, const Vec<VEC> (&xv)[U],
                                               const float (&ck)[U], Vec<VEC> (&ac)[2],
                                               const float *cw = nullptr, float c_l = 0.f) {
+    // PAIR (G = 2) with the coefficients in shared memory: the chunk row is
+    // stored half-warp-major (edge p at (p & 1) * 16 + p / 2, see
+    // pair_coef_slot), so a group's U = 2 steps read one aligned float2 -- one
+    // shared-memory wavefront per two steps instead of one per step
+    constexpr bool C2 = SMC && G == 2 && U == 2 && TLP_PAIR_C2;
+    float2 c2 = make_float2(0.f, 0.f);
+    if constexpr (C2) c2 = *reinterpret_cast<const float2 *>(cw + grp * 16 + j);
 #pragma unroll
     for (int k = 0; k < U; ++k) {
         const int p = G * (j + k) + grp;
@@ -341,7 +357,8 @@ __device__ __forceinline__ void consume_group(int j, int n, int grp, const Vec<V
         if constexpr (HASC && SHC) cvs = __shfl_sync(FULL, c_l, GUARD ? min(p, n - 1) : p);
         if (!GUARD || p < n) {
             float cv = 0.f;
-            if constexpr (HASC) cv = SHC ? cvs : (SMC ? cw[p] : ck[k]);
+            if constexpr (C2) cv = k == 0 ? c2.x : c2.y;
+            else if constexpr (HASC) cv = SHC ? cvs : (SMC ? cw[p] : ck[k]);
 #pragma unroll
             for (int c = 0; c < VEC; ++c) {
                 if constexpr (HASC) ac[ch].v[c] = fmaf(cv, xv[k].v[c], ac[ch].v[c]);
@@ -556,7 +573,7 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
             }
             if constexpr (SMC) {
                 __syncwarp();  // the previous chunk's coefficients are consumed
-                cw[lane] = c_l;
+                cw[pair_coef_slot<G, U>(lane)] = c_l;
                 __syncwarp();
             }
             Vec<VEC> xa[U], xb[U];
