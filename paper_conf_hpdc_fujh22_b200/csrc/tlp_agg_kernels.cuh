@@ -58,6 +58,9 @@ constexpr unsigned FULL = 0xffffffffu;
 #ifndef TLP_MAXT
 #define TLP_MAXT 256   // threads per CTA at most (8 warps)
 #endif
+#ifndef TLP_SCHED_SMEM
+#define TLP_SCHED_SMEM 1  // scheduler loop state in shared memory (agg_body)
+#endif
 #ifndef TLP_MINB
 #define TLP_MINB 3     // register path: 3 CTAs/SM -> <= 85 registers, 24 warps/SM
 #endif
@@ -1703,6 +1706,31 @@ __device__ __forceinline__ void agg_body(const AggArgs &a) {
         }
     }
     const int W = (int)((gridDim.x * blockDim.x) >> 5);
+#if TLP_SCHED_SMEM
+    // the batch start and item index live in per-warp shared memory across
+    // the item (the register-bound kernels otherwise spill them to local
+    // memory, whose write-backs reach L2 and DRAM once per item)
+    __shared__ int tlp_sched_s[TLP_MAXT / 32][2];
+    volatile int *ss = tlp_sched_s[threadIdx.x >> 5];
+    if (lane == 0) ss[0] = wid * a.step;  // static first wave
+    __syncwarp();
+    while (ss[0] < n_items) {
+        unsigned v = 0;
+        if (a.sched == S_DYNAMIC && lane == 0) v = atomicAdd(a.ctr, (unsigned)a.step);
+        __syncwarp();
+        if (lane == 0) ss[1] = ss[0];
+        __syncwarp();
+        while (ss[1] < min(ss[0] + a.step, n_items)) {
+            do_item<VEC, OP, COEF, U, ASYNC, G>(a, ss[1], lane);
+            __syncwarp();
+            if (lane == 0) ss[1] = ss[1] + 1;
+            __syncwarp();
+        }
+        const int nt = (a.sched == S_DYNAMIC) ? W * a.step + (int)__shfl_sync(FULL, v, 0) : ss[0] + W * a.step;
+        if (lane == 0) ss[0] = nt;
+        __syncwarp();
+    }
+#else
     int t = wid * a.step;  // static first wave
     while (t < n_items) {
         // the next batch is claimed before this one is processed (its latency
@@ -1714,6 +1742,7 @@ __device__ __forceinline__ void agg_body(const AggArgs &a) {
         if (a.sched == S_DYNAMIC) t = W * a.step + (int)__shfl_sync(FULL, v, 0);
         else t += W * a.step;
     }
+#endif
     if (a.n_dests > 0) __threadfence_system();  // peer stores visible before the barrier
     if (a.sched == S_DYNAMIC && lane == 0) {
         // last warp out resets the counter: no memset launch between calls
