@@ -650,6 +650,9 @@ __device__ __forceinline__ void reduce_edges(const AggArgs &a, int64_t e0, int64
 #ifndef TLP_DEPTH_MH
 #define TLP_DEPTH_MH 16  // multi-head GAT async ring depth (its scoring pauses the issue)
 #endif
+#ifndef TLP_MH_PAIRW
+#define TLP_MH_PAIRW 1  // multi-head async pairs: weights read as float2 ahead of the wait
+#endif
 #ifndef TLP_ASYNC_PAIR
 #define TLP_ASYNC_PAIR 1  // two edges per cp.async commit group (fewer waits per edge)
 #endif
@@ -1169,8 +1172,18 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
             cp_async_commit();
             // one chunk: the rescale of the (zero) chains is the identity
             mh_chunk_scores(a, (unsigned)u0 & gp.mask, n0, H, h_lo, nh, erv, el0, er0, lane, P, M, Dn, S);
+#if TLP_MH_PAIRW
+            cp_async_wait<0>();
+            for (int j = 0; j < len; j += 2) {  // weights of edges j, j + 1 as two float2
+                const float2 wA = *reinterpret_cast<const float2 *>(pa + j);
+                const float2 wB = *reinterpret_cast<const float2 *>(pb + j);
+                mh_consume<VEC>(ring + j * 32 * VEC, wA.x, wB.x, split, ae);
+                if (j + 1 < len) mh_consume<VEC>(ring + (j + 1) * 32 * VEC, wA.y, wB.y, split, ao);
+            }
+#else
             cp_async_wait<0>();
             for (int j = 0; j < len; ++j) mh_consume<VEC>(ring + j * 32 * VEC, pa[j], pb[j], split, (j & 1) ? ao : ae);
+#endif
             __syncwarp();  // P and the ring are rewritten by the next row
 #pragma unroll
             for (int c = 0; c < VEC; ++c) acc.v[c] = ae.v[c] + ao.v[c];
@@ -1209,9 +1222,18 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
                 cp_async_x<VEC>(ring_s + 4u * wa * 32 * VEC, base, (unsigned)ua, row_bytes, gp, active && (off + ja) < len);
                 cp_async_x<VEC>(ring_s + 4u * wb * 32 * VEC, base, (unsigned)ub, row_bytes, gp, active && (off + jb) < len);
                 cp_async_commit();
+#if TLP_MH_PAIRW
+                // the pair's weights as two float2 (j is even), read ahead of the wait
+                const float2 wA = *reinterpret_cast<const float2 *>(pa + j);
+                const float2 wB = *reinterpret_cast<const float2 *>(pb + j);
+                cp_async_wait<(DD - 2) / 2>();
+                mh_consume<VEC>(ring + slot * 32 * VEC, wA.x, wB.x, split, ae);
+                if (j + 1 < n0) mh_consume<VEC>(ring + (slot + 1) * 32 * VEC, wA.y, wB.y, split, ao);
+#else
                 cp_async_wait<(DD - 2) / 2>();
                 mh_consume<VEC>(ring + slot * 32 * VEC, pa[j], pb[j], split, ae);
                 if (j + 1 < n0) mh_consume<VEC>(ring + (slot + 1) * 32 * VEC, pa[j + 1], pb[j + 1], split, ao);
+#endif
                 slot += 2;
                 if (slot == DD) slot = 0;
             }
