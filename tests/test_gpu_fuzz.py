@@ -17,7 +17,8 @@ DEV = "cuda:0"
 
 KNOBS = [{}, {"TLP_PANEL": "64"}, {"TLP_PANEL": "128"}, {"TLP_PANEL": "0"}, {"TLP_GATHER": "async"},
          {"TLP_GATHER": "reg"}, {"TLP_ROWS": "1"}, {"TLP_ROWS": "0"}, {"TLP_LAYOUT": "panel", "TLP_PANEL": "64"},
-         {"TLP_SCHED": "static"}, {"TLP_SCHED": "clc"}, {"TLP_SCHED": "clc", "TLP_ROWS": "0"}]
+         {"TLP_SCHED": "static"}, {"TLP_SCHED": "clc"}, {"TLP_SCHED": "clc", "TLP_ROWS": "0"},
+         {"TLP_ROWS": "1", "TLP_ROWS_NSI": "1"}, {"TLP_ROWS": "1", "TLP_ROWS_NSI": "2"}]
 
 
 @pytest.fixture(scope="module")
@@ -51,7 +52,7 @@ def _case(seed):
     return rp, ci, n_src, F, ld, ew, knob, dict(hub_threshold=H, hub_chunk=H // 2)
 
 
-@pytest.mark.parametrize("seed", range(32))
+@pytest.mark.parametrize("seed", range(96))
 def test_fuzz_parity_and_knob_invariance(tlp, monkeypatch, seed):
     rp, ci, n_src, F, ld, ew, knob, opts = _case(seed)
     n_dst = len(rp) - 1
