@@ -894,6 +894,9 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     a.act_param = r.act_param;
     a.heads = (int)r.heads;
     a.fh = fh;
+    a.fh_magic = (fh > 1 && r.F < (1 << 16))
+                     ? (unsigned)(((uint64_t(1) << 32) + (uint64_t)fh - 1) / (uint64_t)fh)
+                     : 0u;
     a.scratch = nullptr;
     a.md = nullptr;
     a.hub_ticket = nullptr;

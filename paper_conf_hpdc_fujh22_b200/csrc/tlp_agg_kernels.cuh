@@ -107,6 +107,7 @@ struct AggArgs {
     int act;
     float act_param;
     int heads, fh;  // OP_GATH: H heads of fh columns each (F = heads * fh)
+    unsigned fh_magic;  // OP_GATH: ceil(2^32 / fh) when F < 2^16 and fh > 1 (x / fh = umulhi(x, magic)), else 0
     int mh_nh, mh_words;  // OP_GATH: heads one strip can touch; per-warp head-block floats
     // NEXT-2 fused all-gather: when n_dests > 0 every output row is stored to
     // dests[i] + (row_offset + r) * ldy for each destination (the Y_full of every
@@ -928,6 +929,12 @@ __device__ __forceinline__ void reduce_edges_async(const AggArgs &a, int64_t e0,
 // The per-warp head block (P, M, D, S) is sized at launch for the heads a
 // strip can actually touch (a.mh_nh <= 33 for fh >= VEC; a.mh_words floats,
 // a multiple of 4), so few heads leave room for more resident CTAs.
+// x / fh for 0 <= x < F (a column index): one multiply-high by the host's
+// ceil(2^32 / fh), exact for x * fh < 2^32 (F < 2^16), instead of a signed
+// integer division sequence per row strip
+__device__ __forceinline__ int mh_div(const AggArgs &a, int x) {
+    return a.fh_magic ? (int)__umulhi((unsigned)x, a.fh_magic) : (int)((unsigned)x / (unsigned)a.fh);
+}
 __device__ __forceinline__ float *mh_warp_smem(const AggArgs &a) {
     extern __shared__ __align__(16) float tlp_smem[];
     return tlp_smem + (size_t)(threadIdx.x >> 5) * a.mh_words;
@@ -1024,10 +1031,10 @@ __device__ __forceinline__ void reduce_edges_mh(const AggArgs &a, int64_t e0, in
     const int H = a.heads, fh = a.fh;
     const int c_lo = s * 32 * VEC;
     const int c_hi = min(a.F, c_lo + 32 * VEC) - 1;
-    h_lo = c_lo / fh;
-    nh = c_hi / fh - h_lo + 1;
+    h_lo = mh_div(a, c_lo);
+    nh = mh_div(a, c_hi) - h_lo + 1;
     const int cc = active ? col : c_lo;
-    hl = cc / fh - h_lo;
+    hl = mh_div(a, cc) - h_lo;
     split = (hl + h_lo + 1) * fh - cc;                 // components in head hl
     const int hl2 = min(hl + (split < VEC ? 1 : 0), nh - 1);
     for (int hh = lane; hh < nh; hh += 32) {
@@ -1131,10 +1138,10 @@ __device__ __forceinline__ void reduce_edges_mh_async(const AggArgs &a, int64_t 
     const int H = a.heads, fh = a.fh;
     const int c_lo = s * 32 * VEC;
     const int c_hi = min(a.F, c_lo + 32 * VEC) - 1;
-    h_lo = c_lo / fh;
-    nh = c_hi / fh - h_lo + 1;
+    h_lo = mh_div(a, c_lo);
+    nh = mh_div(a, c_hi) - h_lo + 1;
     const int cc = active ? col : c_lo;
-    hl = cc / fh - h_lo;
+    hl = mh_div(a, cc) - h_lo;
     split = (hl + h_lo + 1) * fh - cc;
     const int hl2 = min(hl + (split < VEC ? 1 : 0), nh - 1);
     for (int hh = lane; hh < nh; hh += 32) {
