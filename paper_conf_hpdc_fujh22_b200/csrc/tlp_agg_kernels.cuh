@@ -307,9 +307,13 @@ __device__ __forceinline__ const float *row_ptr(const char *base, unsigned u, un
 // and the streamed-weight sums (GAT alpha mode, weighted GCN/GIN) fit 64
 // registers, i.e. 4 CTAs / 32 warps per SM like the coefficient-free sums
 // (measured: Reddit GAT 26.46 -> 24.42 ms, at 3 CTAs/SM 25.65 ms; GAT
-// backward 36.3 -> 34.4 ms).
+// backward 36.3 -> 34.4 ms).  TLP_SMEMC 2 (default since round 2, session 3)
+// keeps the chunk's coefficients in the owning lanes' registers instead and
+// shuffles each step's coefficient at consume time (no shared-memory row, no
+// per-chunk store and syncs): Reddit GAT 18.31 -> 17.92 ms per call against
+// the half-warp-major shared row (interleaved A/B); 1 keeps the shared row.
 #ifndef TLP_SMEMC
-#define TLP_SMEMC 1
+#define TLP_SMEMC 2
 #endif
 #ifndef TLP_MINB_SMC
 #define TLP_MINB_SMC 4   // resident CTAs for the shared-memory-coefficient kernels
