@@ -626,6 +626,7 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // kernel stays ahead (9.67 vs 9.82 ms).  TLP_GAT=online|alpha overrides.
     int op = r.op;
     bool gat_alpha = false;
+    bool join_pending = false;  // the GAT pre-pass ran on g->side: s waits for it before the gather
     if (r.op == OP_GAT) {
         const double budget = 0.6 * (double)g->l2_bytes;
         gat_alpha = vec == 4 && 4.0 * (double)g->n_src * (double)r.ldx > budget &&
@@ -649,11 +650,34 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
                 g->device_bytes += need;
             }
             const int64_t pb = g->n_hubs + std::max<int64_t>(1, std::min<int64_t>((g->n_dst + 7) / 8, (int64_t)g->num_sms * 16));
-            k_gat_alpha<<<(unsigned)pb, 256, 0, s>>>(g->rowptr, g->colidx, g->n_dst, r.el, r.er + g->row_offset,
-                                                     r.slope, g->hub_row, g->n_hubs, g->H, g->galpha);
+            // fork: the pre-pass (latency-bound) overlaps the repack of X
+            // (bandwidth-bound) launched next on s; joined before the gather
+            // (TLP_GAT_FORK=0: in order on s)
+            cudaStream_t sa = s;
+            bool fork = true;
+            if (const char *e = knob("TLP_GAT_FORK")) fork = atoi(e) != 0;
+            if (fork && !g->side) {
+                if (cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking) != cudaSuccess ||
+                    cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+                    cudaEventCreateWithFlags(&g->ev_join, cudaEventDisableTiming) != cudaSuccess)
+                    return cuda_error(cudaGetLastError(), "GAT pre-pass stream");
+            }
+            if (fork) {
+                cudaError_t e = cudaEventRecord(g->ev_fork, s);
+                if (e == cudaSuccess) e = cudaStreamWaitEvent(g->side, g->ev_fork, 0);
+                if (e != cudaSuccess) return cuda_error(e, "GAT pre-pass fork");
+                sa = g->side;
+                join_pending = true;
+            }
+            k_gat_alpha<<<(unsigned)pb, 256, 0, sa>>>(g->rowptr, g->colidx, g->n_dst, r.el, r.er + g->row_offset,
+                                                      r.slope, g->hub_row, g->n_hubs, g->H, g->galpha);
             g->launches += 1;
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return cuda_error(e, "k_gat_alpha launch");
+            if (fork) {
+                e = cudaEventRecord(g->ev_join, g->side);
+                if (e != cudaSuccess) return cuda_error(e, "GAT pre-pass join");
+            }
         }
         if (gat_alpha) {
             op = OP_GCN;  // Y[v] = sum_e alpha_e X[u_e]: unnormalised streamed-weight sum
@@ -976,6 +1000,10 @@ tlp_status aggregate(tlp_graph g, const AggRequest &r, cudaStream_t s) {
     // TLP_HINTS=0|1 overrides
     a.stream_hint = (panel && !spread && !async_path) ? 1 : 0;
     if (const char *e = knob("TLP_HINTS")) a.stream_hint = atoi(e) != 0;
+    if (join_pending) {
+        cudaError_t e = cudaStreamWaitEvent(s, g->ev_join, 0);
+        if (e != cudaSuccess) return cuda_error(e, "GAT pre-pass join");
+    }
     KernelFn fn = (r.op == OP_GATH) ? pick_mh(vec, async_path) : pick_kernel(path, vec, op, coef, groups);
     const int wpc = g->warps_per_cta > 0 ? std::min(g->warps_per_cta, TLP_MAXT / 32) : 8;
     const int threads = 32 * wpc;

@@ -234,6 +234,12 @@ static tlp_status dmalloc(void **p, size_t bytes, tlp_graph g) {
 static void graph_free(tlp_graph g) {
     if (!g) return;
     if (g->t) graph_free(g->t);
+    if (g->side) {
+        cudaStreamSynchronize(g->side);
+        cudaStreamDestroy(g->side);
+    }
+    if (g->ev_fork) cudaEventDestroy(g->ev_fork);
+    if (g->ev_join) cudaEventDestroy(g->ev_join);
     void *ptrs[] = {g->rowptr, g->colidx, g->ew, g->in_deg, g->out_deg, g->c_out, g->ew_both,
                     g->c_out_left, g->colidx_tag, g->tpos, g->bwd, g->proj, g->xs, g->galpha,
                     g->tasks, g->hub_row, g->hub_off, g->ctr,

@@ -59,6 +59,10 @@ struct tlp_graph_s {
     size_t proj_bytes = 0;
     float *galpha = nullptr;         // GAT edge softmax alpha_e (k_gat_alpha) [nnz]
     size_t galpha_bytes = 0;
+    // GAT alpha mode: the edge-softmax pre-pass runs on a forked side stream,
+    // concurrently with the gather-copy repack of X (created on first use)
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     int64_t tag_hist[32] = {0};      // sources per out-degree class
 
     int2 *tasks = nullptr;       // [n_tasks]
