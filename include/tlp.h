@@ -259,7 +259,12 @@ tlp_status tlp_gin_aggregate(tlp_graph g, const float *X, int64_t F,
  *   Y[v] = sum_e softmax_e(s) * X[u]      (d = 0: Y[v] = 0)
  * computed in one pass with an online (running max) softmax; scores never
  * leave registers.  el: fp32 device [n_src]; er: fp32 device
- * [row_offset+n_dst].  Edge weights are ignored. */
+ * [row_offset+n_dst].  Edge weights are ignored.
+ * When X exceeds L2 but its 64-column strips fit the call
+ * instead runs an edge-softmax pre-pass (the oracle's two-pass softmax, alpha_e
+ * in a handle-owned buffer) and the streamed-weight sum; the pre-pass runs on
+ * a side stream owned by the handle, forked from and joined back into
+ * `stream` with events, so the call stays ordered on `stream`. */
 tlp_status tlp_gat_aggregate(tlp_graph g, const float *X, int64_t F,
                              int64_t ldx, const float *el, const float *er,
                              float slope, float *Y, int64_t ldy, void *stream);
